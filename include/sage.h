@@ -1,0 +1,183 @@
+/* sage.h — C ABI of the B200-native SAGE hot path (libsage.so).
+ *
+ * SAGE = Sha, Li, Tan, "Self-adaptive Graph Traversal on GPUs", SIGMOD'21.  "P:NNN" below is
+ * line NNN of the paper text; section / algorithm / table names are given beside it.
+ *
+ * What the library computes:
+ *   frontier-driven, node-centric traversal of a plain CSR graph with no preprocessing
+ *   (P:35-38), for BFS (Alg. 1 l.1-6), integer-weight SSSP
+ *   (named at P:235) and PageRank (Alg. 1 l.26-29), with the per-iteration
+ *   neighbour expansion split at runtime into tiles (Tiled Partitioning, Alg. 2)
+ *   that are logged in device memory and consumed by a persistent kernel that every SM steals
+ *   from (Resident Tile Stealing, Alg. 3), push/pull direction switching on symmetric
+ *   graphs, and Sampling-based Reordering (§6, Alg. 4, Fig. 5).
+ *
+ * Conventions (all entry points):
+ *   * extern "C"; every function returns sage_status and never aborts the process.
+ *   * Synchronous: on return every output is complete (the call synchronises its stream).
+ *   * Pointers are host or device memory.  Inputs are detected with SAGE_F_DEVICE_PTRS; output
+ *     buffers are classified with cudaPointerGetAttributes (host pageable / pinned / device).
+ *   * Results are always in the caller's ORIGINAL vertex IDs, also after sage_reorder.
+ *   * Errors: invalid arguments -> SAGE_E_INVALID and nothing is modified; CUDA / NCCL failures
+ *     -> SAGE_E_CUDA / SAGE_E_NCCL and are sticky (the handle may then only be freed).
+ *     sage_last_error() gives a thread-local message for the last failing call.
+ *   * There is no CPU fallback: without a usable GPU every compute call returns
+ *     SAGE_E_UNSUPPORTED.
+ *   * A handle is not thread-safe; distinct handles may be used from distinct threads.
+ */
+#ifndef SAGE_H_
+#define SAGE_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct sage_graph sage_graph; /* opaque; owned by the library until sage_free */
+
+typedef enum {
+  SAGE_OK = 0,
+  SAGE_E_INVALID = 1,     /* bad argument / failed CSR validation; graph unchanged            */
+  SAGE_E_NOMEM = 2,       /* device allocation failed                                          */
+  SAGE_E_CUDA = 3,        /* CUDA runtime error (sticky)                                       */
+  SAGE_E_NCCL = 4,        /* NCCL error (sticky)                                               */
+  SAGE_E_OVERFLOW = 5,    /* a finite shortest distance is >= UINT32_MAX                       */
+  SAGE_E_UNSUPPORTED = 6  /* no GPU, or a feature not available for this graph / build        */
+} sage_status;
+
+enum {
+  SAGE_F_SYMMETRIC = 1u,   /* caller asserts the CSR is symmetric -> pull (bottom-up) steps allowed */
+  SAGE_F_DEVICE_PTRS = 2u, /* row_offsets / col_indices / weights are device pointers               */
+  SAGE_F_BORROW = 4u,      /* with DEVICE_PTRS: use the caller arrays in place (no copy); the caller
+                              keeps them alive and unmodified until sage_free                      */
+  SAGE_F_NO_VALIDATE = 8u, /* skip the validation pass of sage_load_csr                              */
+  SAGE_F_PUSH_ONLY = 16u   /* disable direction switching: every level is the paper's push
+                              expansion (Alg. 2/3).  Can also be set per call (sage_bfs_ex).     */
+};
+
+/* Multi-GPU description (1D vertex partition).  NULL in sage_csr = single GPU.  */
+typedef struct {
+  int32_t rank, world;         /* this process's rank and the number of ranks                    */
+  const void *nccl_unique_id;  /* 128-byte ncclUniqueId created by rank 0 and broadcast by the
+                                  caller (e.g. torch.distributed); required when world > 1       */
+  int64_t v_begin, v_end;      /* global vertex block [v_begin, v_end) owned by this rank; ranks
+                                  cover [0, n) contiguously in rank order                       */
+} sage_dist;
+
+/* Tile ladder used by every kernel and by the reorder's sample (Alg. 2; readings
+ * R9-R14 of DESIGN.md).  NULL = defaults.                                                      */
+typedef struct {
+  int32_t tile_cta;  /* B: largest ("CTA") tile, power of two in [8, 4096]; default 256   */
+  int32_t tile_min;  /* M: MIN_TILE_SIZE, power of two in [1, B]; default 8 (Fig. 3)        */
+  int32_t align;     /* A: tile alignment in elements: 0 = paper mode (no head fragment),
+                        else a power of two in [1, 64]; default 4 (16 B, one int4 load)          */
+  double alpha;      /* Beamer push->pull threshold: pull when arcs(F) > arcs(unvisited)/alpha; 15 */
+  double beta;       /* pull->push threshold: push when |F| < n/beta; default 18                     */
+} sage_options;
+
+/* CSR input of sage_load_csr (Fig. 1: u_offset / v arrays).                         */
+typedef struct {
+  int64_t n;                     /* GLOBAL vertex count, 0 < n < 2^31                              */
+  int64_t m;                     /* LOCAL arc count; must equal row_offsets[n_local]                */
+  const int64_t *row_offsets;    /* n_local + 1 entries, row_offsets[0] = 0, non-decreasing.
+                                    n_local = v_end - v_begin (multi-GPU) or n                     */
+  const int32_t *col_indices;    /* m entries, GLOBAL ids in [0, n); rows need not be sorted       */
+  const uint32_t *weights;       /* m entries >= 1, or NULL (SSSP then returns SAGE_E_INVALID)     */
+  uint32_t flags;                /* SAGE_F_*                                                        */
+  void *cuda_stream;             /* cudaStream_t used by every call on this graph; NULL = a stream
+                                    owned by the library                                            */
+  const sage_options *opts;      /* NULL = defaults                                                 */
+  const sage_dist *dist;         /* NULL = single GPU                                               */
+} sage_csr;
+
+/* Per-call statistics; every field is filled on SAGE_OK (SURVEY §8(d) byte model).           */
+typedef struct {
+  int32_t levels;              /* BFS levels / SSSP iterations / PR iterations executed            */
+  int32_t push_levels, pull_levels;
+  int64_t edges_traversed;     /* R1: directed = sum of out(v) over reached v; symmetric = that/2;
+                                  PageRank = iterations * m                                          */
+  int64_t arcs_inspected;      /* arcs whose target status was examined (push: all arcs of F)      */
+  int64_t vertices_expanded;   /* sum over levels of |F|                                            */
+  int64_t vertices_discovered; /* BFS: reached vertices; SSSP: improvements that entered a frontier */
+  double ms;                   /* device time of the traversal kernels (CUDA events on the graph's
+                                  stream; excludes output D2H and ID translation)                 */
+  double model_bytes;          /* algorithmic bytes of the frozen model of SURVEY §8(d)             */
+  double kernel_ms;            /* device time of the dominant (persistent) kernel alone             */
+} sage_stats;
+
+typedef struct {
+  int32_t sector_width;        /* S: node ids per sector (R17); power of two; default 8             */
+  const int32_t *candidates;   /* optional (host) list of CURRENT labels allowed to move in the
+                                  first round (Fig. 5's "only consider node-8"); NULL = all   */
+  int64_t n_candidates;
+} sage_reorder_opts;
+
+/* ---------------------------------------------------------------------------------------------
+ * sage_load_csr — load (copy or borrow) a CSR graph onto the current CUDA device and validate it
+ * ("after loading ... immediately respond to queries"; no preprocessing: no transpose, no
+ * partitioning, no reordering).  Validation (unless SAGE_F_NO_VALIDATE): row_offsets[0] = 0,
+ * non-decreasing, row_offsets[n_local] = m, 0 <= col < n, weights >= 1.  On failure *out is NULL.
+ * Multi-GPU (dist->world > 1): collective over the ranks; creates the NCCL communicator.       */
+sage_status sage_load_csr(const sage_csr *in, sage_graph **out);
+
+/* Free the handle and every library-owned device array.  NULL is a no-op.                     */
+sage_status sage_free(sage_graph *g);
+
+/* BFS from `source` (global id): level_out[v] = hop distance, -1 = unreachable (Alg. 1 l.2,
+ * P:112).  level_out has n entries (n_local multi-GPU, the rank's slice).  parent_out (nullable)
+ * receives a valid BFS-tree parent (-1 for the source and for unreachable vertices).
+ * Direction switching is used iff the graph is SAGE_F_SYMMETRIC and not SAGE_F_PUSH_ONLY.     */
+sage_status sage_bfs(sage_graph *g, int32_t source, int32_t *level_out, int32_t *parent_out,
+                     sage_stats *st);
+
+/* sage_bfs with a per-call flag word (SAGE_F_PUSH_ONLY honoured).                              */
+sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level_out, int32_t *parent_out,
+                        uint32_t call_flags, sage_stats *st);
+
+/* Integer-weight SSSP ("iteratively update neighbors' distances"; reading R4): frontier
+ * Bellman-Ford with atomicMin.  dist_out[v] = shortest distance, UINT32_MAX = unreachable.
+ * Requires weights.  A finite distance >= UINT32_MAX -> SAGE_E_OVERFLOW (dist_out unspecified). */
+sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_out, sage_stats *st);
+
+/* PageRank, push form of Alg. 1 l.26-29 over the resident all-V tile log;
+ * readings R5-R7: x0 = 1/N, x <- (1-d)/N + d*(A^T D^-1 x + dangling/N), fixed `iterations`,
+ * fp64.  rank_out has n doubles summing to 1.  damping in [0, 1), iterations >= 0.             */
+sage_status sage_pagerank(sage_graph *g, double damping, int32_t iterations, double *rank_out,
+                          sage_stats *st);
+
+/* `rounds` rounds of Sampling-based Reordering (§6; readings R17-R25): relabels the
+ * vertices in place (the CSR is rewritten, rows sorted, weights moved with their arcs) and
+ * composes the permutation; later queries still speak original ids.  Single GPU only.         */
+sage_status sage_reorder(sage_graph *g, int32_t rounds, const sage_reorder_opts *opt,
+                         sage_stats *st);
+
+/* new_id_of_old[v] = current label of original vertex v (n entries; identity before reorder). */
+sage_status sage_get_permutation(const sage_graph *g, int32_t *new_id_of_old);
+
+/* Copy the CURRENT (possibly reordered) CSR to caller buffers (host or device): off n+1,
+ * col m, w m (w may be NULL).  Used to check the relabelled graph's isomorphism.             */
+sage_status sage_get_csr(const sage_graph *g, int64_t *off_out, int32_t *col_out, uint32_t *w_out);
+
+/* Graph sizes: any pointer may be NULL.                                                        */
+sage_status sage_graph_info(const sage_graph *g, int64_t *n, int64_t *m, int64_t *n_local,
+                            int64_t *v_begin, uint32_t *flags);
+
+/* Test entry point (not part of the release ABI): the resident tile log of `count` vertices
+ * (host ids, current labels) as (vertex, offset, size, kind) quadruples, kind 0 = tile,
+ * 1 = fragment, produced by the same device classifier the traversal kernels use (Alg. 3
+ * l.2-7).  triples_out holds 4*cap int64 (host); *n_out = number of quadruples.  If cap is too
+ * small nothing is written and *n_out is the required count.                                   */
+sage_status sage_debug_export_tiles(sage_graph *g, const int32_t *vertices, int64_t count,
+                                    int64_t *quads_out, int64_t cap, int64_t *n_out);
+
+/* Thread-local message of the last failing call on this thread ("" if none).                   */
+const char *sage_last_error(void);
+
+/* Library version string.                                                                      */
+const char *sage_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SAGE_H_ */

@@ -1,0 +1,385 @@
+// common.cuh — device-side building blocks shared by the SAGE kernels (sm_100a).
+//
+// Product code (libsage.so).  Shares nothing with oracle/ (the CPU checker).
+//
+//  * Tile geometry of Tiled Partitioning (Alg. 2; §5.1; Fig. 3):
+//    a row [b, e) is split into an optional head fragment that brings b to a multiple of the
+//    alignment A (tile alignment, reading R14), q = floor(rest/B) "CTA" tiles of B
+//    elements, one tile per set bit t in B/2 .. M of the residual r = rest mod B (the binary
+//    partition of P:257, residual kept at the row end, Alg. 2 l.14-16, R12), and a tail
+//    fragment of r mod M elements (< MIN_TILE_SIZE, Alg. 2 l.32).  Closed form used by every
+//    consumer: the class-t tile of the row is [e - (r & (2t-1)), + t).
+//  * Resident tile log (Alg. 3 l.2-7): per class c (tile size B >> c) a queue.
+//    Class 0 entries are explicit (start, vertex) CTA tiles (Alg. 3's (node, offset, size));
+//    classes 1..ncls-1 and the fragment queue hold vertex ids, the offset being implied by the
+//    closed form above (4 B per entry instead of 16).
+//  * The warp-aggregated enqueue (contraction) classifies a newly filtered-in vertex into
+//    the next level's log in the same pass (expandTiles fused with filter_in).
+#pragma once
+#include <cooperative_groups.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace sage {
+
+namespace cg = cooperative_groups;
+
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int kMaxCls = 13;          // B/M <= 4096 -> at most 13 tile classes
+constexpr int kQueues = kMaxCls + 1; // + fragment queue
+constexpr int kBlock = 256;          // threads per CTA of the persistent kernels
+constexpr int kWarps = kBlock / 32;
+
+struct CtaTile {       // explicit CTA-class tile (Alg. 3's (node, offset, size) triple)
+  long long start;     // first arc index
+  int u;               // source vertex (local row index)
+  int len;             // == B
+};
+
+struct Ladder {        // tile ladder (sage_options)
+  int B, M, A;         // CTA tile, MIN_TILE_SIZE, alignment (elements; 0 = paper mode)
+  int lgB;             // log2(B)
+  int ncls;            // number of tile classes = log2(B/M) + 1 (class c has size B >> c)
+};
+
+struct Queues {        // one resident tile log (one level's, or the all-V log of PageRank)
+  CtaTile *cta;        // class 0
+  int *cls[kMaxCls];   // cls[c], 1 <= c < ncls
+  int *frag;           // fragment queue (vertex ids)
+};
+
+struct CounterSet {                      // counters of one log (rotated over 3 levels)
+  unsigned long long cnt[kQueues];       // entries per queue (index ncls = fragment queue)
+  unsigned long long tk[kQueues];        // stealing tickets per queue
+  unsigned long long nF, arcsF;          // |F| and arcs(F) of the vertices enqueued here
+  unsigned long long inspected;          // pull: arcs inspected while consuming this level
+  unsigned long long scanned;            // pull: unvisited non-isolated vertices scanned
+  unsigned long long pad[4];
+};
+
+struct LevelRec {                        // per-level record (first kMaxRec levels)
+  int dir;                               // 0 push, 1 pull
+  int pad;
+  unsigned long long nF, arcsF, inspected, scanned, discovered;
+};
+constexpr int kMaxRec = 4096;
+
+struct Ctl {                             // control block of one query (device memory)
+  CounterSet set[3];
+  unsigned long long tot_push_expanded, tot_push_arcs, tot_push_disc;
+  unsigned long long tot_pull_scanned, tot_pull_inspected, tot_pull_disc;
+  unsigned long long tot_arcs_reached;   // sum of out-degrees of reached / enqueued vertices
+  int levels, push_levels, pull_levels;
+  int status;                            // 0 ok, 1 iteration cap hit, 2 possible overflow
+  double D[3];                           // PageRank dangling mass (rotated)
+  unsigned long long tot_improved;
+  LevelRec rec[kMaxRec];
+};
+
+// ------------------------------------------------------------------------------------------
+// Loads.  col / w / off are read-only for the lifetime of every kernel -> non-coherent path,
+// streaming (no L1 allocation) for the column stream.  Data produced inside a persistent
+// kernel (queues, counters) is read through L2 (ld.cg).
+__device__ __forceinline__ int4 ld_stream4(const int *p) {
+  int4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint4 ld_stream4u(const uint32_t *p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ int ld_stream1(const int *p) {
+  int r;
+  asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint32_t ld_stream1u(const uint32_t *p) {
+  uint32_t r;
+  asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ long long ld_off(const long long *p) { return __ldg(p); }
+template <class T> __device__ __forceinline__ T ldcg(const T *p) { return __ldcg(p); }
+__device__ __forceinline__ CtaTile ldcg_tile(const CtaTile *p) {
+  longlong2 v = __ldcg(reinterpret_cast<const longlong2 *>(p));
+  CtaTile t;
+  t.start = v.x;
+  t.u = (int)(v.y & 0xffffffffll);
+  t.len = (int)(v.y >> 32);
+  return t;
+}
+__device__ __forceinline__ void st_tile(CtaTile *p, long long start, int u, int len) {
+  longlong2 v;
+  v.x = start;
+  v.y = (long long)(unsigned)u | ((long long)len << 32);
+  *reinterpret_cast<longlong2 *>(p) = v;
+}
+
+__device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31; }
+__device__ __forceinline__ unsigned lanemask_lt() {
+  unsigned m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+__device__ __forceinline__ unsigned long long shfl64(unsigned long long v, int src) {
+  return __shfl_sync(FULL, v, src);
+}
+__device__ __forceinline__ unsigned long long warp_sum64(unsigned long long v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+  return v;
+}
+__device__ __forceinline__ double warp_sumd(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+  return v;
+}
+
+// ------------------------------------------------------------------------------------------
+// Row split of Tiled Partitioning (see header comment).
+struct RowSplit {
+  long long b2;  // first element after the head fragment
+  long long q;   // number of CTA tiles
+  int r;         // residual after the CTA tiles (< B)
+  int h;         // head-fragment length (< A)
+};
+__device__ __forceinline__ RowSplit split_row(long long b, long long e, const Ladder &L) {
+  RowSplit s;
+  long long d = e - b;
+  int h = 0;
+  if (L.A > 0) {
+    h = (int)((L.A - (b & (L.A - 1))) & (L.A - 1));
+    if (h > d) h = (int)d;
+  }
+  s.h = h;
+  s.b2 = b + h;
+  long long rest = e - s.b2;
+  s.q = rest >> L.lgB;
+  s.r = (int)(rest & (L.B - 1));
+  return s;
+}
+// start of the class-t tile of a row ending at e with residual r (requires r & t)
+__device__ __forceinline__ long long class_tile_start(long long e, int r, int t) {
+  return e - (long long)(r & (2 * t - 1));
+}
+
+// ------------------------------------------------------------------------------------------
+// Warp-aggregated enqueue = expandTiles (Alg. 3 l.2-7) of the vertices filtered in by this warp.
+// Every lane of the warp must call it (convergent).  `active` lanes carry vertex v with row
+// [b, e).  Appends v's tiles to the log Q, counting in cs.  Also accumulates |F| and arcs(F).
+__device__ __forceinline__ void enqueue_warp(bool active, int v, long long b, long long e,
+                                             const Ladder &L, const Queues &Q, CounterSet *cs) {
+  const unsigned am = __ballot_sync(FULL, active);
+  if (!am) return;
+  const unsigned lane = lane_id();
+  RowSplit s{0, 0, 0, 0};
+  if (active) s = split_row(b, e, L);
+  unsigned long long deg = active ? (unsigned long long)(e - b) : 0ull;
+  deg = warp_sum64(deg);
+  if (lane == 0) {
+    atomicAdd(&cs->nF, (unsigned long long)__popc(am));
+    if (deg) atomicAdd(&cs->arcsF, deg);
+  }
+  // CTA class: cooperative write of every heavy vertex's q explicit tiles.
+  unsigned hm = __ballot_sync(FULL, active && s.q > 0);
+  while (hm) {
+    const int src = __ffs(hm) - 1;
+    hm &= hm - 1;
+    const unsigned long long q = shfl64((unsigned long long)s.q, src);
+    const long long b2 = (long long)shfl64((unsigned long long)s.b2, src);
+    const int vv = __shfl_sync(FULL, v, src);
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(&cs->cnt[0], q);
+    base = shfl64(base, 0);
+    for (unsigned long long j = lane; j < q; j += 32)
+      st_tile(Q.cta + base + j, b2 + (long long)j * L.B, vv, L.B);
+  }
+  // Sub-CTA classes: one entry per set bit of the residual.
+  const unsigned lt = lanemask_lt();
+  for (int c = 1; c < L.ncls; ++c) {
+    const int t = L.B >> c;
+    const bool mine = active && (s.r & t);
+    const unsigned cm = __ballot_sync(FULL, mine);
+    if (!cm) continue;
+    const int leader = __ffs(cm) - 1;
+    unsigned long long base = 0;
+    if ((int)lane == leader) base = atomicAdd(&cs->cnt[c], (unsigned long long)__popc(cm));
+    base = shfl64(base, leader);
+    if (mine) Q.cls[c][base + __popc(cm & lt)] = v;
+  }
+  // Fragments (head and/or tail).
+  const bool fr = active && (s.h > 0 || (s.r & (L.M - 1)) != 0);
+  const unsigned fm = __ballot_sync(FULL, fr);
+  if (fm) {
+    const int leader = __ffs(fm) - 1;
+    unsigned long long base = 0;
+    if ((int)lane == leader) base = atomicAdd(&cs->cnt[L.ncls], (unsigned long long)__popc(fm));
+    base = shfl64(base, leader);
+    if (fr) Q.frag[base + __popc(fm & lt)] = v;
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// The stealing consumer (Resident Tile Stealing, Alg. 3 l.9-17).  Every warp of the
+// persistent grid takes batches of tiles of one class from a device-wide ticket counter, so any
+// SM consumes any tile; classes are drained largest first.  A tile of t elements is covered by
+// t/VEC lanes, each holding one VEC-wide (16 B for VEC=4) coalesced load of `col` per step
+// (the paper's one-neighbour-per-thread tile, vectorised for sm_100a).  Fragments (< M) are
+// consumed by a warp scan-based gather ([30]): 32 fragment vertices per round, lane k
+// takes the k-th element of their concatenation.
+//
+// Filter policy F provides:
+//   struct Src;                                    per-source-vertex context
+//   __device__ Src src(bool valid, int u, long long b, long long e);  (b,e = row of u)
+//   template<int N> __device__ void visit(bool valid, const Src&, const int (&v)[N],
+//                                          const uint32_t (&w)[N]);   convergent (whole warp)
+//   static constexpr bool kWeights;                 load weights alongside col
+
+struct FragSmem {        // per-warp scratch of the fragment gather
+  int pre[32];
+  int hl[32];
+  long long hb[32];
+  long long tb[32];
+};
+
+template <int VEC, class F>
+__device__ __forceinline__ void consume_log(F &f, const Ladder &L, const Queues &Q,
+                                            CounterSet *cs, const long long *__restrict__ off,
+                                            const int *__restrict__ col,
+                                            const uint32_t *__restrict__ w, FragSmem *fs,
+                                            typename F::Src *fsrc) {
+  const unsigned lane = lane_id();
+  for (int c = 0; c < L.ncls; ++c) {
+    const int t = L.B >> c;
+    const unsigned long long count = ldcg(&cs->cnt[c]);
+    if (count == 0) continue;
+    const int lpt = (t / VEC) < 32 ? (t / VEC) : 32;  // lanes per tile
+    const int tps = 32 / lpt;                           // tiles per warp step
+    const int spt = (t / VEC) > 32 ? (t / (32 * VEC)) : 1;  // steps per tile
+    // batch ≈ 4 KB of column data per ticket (bounded by 4 tiles of the largest class)
+    int batch = (1024 / t);
+    if (batch < 1) batch = 1;
+    if (batch < tps) batch = tps;
+    const int sub = lane / lpt, sl = lane % lpt;
+    for (;;) {
+      unsigned long long base = 0;
+      if (lane == 0) base = atomicAdd(&cs->tk[c], (unsigned long long)batch);
+      base = shfl64(base, 0);
+      if (base >= count) break;
+      const unsigned long long end = (base + batch < count) ? base + batch : count;
+      for (unsigned long long i = base; i < end; i += tps) {
+        const unsigned long long ti = i + sub;
+        const bool valid = ti < end;
+        long long start = 0, rb = 0, re = 0;
+        int u = 0;
+        if (valid) {
+          if (c == 0) {
+            CtaTile T = ldcg_tile(Q.cta + ti);
+            start = T.start;
+            u = T.u;
+            if (F::kNeedRow) { rb = ld_off(off + u); re = ld_off(off + u + 1); }
+          } else {
+            u = ldcg(Q.cls[c] + ti);
+            rb = ld_off(off + u);
+            re = ld_off(off + u + 1);
+            RowSplit s = split_row(rb, re, L);
+            start = class_tile_start(re, s.r, t);
+          }
+        }
+        const typename F::Src sc = f.src(valid, u, rb, re);
+        for (int s = 0; s < spt; ++s) {
+          const long long pos = start + (long long)s * (32 * VEC) + (long long)sl * VEC;
+          int v[VEC];
+          uint32_t ww[VEC];
+          if constexpr (VEC == 4) {
+            int4 c4 = make_int4(0, 0, 0, 0);
+            uint4 w4 = make_uint4(0, 0, 0, 0);
+            if (valid) {
+              c4 = ld_stream4(col + pos);
+              if (F::kWeights) w4 = ld_stream4u(w + pos);
+            }
+            v[0] = c4.x; v[1] = c4.y; v[2] = c4.z; v[3] = c4.w;
+            ww[0] = w4.x; ww[1] = w4.y; ww[2] = w4.z; ww[3] = w4.w;
+          } else {
+#pragma unroll
+            for (int j = 0; j < VEC; ++j) {
+              v[j] = valid ? ld_stream1(col + pos + j) : 0;
+              ww[j] = (valid && F::kWeights) ? ld_stream1u(w + pos + j) : 0u;
+            }
+          }
+          f.template visit<VEC>(valid, sc, v, ww);
+        }
+      }
+    }
+  }
+  // ---- fragments: warp scan-based gather
+  const unsigned long long fcount = ldcg(&cs->cnt[L.ncls]);
+  if (fcount == 0) return;
+  for (;;) {
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(&cs->tk[L.ncls], 32ull);
+    base = shfl64(base, 0);
+    if (base >= fcount) break;
+    const bool valid = base + lane < fcount;
+    int u = 0, hl = 0, tl = 0;
+    long long hb = 0, tb = 0, rb = 0, re = 0;
+    if (valid) {
+      u = ldcg(Q.frag + base + lane);
+      rb = ld_off(off + u);
+      re = ld_off(off + u + 1);
+      RowSplit s = split_row(rb, re, L);
+      hb = rb;
+      hl = s.h;
+      tl = s.r & (L.M - 1);
+      tb = re - tl;
+    }
+    const typename F::Src sc = f.src(valid, u, rb, re);
+    int fl = hl + tl;
+    // inclusive warp scan of fl
+    int inc = fl;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      int y = __shfl_up_sync(FULL, inc, o);
+      if ((int)lane >= o) inc += y;
+    }
+    const int total = __shfl_sync(FULL, inc, 31);
+    fs->pre[lane] = inc - fl;
+    fs->hl[lane] = hl;
+    fs->hb[lane] = hb;
+    fs->tb[lane] = tb;
+    fsrc[lane] = sc;
+    __syncwarp();
+    for (int k0 = 0; k0 < total; k0 += 32) {
+      const int k = k0 + (int)lane;
+      const bool kv = k < total;
+      int o = 0;
+      if (kv) {   // largest o with pre[o] <= k
+        int lo = 0, hi = 31;
+        while (lo < hi) {
+          int mid = (lo + hi + 1) >> 1;
+          if (fs->pre[mid] <= k) lo = mid; else hi = mid - 1;
+        }
+        o = lo;
+      }
+      int vv[1];
+      uint32_t w1[1];
+      vv[0] = 0;
+      w1[0] = 0;
+      typename F::Src so = fsrc[o];
+      if (kv) {
+        const int idx = k - fs->pre[o];
+        const long long pos = idx < fs->hl[o] ? fs->hb[o] + idx : fs->tb[o] + (idx - fs->hl[o]);
+        vv[0] = ld_stream1(col + pos);
+        if (F::kWeights) w1[0] = ld_stream1u(w + pos);
+      }
+      f.template visit<1>(kv, so, vv, w1);
+    }
+    __syncwarp();
+  }
+}
+
+}  // namespace sage

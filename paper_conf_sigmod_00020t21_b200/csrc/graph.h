@@ -1,0 +1,76 @@
+// graph.h — host-side state of a loaded graph (the opaque sage_graph of include/sage.h).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "common.cuh"
+#include "sage.h"
+
+namespace sage {
+
+// Thread-local error message + status helpers (capi.cu).
+void set_error(const char *fmt, ...);
+void clear_error();
+
+struct DeviceBuf {          // a library-owned device allocation
+  void *p = nullptr;
+  size_t bytes = 0;
+};
+
+struct Comm;                // multi-GPU communicator (comm.cu); null on one GPU
+
+struct TraversalState {     // per-query scratch, allocated on first use and kept
+  bool ready = false;
+  int32_t *level = nullptr;       // BFS levels (int32, -1 = unvisited), n_local
+  int32_t *parent = nullptr;      // BFS parents (allocated on first parent request)
+  uint32_t *dist = nullptr;       // SSSP distances, n_local
+  uint32_t *visited = nullptr;    // visited bitmap, ceil(n/32) words (+ padding)
+  uint32_t *fb[3] = {nullptr, nullptr, nullptr};  // frontier bitmaps (rotated), pull + SSSP dedupe
+  Queues q[2];                    // double-buffered per-level tile logs
+  Ctl *ctl = nullptr;             // device control block
+  int32_t *tmp_out = nullptr;     // ID-translation scratch (n_local)
+};
+
+struct PageRankState {      // the all-V resident tile log (built once, reused)
+  bool valid = false;
+  Queues q;
+  unsigned long long cnt[kQueues] = {0};
+  int32_t *dangling = nullptr;    // vertices with out-degree 0
+  long long n_dangling = 0;
+  double *x = nullptr, *y = nullptr;
+  CounterSet *cs = nullptr;       // device copy of the log's counters (+ rotating tickets)
+};
+
+}  // namespace sage
+
+struct sage_graph {
+  int64_t n = 0;              // global vertex count
+  int64_t n_local = 0;        // rows owned here
+  int64_t v_begin = 0, v_end = 0;
+  int64_t m = 0;              // local arcs
+  uint32_t flags = 0;
+  int device = 0;
+  int num_sms = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int64_t *off = nullptr;     // device, n_local + 1
+  int32_t *col = nullptr;     // device, m
+  uint32_t *w = nullptr;      // device, m or null
+  bool own_off = false, own_col = false, own_w = false;
+  bool rows_sorted = false;
+  int64_t max_degree = 0;
+  int64_t n_isolated = 0;
+  sage::Ladder ladder{};
+  double alpha = 15.0, beta = 18.0;
+  int vec = 4;                // 4 = int4 column loads, 1 = scalar (paper mode / unaligned)
+  // reordering: sigma[v_orig] = current label; sigma_inv[label] = v_orig (null = identity)
+  int32_t *sigma = nullptr, *sigma_inv = nullptr;
+  bool reordered = false;
+  int sticky = 0;             // sticky SAGE_E_CUDA / SAGE_E_NCCL
+  sage::TraversalState ts;
+  sage::PageRankState pr;
+  sage::Comm *comm = nullptr;
+  int grid_bfs = 0, grid_sssp = 0, grid_pr = 0;   // persistent grid sizes (cooperative)
+};

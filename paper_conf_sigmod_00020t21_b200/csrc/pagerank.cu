@@ -1,0 +1,264 @@
+// pagerank.cu — PageRank as SAGE's "global traversal": the frontier is all of V every
+// iteration, so the all-V tile log is built ONCE by Tiled Partitioning and kept resident in
+// device memory (the scheduling log reused on revisits; reading R15), then consumed
+// by the stealing persistent kernel every iteration.
+//
+// Filter = push form of Alg. 1 l.26-29: every arc u->v adds x_u / out(u) into y_v
+// with an fp64 atomic (red.global.add.f64; reading R7: fp32 atomics miss the 1e-6 bar).
+// Readings R5/R6: x0 = 1/N; per iteration D = sum of x over dangling vertices,
+// x_v <- (1-d)/N + d*(y_v + D/N); fixed number of iterations.
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include "common.cuh"
+#include "graph.h"
+#include "internal.h"
+
+namespace sage {
+
+struct PrPush {
+  struct Src {
+    double c;
+  };
+  static constexpr bool kWeights = false;
+  static constexpr bool kNeedRow = true;
+  const double *x;
+  double *y;
+
+  __device__ __forceinline__ Src src(bool valid, int u, long long b, long long e) const {
+    // x is rewritten by the finalize phase of the previous iteration: read through L2
+    return Src{(valid && e > b) ? ldcg(x + u) / (double)(e - b) : 0.0};
+  }
+  template <int N>
+  __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
+                                        const uint32_t (&)[N]) const {
+    if (!valid) return;
+#pragma unroll
+    for (int j = 0; j < N; ++j) atomicAdd(y + v[j], s.c);
+  }
+};
+
+struct PrArgs {
+  const long long *off;
+  const int *col;
+  long long n;        // rows here
+  double N;           // global vertex count
+  double d;
+  int iters;
+  Ladder L;
+  Queues q;
+  CounterSet *sets;   // 3 rotating copies of the log's counters (tickets reset each iteration)
+  const int *dangling;
+  long long n_dangling;
+  double *x, *y;
+  Ctl *ctl;
+};
+
+// Build the all-V resident log: one thread per vertex, warp-aggregated classification.
+__global__ void k_build_log(const long long *__restrict__ off, long long n, Ladder L, Queues Q,
+                            CounterSet *cs, int *dangling, unsigned long long *n_dangling) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  const long long nthr = ((n + 31) / 32) * 32;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nthr; i += stride) {
+    const bool in = i < n;
+    long long b = 0, e = 0;
+    if (in) {
+      b = off[i];
+      e = off[i + 1];
+    }
+    const bool act = in && e > b;
+    enqueue_warp(act, (int)i, b, e, L, Q, cs);
+    const bool dg = in && e == b;
+    const unsigned dm = __ballot_sync(FULL, dg);
+    if (dm) {
+      const int leader = __ffs(dm) - 1;
+      unsigned long long base = 0;
+      if ((int)lane_id() == leader) base = atomicAdd(n_dangling, (unsigned long long)__popc(dm));
+      base = shfl64(base, leader);
+      if (dg) dangling[base + __popc(dm & lanemask_lt())] = (int)i;
+    }
+  }
+}
+
+__global__ void k_pr_init(double *x, double *y, long long n, double v0) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+    x[i] = v0;
+    y[i] = 0.0;
+  }
+}
+
+template <int VEC>
+__global__ void __launch_bounds__(kBlock) k_pagerank(PrArgs a) {
+  cg::grid_group grid = cg::this_grid();
+  __shared__ FragSmem fsm[kWarps];
+  __shared__ PrPush::Src fsrc[kWarps][32];
+  __shared__ double red[kWarps];
+  const int warp = threadIdx.x >> 5;
+  const unsigned lane = lane_id();
+  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  const double base = (1.0 - a.d) / a.N;
+  for (int it = 0; it < a.iters; ++it) {
+    CounterSet *cs = &a.sets[it % 3];
+    __syncthreads();
+    if (blockIdx.x == 0 && threadIdx.x < kQueues) a.sets[(it + 2) % 3].tk[threadIdx.x] = 0ull;
+    if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->D[(it + 2) % 3] = 0.0;
+    // push phase over the resident log
+    PrPush f;
+    f.x = a.x;
+    f.y = a.y;
+    consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &fsm[warp], fsrc[warp]);
+    // dangling mass of this iteration's x
+    double dsum = 0.0;
+    for (long long i = tid; i < a.n_dangling; i += stride) dsum += ldcg(a.x + a.dangling[i]);
+    dsum = warp_sumd(dsum);
+    if (lane == 0) red[warp] = dsum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      double s = 0.0;
+      for (int k = 0; k < kWarps; ++k) s += red[k];
+      if (s != 0.0) atomicAdd(&a.ctl->D[it % 3], s);
+    }
+    grid.sync();
+    // finalize: x = (1-d)/N + d*(y + D/N); y = 0
+    const double D = ldcg(&a.ctl->D[it % 3]);
+    const double add = base + a.d * D / a.N;
+    for (long long v = tid; v < a.n; v += stride) {
+      const double yv = ldcg(a.y + v);
+      a.x[v] = add + a.d * yv;
+      a.y[v] = 0.0;
+    }
+    grid.sync();
+  }
+}
+
+void free_pagerank_state(sage_graph *g) {
+  PageRankState &p = g->pr;
+  free_queues(g, &p.q);
+  dfree(g, p.dangling);
+  dfree(g, p.x);
+  dfree(g, p.y);
+  dfree(g, p.cs);
+  p = PageRankState();
+}
+
+sage_status ensure_pagerank_log(sage_graph *g) {
+  PageRankState &p = g->pr;
+  if (p.valid) return SAGE_OK;
+  sage_status s;
+  const long long n = g->n_local;
+  if (!p.x) {
+    if ((s = dalloc(g, (void **)&p.x, sizeof(double) * (size_t)n)) != SAGE_OK ||
+        (s = dalloc(g, (void **)&p.y, sizeof(double) * (size_t)n)) != SAGE_OK ||
+        (s = dalloc(g, (void **)&p.cs, sizeof(CounterSet) * 3 + 64)) != SAGE_OK) {
+      free_pagerank_state(g);
+      return s;
+    }
+  }
+  if ((s = alloc_queues(g, &p.q, n, g->m)) != SAGE_OK ||
+      (s = dalloc(g, (void **)&p.dangling, sizeof(int) * (size_t)(n + 1))) != SAGE_OK) {
+    free_pagerank_state(g);
+    return s;
+  }
+  unsigned long long *nd = reinterpret_cast<unsigned long long *>(p.cs + 3);
+  cudaMemsetAsync(p.cs, 0, sizeof(CounterSet) * 3 + 64, g->stream);
+  k_build_log<<<g->num_sms * 8, 256, 0, g->stream>>>((const long long *)g->off, n, g->ladder,
+                                                     p.q, p.cs, p.dangling, nd);
+  // replicate the counts into the two other rotating sets
+  cudaMemcpyAsync(p.cs + 1, p.cs, sizeof(CounterSet), cudaMemcpyDeviceToDevice, g->stream);
+  cudaMemcpyAsync(p.cs + 2, p.cs, sizeof(CounterSet), cudaMemcpyDeviceToDevice, g->stream);
+  CounterSet h;
+  unsigned long long hnd = 0;
+  cudaMemcpyAsync(&h, p.cs, sizeof(h), cudaMemcpyDeviceToHost, g->stream);
+  cudaMemcpyAsync(&hnd, nd, sizeof(hnd), cudaMemcpyDeviceToHost, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "PageRank log build");
+  memcpy(p.cnt, h.cnt, sizeof(p.cnt));
+  p.n_dangling = (long long)hnd;
+  p.valid = true;
+  return SAGE_OK;
+}
+
+sage_status run_pagerank_multi(sage_graph *g, double damping, int32_t iterations, double *rank_out,
+                               sage_stats *st);
+
+}  // namespace sage
+
+using namespace sage;
+
+extern "C" sage_status sage_pagerank(sage_graph *g, double damping, int32_t iterations,
+                                     double *rank_out, sage_stats *st) {
+  clear_error();
+  if (!g || !rank_out) {
+    set_error("null argument");
+    return SAGE_E_INVALID;
+  }
+  if (g->sticky) return (sage_status)g->sticky;
+  if (!(damping >= 0.0 && damping < 1.0) || iterations < 0) {
+    set_error("damping must be in [0, 1) and iterations >= 0");
+    return SAGE_E_INVALID;
+  }
+  if (g->comm) return run_pagerank_multi(g, damping, iterations, rank_out, st);
+  sage_status s;
+  if ((s = ensure_traversal_state(g)) != SAGE_OK) return s;
+  cudaEvent_t e0, e1, e2;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  cudaEventCreate(&e2);
+  cudaEventRecord(e0, g->stream);
+  if ((s = ensure_pagerank_log(g)) != SAGE_OK) return s;
+  PageRankState &p = g->pr;
+  k_pr_init<<<g->num_sms * 8, 256, 0, g->stream>>>(p.x, p.y, g->n_local, 1.0 / (double)g->n);
+  cudaMemsetAsync(g->ts.ctl, 0, offsetof(Ctl, rec), g->stream);
+  for (int i = 0; i < 3; ++i)   // fresh stealing tickets for every call
+    cudaMemsetAsync(&p.cs[i].tk, 0, sizeof(p.cs[i].tk), g->stream);
+  cudaEventRecord(e1, g->stream);
+  PrArgs a;
+  memset(&a, 0, sizeof(a));
+  a.off = (const long long *)g->off;
+  a.col = g->col;
+  a.n = g->n_local;
+  a.N = (double)g->n;
+  a.d = damping;
+  a.iters = iterations;
+  a.L = g->ladder;
+  a.q = p.q;
+  a.sets = p.cs;
+  a.dangling = p.dangling;
+  a.n_dangling = p.n_dangling;
+  a.x = p.x;
+  a.y = p.y;
+  a.ctl = g->ts.ctl;
+  if (iterations > 0) {
+    const void *fn = g->vec == 4 ? (const void *)k_pagerank<4> : (const void *)k_pagerank<1>;
+    const int grid = coop_grid(g, fn, &g->grid_pr);
+    void *args[] = {&a};
+    if ((s = launch_coop(g, fn, grid, args, "PageRank kernel")) != SAGE_OK) return s;
+  }
+  cudaEventRecord(e2, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "PageRank");
+  float ms = 0, kms = 0;
+  cudaEventElapsedTime(&ms, e0, e2);
+  cudaEventElapsedTime(&kms, e1, e2);
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaEventDestroy(e2);
+  if (st) {
+    memset(st, 0, sizeof(*st));
+    st->levels = iterations;
+    st->push_levels = iterations;
+    st->edges_traversed = (int64_t)iterations * g->m;
+    st->arcs_inspected = (int64_t)iterations * g->m;
+    st->vertices_expanded = (int64_t)iterations * (g->n_local - p.n_dangling);
+    st->ms = ms;
+    st->kernel_ms = kms;
+    // 40 B per vertex + 12 B per arc, per iteration
+    st->model_bytes = (double)iterations * (40.0 * (double)g->n_local + 12.0 * (double)g->m);
+  }
+  if ((s = translate_out_f64(g, p.x, rank_out)) != SAGE_OK) return s;
+  e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "PageRank output");
+  return SAGE_OK;
+}

@@ -1,0 +1,876 @@
+// traversal.cu — BFS and SSSP: the node-centric pipeline of SAGE (§4; Fig. 2) as ONE
+// persistent cooperative kernel per query.
+//
+// Per level L (all in the same launch, one grid-wide barrier per level):
+//   push : the stealing consumer (Resident Tile Stealing, Alg. 3) drains level L's tile log
+//          (built by Tiled Partitioning, Alg. 2) and applies the filter (Alg. 1) to every
+//          neighbour; filtered-in vertices are classified into level L+1's log in the same
+//          pass (warp-aggregated expandTiles + contraction).
+//   pull : (symmetric graphs, not in the paper; north_star) each unvisited vertex scans its
+//          row until it meets a vertex of the frontier bitmap.
+//   barrier; every CTA reads the same counters and takes the same decision: stop (empty
+//   frontier), continue, and the Beamer direction for the next level.
+// BFS filter (Alg. 1 l.1-6): visited-bitmap test-and-set, level := L+1.  The paper's
+// non-atomic "dirty writes" are replaced by an atomicOr claim so every vertex enters
+// the next log exactly once (reading R3); levels are identical.
+// SSSP filter (reading R4): nd = dist[u] + w; atomicMin; improved vertices enter the next
+// log once per iteration (bitmap dedupe) -> frontier Bellman-Ford.
+#include <cuda_runtime.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+
+#include "common.cuh"
+#include "graph.h"
+#include "internal.h"
+
+namespace sage {
+
+// ============================================================================ filters
+struct BfsPush {
+  struct Src {
+    int u;
+  };
+  static constexpr bool kWeights = false;
+  static constexpr bool kNeedRow = false;
+  uint32_t *visited;
+  int *level;
+  int *parent;
+  uint32_t *fb_next;   // next-frontier bitmap (only when direction switching is enabled)
+  int next_level;
+  int v_base;          // global id of local row 0 (0 on one GPU)
+  const long long *off;
+  Ladder L;
+  Queues Qn;
+  CounterSet *csn;
+
+  __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
+
+  template <int N>
+  __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
+                                        const uint32_t (&)[N]) const {
+    bool disc[N];
+    uint32_t wd[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) wd[j] = valid ? visited[v[j] >> 5] : 0xffffffffu;
+    bool anyd = false;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const uint32_t bit = 1u << (v[j] & 31);
+      disc[j] = false;
+      if (!(wd[j] & bit)) {
+        const uint32_t old = atomicOr(visited + (v[j] >> 5), bit);
+        disc[j] = !(old & bit);
+      }
+      anyd |= disc[j];
+    }
+    if (!__any_sync(FULL, anyd)) return;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      long long b = 0, e = 0;
+      if (disc[j]) {
+        level[v[j]] = next_level;
+        if (parent) parent[v[j]] = s.u + v_base;
+        if (fb_next) atomicOr(fb_next + (v[j] >> 5), 1u << (v[j] & 31));
+        b = ld_off(off + v[j]);
+        e = ld_off(off + v[j] + 1);
+      }
+      enqueue_warp(disc[j], v[j], b, e, L, Qn, csn);
+    }
+  }
+};
+
+struct SsspPush {
+  struct Src {
+    uint32_t du;
+  };
+  static constexpr bool kWeights = true;
+  static constexpr bool kNeedRow = false;
+  uint32_t *dist;
+  uint32_t *inq_next;   // dedupe bitmap of the next frontier
+  int *overflow;
+  const long long *off;
+  Ladder L;
+  Queues Qn;
+  CounterSet *csn;
+
+  __device__ __forceinline__ Src src(bool valid, int u, long long, long long) const {
+    // dist[u] may have been lowered by another SM in an earlier iteration: read through L2
+    return Src{valid ? ldcg(dist + u) : 0xffffffffu};
+  }
+
+  template <int N>
+  __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
+                                        const uint32_t (&w)[N]) const {
+    bool enq[N];
+    bool anye = false;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      enq[j] = false;
+      if (valid) {
+        const unsigned long long nd = (unsigned long long)s.du + w[j];
+        if (nd >= 0xffffffffull) {
+          *overflow = 1;     // possible overflow: resolved exactly after the traversal
+        } else {
+          const uint32_t cur = dist[v[j]];
+          if ((uint32_t)nd < cur) {
+            const uint32_t old = atomicMin(dist + v[j], (uint32_t)nd);
+            if ((uint32_t)nd < old) {
+              const uint32_t bit = 1u << (v[j] & 31);
+              const uint32_t o2 = atomicOr(inq_next + (v[j] >> 5), bit);
+              enq[j] = !(o2 & bit);
+            }
+          }
+        }
+      }
+      anye |= enq[j];
+    }
+    if (!__any_sync(FULL, anye)) return;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      long long b = 0, e = 0;
+      if (enq[j]) {
+        b = ld_off(off + v[j]);
+        e = ld_off(off + v[j] + 1);
+      }
+      enqueue_warp(enq[j], v[j], b, e, L, Qn, csn);
+    }
+  }
+};
+
+// ============================================================================ kernel args
+struct TravArgs {
+  const long long *off;
+  const int *col;
+  const uint32_t *w;
+  long long n;          // local rows (== global n on one GPU)
+  long long m;
+  Ladder L;
+  Queues q[2];
+  uint32_t *fb[3];
+  uint32_t *visited;
+  int *level;
+  int *parent;
+  uint32_t *dist;
+  Ctl *ctl;
+  int do_enabled;       // direction switching allowed
+  double alpha, beta;
+  int max_levels;
+};
+
+// Pull (bottom-up) step over the visited bitmap: one warp per 32-vertex word.
+__device__ __forceinline__ void pull_level(const TravArgs &a, int next_level, const uint32_t *fbc,
+                                           uint32_t *fbn, const Queues &Qn, CounterSet *cur,
+                                           CounterSet *nxt) {
+  const unsigned lane = lane_id();
+  const long long nwords = (a.n + 31) >> 5;
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  unsigned long long insp = 0, scanned = 0;
+  for (long long wd = gw; wd < nwords; wd += nw) {
+    const long long v = (wd << 5) + lane;
+    const uint32_t vis = ldcg(a.visited + wd);
+    const bool todo = v < a.n && !((vis >> lane) & 1u);
+    long long b = 0, e = 0;
+    bool found = false;
+    int par = -1;
+    if (todo) {
+      b = ld_off(a.off + v);
+      e = ld_off(a.off + v + 1);
+      if (e > b) scanned++;
+      for (long long k = b; k < e; ++k) {
+        const int u = ld_stream1(a.col + k);
+        ++insp;
+        if ((ldcg(fbc + (u >> 5)) >> (u & 31)) & 1u) {
+          found = true;
+          par = u;
+          break;
+        }
+      }
+    }
+    const unsigned fm = __ballot_sync(FULL, found);
+    if (fm) {
+      if (lane == 0) {
+        a.visited[wd] = vis | fm;
+        fbn[wd] = fm;
+      }
+      if (found) {
+        a.level[v] = next_level;
+        if (a.parent) a.parent[v] = par;
+      }
+    }
+    enqueue_warp(found, (int)v, b, e, a.L, Qn, nxt);
+  }
+  insp = warp_sum64(insp);
+  scanned = warp_sum64(scanned);
+  if (lane == 0) {
+    if (insp) atomicAdd(&cur->inspected, insp);
+    if (scanned) atomicAdd(&cur->scanned, scanned);
+  }
+}
+
+__device__ __forceinline__ void zero_counterset(CounterSet *s) {
+  constexpr int words = sizeof(CounterSet) / 8;
+  if (blockIdx.x == 0 && threadIdx.x < words)
+    reinterpret_cast<unsigned long long *>(s)[threadIdx.x] = 0ull;
+}
+
+__device__ __forceinline__ void clear_words(uint32_t *p, long long nwords) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nwords; i += stride)
+    p[i] = 0u;
+}
+
+// Record level L's statistics (single thread).
+__device__ __forceinline__ void record_level(Ctl *ctl, int L, int dir, const CounterSet *cur,
+                                             const CounterSet *nxt) {
+  const unsigned long long nF = ldcg(&cur->nF), aF = ldcg(&cur->arcsF);
+  const unsigned long long disc = ldcg(&nxt->nF), aN = ldcg(&nxt->arcsF);
+  const unsigned long long insp = ldcg(&cur->inspected), sc = ldcg(&cur->scanned);
+  if (dir == 0) {
+    ctl->tot_push_expanded += nF;
+    ctl->tot_push_arcs += aF;
+    ctl->tot_push_disc += disc;
+    ctl->push_levels++;
+  } else {
+    ctl->tot_pull_scanned += sc;
+    ctl->tot_pull_inspected += insp;
+    ctl->tot_pull_disc += disc;
+    ctl->pull_levels++;
+  }
+  ctl->tot_arcs_reached += aN;
+  ctl->tot_improved += disc;
+  if (L < kMaxRec) {
+    LevelRec &r = ctl->rec[L];
+    r.dir = dir;
+    r.nF = nF;
+    r.arcsF = aF;
+    r.inspected = dir == 0 ? aF : insp;
+    r.scanned = sc;
+    r.discovered = disc;
+  }
+  ctl->levels = L + 1;
+}
+
+// ============================================================================ BFS kernel
+template <int VEC>
+__global__ void __launch_bounds__(kBlock) k_bfs(TravArgs a) {
+  cg::grid_group grid = cg::this_grid();
+  __shared__ FragSmem fsm[kWarps];
+  __shared__ BfsPush::Src fsrc[kWarps][32];
+  const int warp = threadIdx.x >> 5;
+  Ctl *ctl = a.ctl;
+  double mU = (double)a.m - (double)ldcg(&ctl->set[0].arcsF);
+  int dir = 0;
+  unsigned long long prev_nF = 1;
+  const long long nwords = (a.n + 31) >> 5;
+  for (int L = 0;; ++L) {
+    CounterSet *cur = &ctl->set[L % 3];
+    CounterSet *nxt = &ctl->set[(L + 1) % 3];
+    __syncthreads();   // block 0: record_level(L-1) finished before set (L+2)%3 is zeroed
+    zero_counterset(&ctl->set[(L + 2) % 3]);
+    uint32_t *fbc = a.fb[L % 3], *fbn = a.fb[(L + 1) % 3];
+    if (a.do_enabled) clear_words(a.fb[(L + 2) % 3], nwords);
+    if (dir == 0) {
+      BfsPush f;
+      f.visited = a.visited;
+      f.level = a.level;
+      f.parent = a.parent;
+      f.fb_next = a.do_enabled ? fbn : nullptr;
+      f.next_level = L + 1;
+      f.v_base = 0;
+      f.off = a.off;
+      f.L = a.L;
+      f.Qn = a.q[(L + 1) & 1];
+      f.csn = nxt;
+      consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &fsm[warp], fsrc[warp]);
+    } else {
+      pull_level(a, L + 1, fbc, fbn, a.q[(L + 1) & 1], cur, nxt);
+    }
+    grid.sync();
+    const unsigned long long nF = ldcg(&nxt->nF);
+    const unsigned long long aF = ldcg(&nxt->arcsF);
+    if (blockIdx.x == 0 && threadIdx.x == 0) record_level(ctl, L, dir, cur, nxt);
+    if (nF == 0) break;
+    if (L + 1 >= a.max_levels) {
+      if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = 1;
+      break;
+    }
+    mU -= (double)aF;
+    if (a.do_enabled) {
+      if (dir == 0) {
+        if ((double)aF > mU / a.alpha) dir = 1;
+      } else {
+        if (!(nF >= prev_nF || (double)nF > (double)a.n / a.beta)) dir = 0;
+      }
+    }
+    prev_nF = nF;
+  }
+}
+
+// ============================================================================ SSSP kernel
+template <int VEC>
+__global__ void __launch_bounds__(kBlock) k_sssp(TravArgs a, int *overflow) {
+  cg::grid_group grid = cg::this_grid();
+  __shared__ FragSmem fsm[kWarps];
+  __shared__ SsspPush::Src fsrc[kWarps][32];
+  const int warp = threadIdx.x >> 5;
+  Ctl *ctl = a.ctl;
+  const long long nwords = (a.n + 31) >> 5;
+  for (int L = 0;; ++L) {
+    CounterSet *cur = &ctl->set[L % 3];
+    CounterSet *nxt = &ctl->set[(L + 1) % 3];
+    __syncthreads();   // block 0: record_level(L-1) finished before set (L+2)%3 is zeroed
+    zero_counterset(&ctl->set[(L + 2) % 3]);
+    clear_words(a.fb[(L + 2) % 3], nwords);
+    SsspPush f;
+    f.dist = a.dist;
+    f.inq_next = a.fb[(L + 1) % 3];
+    f.overflow = overflow;
+    f.off = a.off;
+    f.L = a.L;
+    f.Qn = a.q[(L + 1) & 1];
+    f.csn = nxt;
+    consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &fsm[warp], fsrc[warp]);
+    grid.sync();
+    const unsigned long long nF = ldcg(&nxt->nF);
+    if (blockIdx.x == 0 && threadIdx.x == 0) record_level(ctl, L, 0, cur, nxt);
+    if (nF == 0) break;
+    if (L + 1 >= a.max_levels) {
+      if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = 1;
+      break;
+    }
+  }
+}
+
+// Seed the level-0 log with the source (one warp).
+__global__ void k_seed(TravArgs a, int src, int mode /*0 bfs, 1 sssp*/) {
+  const bool act = threadIdx.x == 0;
+  long long b = 0, e = 0;
+  if (act) {
+    b = a.off[src];
+    e = a.off[src + 1];
+    a.visited[src >> 5] |= 1u << (src & 31);
+    a.fb[0][src >> 5] |= 1u << (src & 31);
+    if (mode == 0) a.level[src] = 0;
+    else a.dist[src] = 0u;
+  }
+  enqueue_warp(act, src, b, e, a.L, a.q[0], &a.ctl->set[0]);
+}
+
+// SSSP overflow resolution: a finite distance >= UINT32_MAX exists iff some arc leaves a reached
+// vertex towards an unreached one.
+__global__ void k_overflow_check(const long long *__restrict__ off, const int *__restrict__ col,
+                                 const uint32_t *__restrict__ dist, long long n, int *found) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long u = (long long)blockIdx.x * blockDim.x + threadIdx.x; u < n; u += stride) {
+    if (dist[u] == 0xffffffffu) continue;
+    for (long long k = off[u]; k < off[u + 1]; ++k)
+      if (dist[col[k]] == 0xffffffffu) {
+        *found = 1;
+        return;
+      }
+  }
+}
+
+// R1 edge count of an SSSP result: sum of out-degrees of the reached vertices.
+__global__ void k_reached_arcs(const long long *__restrict__ off, const uint32_t *__restrict__ dist,
+                               long long n, unsigned long long *out) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  unsigned long long s = 0;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+    if (dist[v] != 0xffffffffu) s += (unsigned long long)(off[v + 1] - off[v]);
+  s = warp_sum64(s);
+  if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, s);
+}
+
+__global__ void k_gather_i32(const int32_t *__restrict__ src, const int32_t *__restrict__ sigma,
+                             const int32_t *__restrict__ sigma_inv, int32_t *__restrict__ dst,
+                             long long n, int map_values) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+    int32_t x = src[sigma[v]];
+    if (map_values && x >= 0) x = sigma_inv[x];
+    dst[v] = x;
+  }
+}
+__global__ void k_gather_u32(const uint32_t *__restrict__ src, const int32_t *__restrict__ sigma,
+                             uint32_t *__restrict__ dst, long long n) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+    dst[v] = src[sigma[v]];
+}
+__global__ void k_gather_f64(const double *__restrict__ src, const int32_t *__restrict__ sigma,
+                             double *__restrict__ dst, long long n) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+    dst[v] = src[sigma[v]];
+}
+__global__ void k_iota(int32_t *p, long long n) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+    p[v] = (int32_t)v;
+}
+
+// Debug export of the tile log of a vertex set (sage_debug_export_tiles).
+__global__ void k_classify_list(const long long *__restrict__ off, const int *__restrict__ verts,
+                                long long count, Ladder L, Queues Q, CounterSet *cs) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  const long long nthr = ((count + 31) / 32) * 32;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nthr; i += stride) {
+    const bool act = i < count;
+    int v = 0;
+    long long b = 0, e = 0;
+    if (act) {
+      v = verts[i];
+      b = off[v];
+      e = off[v + 1];
+    }
+    enqueue_warp(act, v, b, e, L, Q, cs);
+  }
+}
+__global__ void k_expand_log(const long long *__restrict__ off, Ladder L, Queues Q,
+                             const CounterSet *cs, long long *quads, unsigned long long *nq,
+                             long long cap) {
+  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  auto emit = [&](long long u, long long o, long long s, long long kind) {
+    unsigned long long k = atomicAdd(nq, 1ull);
+    if ((long long)k < cap) {
+      quads[4 * k] = u;
+      quads[4 * k + 1] = o;
+      quads[4 * k + 2] = s;
+      quads[4 * k + 3] = kind;
+    }
+  };
+  for (long long i = tid; i < (long long)cs->cnt[0]; i += stride) {
+    CtaTile T = Q.cta[i];
+    emit(T.u, T.start, T.len, 0);
+  }
+  for (int c = 1; c < L.ncls; ++c) {
+    const int t = L.B >> c;
+    for (long long i = tid; i < (long long)cs->cnt[c]; i += stride) {
+      const int u = Q.cls[c][i];
+      const long long b = off[u], e = off[u + 1];
+      RowSplit s = split_row(b, e, L);
+      emit(u, class_tile_start(e, s.r, t), t, 0);
+    }
+  }
+  for (long long i = tid; i < (long long)cs->cnt[L.ncls]; i += stride) {
+    const int u = Q.frag[i];
+    const long long b = off[u], e = off[u + 1];
+    RowSplit s = split_row(b, e, L);
+    if (s.h > 0) emit(u, b, s.h, 1);
+    const int tl = s.r & (L.M - 1);
+    if (tl > 0) emit(u, e - tl, tl, 1);
+  }
+}
+
+// ============================================================================ host side
+void iota_device(sage_graph *g, int32_t *p, int64_t n) {
+  k_iota<<<g->num_sms * 4, 256, 0, g->stream>>>(p, n);
+}
+
+sage_status alloc_queues(sage_graph *g, Queues *q, long long n_rows, long long m) {
+  memset(q, 0, sizeof(*q));
+  sage_status st;
+  const long long cta_cap = m / g->ladder.B + 1;
+  if ((st = dalloc(g, (void **)&q->cta, sizeof(CtaTile) * (size_t)cta_cap)) != SAGE_OK) return st;
+  for (int c = 1; c < g->ladder.ncls; ++c)
+    if ((st = dalloc(g, (void **)&q->cls[c], sizeof(int) * (size_t)(n_rows + 1))) != SAGE_OK)
+      return st;
+  if ((st = dalloc(g, (void **)&q->frag, sizeof(int) * (size_t)(n_rows + 1))) != SAGE_OK) return st;
+  return SAGE_OK;
+}
+void free_queues(sage_graph *g, Queues *q) {
+  dfree(g, q->cta);
+  for (int c = 0; c < kMaxCls; ++c) dfree(g, q->cls[c]);
+  dfree(g, q->frag);
+  memset(q, 0, sizeof(*q));
+}
+
+void free_traversal_state(sage_graph *g) {
+  TraversalState &t = g->ts;
+  dfree(g, t.level);
+  dfree(g, t.parent);
+  dfree(g, t.dist);
+  dfree(g, t.visited);
+  for (int i = 0; i < 3; ++i) dfree(g, t.fb[i]);
+  free_queues(g, &t.q[0]);
+  free_queues(g, &t.q[1]);
+  dfree(g, t.ctl);
+  dfree(g, t.tmp_out);
+  t = TraversalState();
+}
+
+sage_status ensure_traversal_state(sage_graph *g) {
+  TraversalState &t = g->ts;
+  if (t.ready) return SAGE_OK;
+  const long long n = g->n_local;
+  const size_t words = (size_t)((g->n + 31) / 32 + 8);
+  sage_status st;
+  if ((st = dalloc(g, (void **)&t.level, sizeof(int32_t) * (size_t)n)) != SAGE_OK ||
+      (st = dalloc(g, (void **)&t.visited, sizeof(uint32_t) * words)) != SAGE_OK ||
+      (st = dalloc(g, (void **)&t.ctl, sizeof(Ctl))) != SAGE_OK ||
+      (st = dalloc(g, (void **)&t.tmp_out, sizeof(int64_t) * (size_t)n)) != SAGE_OK) {
+    free_traversal_state(g);
+    return st;
+  }
+  for (int i = 0; i < 3; ++i)
+    if ((st = dalloc(g, (void **)&t.fb[i], sizeof(uint32_t) * words)) != SAGE_OK) {
+      free_traversal_state(g);
+      return st;
+    }
+  for (int i = 0; i < 2; ++i)
+    if ((st = alloc_queues(g, &t.q[i], n, g->m)) != SAGE_OK) {
+      free_traversal_state(g);
+      return st;
+    }
+  t.ready = true;
+  return SAGE_OK;
+}
+
+int coop_grid(sage_graph *g, const void *fn, int *cache) {
+  if (*cache) return *cache;
+  int nb = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, kBlock, 0);
+  if (nb < 1) nb = 1;
+  *cache = nb * g->num_sms;
+  return *cache;
+}
+
+sage_status launch_coop(sage_graph *g, const void *fn, int grid, void **args, const char *what) {
+  cudaError_t e = cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kBlock), args, 0, g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, what);
+  return SAGE_OK;
+}
+
+int32_t to_internal_id(sage_graph *g, int32_t v) {
+  return g->reordered ? g->h_sigma[(size_t)v] : v;
+}
+
+sage_status translate_out_i32(sage_graph *g, const int32_t *src, int32_t *dst_user,
+                              bool map_values) {
+  const size_t bytes = sizeof(int32_t) * (size_t)g->n_local;
+  if (!g->reordered) return copy_out(g, dst_user, src, bytes);
+  int32_t *tmp = (int32_t *)g->ts.tmp_out;
+  k_gather_i32<<<g->num_sms * 8, 256, 0, g->stream>>>(src, g->sigma, g->sigma_inv, tmp,
+                                                      g->n_local, map_values ? 1 : 0);
+  return copy_out(g, dst_user, tmp, bytes);
+}
+sage_status translate_out_u32(sage_graph *g, const uint32_t *src, uint32_t *dst_user) {
+  const size_t bytes = sizeof(uint32_t) * (size_t)g->n_local;
+  if (!g->reordered) return copy_out(g, dst_user, src, bytes);
+  uint32_t *tmp = (uint32_t *)g->ts.tmp_out;
+  k_gather_u32<<<g->num_sms * 8, 256, 0, g->stream>>>(src, g->sigma, tmp, g->n_local);
+  return copy_out(g, dst_user, tmp, bytes);
+}
+sage_status translate_out_f64(sage_graph *g, const double *src, double *dst_user) {
+  const size_t bytes = sizeof(double) * (size_t)g->n_local;
+  if (!g->reordered) return copy_out(g, dst_user, src, bytes);
+  double *tmp = (double *)g->ts.tmp_out;
+  k_gather_f64<<<g->num_sms * 8, 256, 0, g->stream>>>(src, g->sigma, tmp, g->n_local);
+  return copy_out(g, dst_user, tmp, bytes);
+}
+
+static TravArgs make_args(sage_graph *g) {
+  TravArgs a;
+  memset(&a, 0, sizeof(a));
+  a.off = (const long long *)g->off;
+  a.col = g->col;
+  a.w = g->w;
+  a.n = g->n_local;
+  a.m = g->m;
+  a.L = g->ladder;
+  a.q[0] = g->ts.q[0];
+  a.q[1] = g->ts.q[1];
+  for (int i = 0; i < 3; ++i) a.fb[i] = g->ts.fb[i];
+  a.visited = g->ts.visited;
+  a.level = g->ts.level;
+  a.parent = g->ts.parent;
+  a.dist = g->ts.dist;
+  a.ctl = g->ts.ctl;
+  a.alpha = g->alpha;
+  a.beta = g->beta;
+  a.max_levels = (int)std::min<long long>(g->n + 1, 0x7fffffffll);
+  return a;
+}
+
+static void fill_stats(sage_graph *g, const Ctl &h, bool bfs, bool symmetric, double ms,
+                       double kms, sage_stats *st) {
+  if (!st) return;
+  memset(st, 0, sizeof(*st));
+  st->levels = h.levels;
+  st->push_levels = h.push_levels;
+  st->pull_levels = h.pull_levels;
+  st->vertices_expanded = (int64_t)(h.tot_push_expanded + h.tot_pull_scanned);
+  st->arcs_inspected = (int64_t)(h.tot_push_arcs + h.tot_pull_inspected);
+  st->ms = ms;
+  st->kernel_ms = kms;
+  const double n = (double)g->n_local;
+  if (bfs) {
+    // reached arcs = arcs of the source + arcs of every discovered vertex
+    const double reached_arcs = (double)h.tot_arcs_reached;
+    st->vertices_discovered = (int64_t)(h.tot_push_disc + h.tot_pull_disc);
+    st->edges_traversed = (int64_t)(symmetric ? reached_arcs / 2.0 : reached_arcs);
+    // SURVEY §8(d) frozen byte model
+    double mb = 4.0 * n;
+    mb += 20.0 * h.tot_push_expanded + 8.0 * h.tot_push_arcs + 8.0 * h.tot_push_disc;
+    mb += 16.0 * h.tot_pull_scanned + (n / 8.0) * h.pull_levels +
+          4.125 * h.tot_pull_inspected + 4.125 * h.tot_pull_disc;
+    st->model_bytes = mb;
+  } else {
+    st->vertices_discovered = (int64_t)h.tot_improved;
+    st->edges_traversed = 0;   // filled by the caller from the reached set (R1)
+    double mb = 4.0 * n + 24.0 * h.tot_push_expanded + 12.0 * h.tot_push_arcs +
+                8.0 * h.tot_push_disc;
+    st->model_bytes = mb;
+  }
+}
+
+static sage_status check_common(sage_graph *g, int32_t source, const void *out) {
+  if (!g || !out) {
+    set_error("null argument");
+    return SAGE_E_INVALID;
+  }
+  if (g->sticky) {
+    set_error("graph handle is in a failed state (sticky error %d); free it", g->sticky);
+    return (sage_status)g->sticky;
+  }
+  if (source < 0 || source >= g->n) {
+    set_error("source %d out of range [0, %lld)", source, (long long)g->n);
+    return SAGE_E_INVALID;
+  }
+  return SAGE_OK;
+}
+
+sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int32_t *parent_out,
+                          uint32_t call_flags, sage_stats *st);
+sage_status run_sssp_multi(sage_graph *g, int32_t source, uint32_t *dist_out, sage_stats *st);
+
+}  // namespace sage
+
+using namespace sage;
+
+extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level_out,
+                                   int32_t *parent_out, uint32_t call_flags, sage_stats *st) {
+  clear_error();
+  sage_status s = check_common(g, source, level_out);
+  if (s != SAGE_OK) return s;
+  if (g->comm) return run_bfs_multi(g, source, level_out, parent_out, call_flags, st);
+  if ((s = ensure_traversal_state(g)) != SAGE_OK) return s;
+  TraversalState &t = g->ts;
+  if (parent_out && !t.parent) {
+    if ((s = dalloc(g, (void **)&t.parent, sizeof(int32_t) * (size_t)g->n_local)) != SAGE_OK)
+      return s;
+  }
+  const int32_t src = to_internal_id(g, source);
+  const bool symmetric = g->flags & SAGE_F_SYMMETRIC;
+  const bool push_only = (g->flags | call_flags) & SAGE_F_PUSH_ONLY;
+  cudaEvent_t e0, e1, e2;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  cudaEventCreate(&e2);
+  cudaEventRecord(e0, g->stream);
+  const size_t words = (size_t)((g->n + 31) / 32 + 8);
+  cudaMemsetAsync(t.level, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
+  if (parent_out) cudaMemsetAsync(t.parent, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
+  cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
+  for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
+  cudaMemsetAsync(t.ctl, 0, offsetof(Ctl, rec), g->stream);
+  TravArgs a = make_args(g);
+  a.parent = parent_out ? t.parent : nullptr;
+  a.do_enabled = (symmetric && !push_only) ? 1 : 0;
+  k_seed<<<1, 32, 0, g->stream>>>(a, src, 0);
+  cudaEventRecord(e1, g->stream);
+  const void *fn = g->vec == 4 ? (const void *)k_bfs<4> : (const void *)k_bfs<1>;
+  const int grid = coop_grid(g, fn, &g->grid_bfs);
+  void *args[] = {&a};
+  if ((s = launch_coop(g, fn, grid, args, "BFS kernel")) != SAGE_OK) return s;
+  cudaEventRecord(e2, g->stream);
+  Ctl h;
+  cudaMemcpyAsync(&h, t.ctl, offsetof(Ctl, rec), cudaMemcpyDeviceToHost, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "BFS");
+  float ms = 0, kms = 0;
+  cudaEventElapsedTime(&ms, e0, e2);
+  cudaEventElapsedTime(&kms, e1, e2);
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaEventDestroy(e2);
+  if (h.status == 1) {
+    set_error("BFS exceeded the level cap (internal error)");
+    g->sticky = SAGE_E_CUDA;
+    return SAGE_E_CUDA;
+  }
+  // the source's own arcs (set[0] of level 0) are part of the reached arcs
+  {
+    long long sb = 0, se = 0;
+    cudaMemcpy(&sb, g->off + src, 8, cudaMemcpyDeviceToHost);
+    cudaMemcpy(&se, g->off + src + 1, 8, cudaMemcpyDeviceToHost);
+    h.tot_arcs_reached += (unsigned long long)(se - sb);
+  }
+  fill_stats(g, h, true, symmetric, ms, kms, st);
+  if ((s = translate_out_i32(g, t.level, level_out, false)) != SAGE_OK) return s;
+  if (parent_out && (s = translate_out_i32(g, t.parent, parent_out, true)) != SAGE_OK) return s;
+  e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "BFS output");
+  return SAGE_OK;
+}
+
+extern "C" sage_status sage_bfs(sage_graph *g, int32_t source, int32_t *level_out,
+                                int32_t *parent_out, sage_stats *st) {
+  return sage_bfs_ex(g, source, level_out, parent_out, 0u, st);
+}
+
+extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_out,
+                                 sage_stats *st) {
+  clear_error();
+  sage_status s = check_common(g, source, dist_out);
+  if (s != SAGE_OK) return s;
+  if (!g->w) {
+    set_error("SSSP needs weights (load the CSR with weights)");
+    return SAGE_E_INVALID;
+  }
+  if (g->comm) return run_sssp_multi(g, source, dist_out, st);
+  if ((s = ensure_traversal_state(g)) != SAGE_OK) return s;
+  TraversalState &t = g->ts;
+  if (!t.dist && (s = dalloc(g, (void **)&t.dist, sizeof(uint32_t) * (size_t)g->n_local)) != SAGE_OK)
+    return s;
+  const int32_t src = to_internal_id(g, source);
+  int *ovf = nullptr;
+  if ((s = dalloc(g, (void **)&ovf, sizeof(int) * 2)) != SAGE_OK) return s;
+  cudaEvent_t e0, e1, e2;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  cudaEventCreate(&e2);
+  cudaEventRecord(e0, g->stream);
+  const size_t words = (size_t)((g->n + 31) / 32 + 8);
+  cudaMemsetAsync(ovf, 0, sizeof(int) * 2, g->stream);
+  cudaMemsetAsync(t.dist, 0xff, sizeof(uint32_t) * (size_t)g->n_local, g->stream);
+  cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
+  for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
+  cudaMemsetAsync(t.ctl, 0, offsetof(Ctl, rec), g->stream);
+  TravArgs a = make_args(g);
+  k_seed<<<1, 32, 0, g->stream>>>(a, src, 1);
+  cudaEventRecord(e1, g->stream);
+  const void *fn = g->vec == 4 ? (const void *)k_sssp<4> : (const void *)k_sssp<1>;
+  const int grid = coop_grid(g, fn, &g->grid_sssp);
+  void *args[] = {&a, &ovf};
+  if ((s = launch_coop(g, fn, grid, args, "SSSP kernel")) != SAGE_OK) {
+    dfree(g, ovf);
+    return s;
+  }
+  cudaEventRecord(e2, g->stream);
+  int hovf[2] = {0, 0};
+  cudaMemcpyAsync(hovf, ovf, sizeof(int), cudaMemcpyDeviceToHost, g->stream);
+  Ctl h;
+  cudaMemcpyAsync(&h, t.ctl, offsetof(Ctl, rec), cudaMemcpyDeviceToHost, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) {
+    dfree(g, ovf);
+    return cuda_fail(g, e, "SSSP");
+  }
+  float ms = 0, kms = 0;
+  cudaEventElapsedTime(&ms, e0, e2);
+  cudaEventElapsedTime(&kms, e1, e2);
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaEventDestroy(e2);
+  if (h.status == 1) {
+    dfree(g, ovf);
+    set_error("SSSP exceeded the iteration cap (internal error)");
+    g->sticky = SAGE_E_CUDA;
+    return SAGE_E_CUDA;
+  }
+  if (hovf[0]) {
+    cudaMemsetAsync(ovf + 1, 0, sizeof(int), g->stream);
+    k_overflow_check<<<g->num_sms * 8, 256, 0, g->stream>>>((const long long *)g->off, g->col,
+                                                            t.dist, g->n_local, ovf + 1);
+    cudaMemcpyAsync(hovf + 1, ovf + 1, sizeof(int), cudaMemcpyDeviceToHost, g->stream);
+    cudaStreamSynchronize(g->stream);
+  }
+  dfree(g, ovf);
+  if (hovf[1]) {
+    set_error("a finite shortest distance is >= UINT32_MAX");
+    return SAGE_E_OVERFLOW;
+  }
+  fill_stats(g, h, false, g->flags & SAGE_F_SYMMETRIC, ms, kms, st);
+  if (st) {
+    unsigned long long *dra = nullptr, hra = 0;
+    if ((s = dalloc(g, (void **)&dra, sizeof(unsigned long long))) != SAGE_OK) return s;
+    cudaMemsetAsync(dra, 0, sizeof(unsigned long long), g->stream);
+    k_reached_arcs<<<g->num_sms * 8, 256, 0, g->stream>>>((const long long *)g->off, t.dist,
+                                                          g->n_local, dra);
+    cudaMemcpyAsync(&hra, dra, sizeof(hra), cudaMemcpyDeviceToHost, g->stream);
+    cudaStreamSynchronize(g->stream);
+    dfree(g, dra);
+    st->edges_traversed = (int64_t)((g->flags & SAGE_F_SYMMETRIC) ? hra / 2 : hra);
+  }
+  if ((s = translate_out_u32(g, t.dist, dist_out)) != SAGE_OK) return s;
+  e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "SSSP output");
+  return SAGE_OK;
+}
+
+extern "C" sage_status sage_debug_export_tiles(sage_graph *g, const int32_t *vertices,
+                                               int64_t count, int64_t *quads_out, int64_t cap,
+                                               int64_t *n_out) {
+  clear_error();
+  if (!g || (count > 0 && !vertices) || !n_out || count < 0) {
+    set_error("null argument");
+    return SAGE_E_INVALID;
+  }
+  if (g->sticky) return (sage_status)g->sticky;
+  for (int64_t i = 0; i < count; ++i)
+    if (vertices[i] < 0 || vertices[i] >= g->n_local) {
+      set_error("vertex %d out of range", vertices[i]);
+      return SAGE_E_INVALID;
+    }
+  sage_status s;
+  Queues q;
+  // queue capacity: each listed vertex appears once per class
+  long long msum = 0;
+  {
+    std::vector<long long> hoff((size_t)g->n_local + 1);
+    cudaMemcpy(hoff.data(), g->off, sizeof(long long) * hoff.size(), cudaMemcpyDeviceToHost);
+    for (int64_t i = 0; i < count; ++i) msum += hoff[vertices[i] + 1] - hoff[vertices[i]];
+  }
+  if ((s = alloc_queues(g, &q, count, msum)) != SAGE_OK) return s;
+  int *dv = nullptr;
+  CounterSet *cs = nullptr;
+  long long *dq = nullptr;
+  unsigned long long *dn = nullptr;
+  const long long dcap = msum / g->ladder.B + 16 * count + 16;
+  if ((s = dalloc(g, (void **)&dv, sizeof(int) * (size_t)(count + 1))) != SAGE_OK ||
+      (s = dalloc(g, (void **)&cs, sizeof(CounterSet))) != SAGE_OK ||
+      (s = dalloc(g, (void **)&dq, sizeof(long long) * 4 * (size_t)dcap)) != SAGE_OK ||
+      (s = dalloc(g, (void **)&dn, sizeof(unsigned long long))) != SAGE_OK) {
+    free_queues(g, &q);
+    return s;
+  }
+  cudaMemcpyAsync(dv, vertices, sizeof(int) * (size_t)count, cudaMemcpyHostToDevice, g->stream);
+  cudaMemsetAsync(cs, 0, sizeof(CounterSet), g->stream);
+  cudaMemsetAsync(dn, 0, sizeof(unsigned long long), g->stream);
+  if (count > 0) {
+    k_classify_list<<<g->num_sms * 4, 256, 0, g->stream>>>((const long long *)g->off, dv, count,
+                                                           g->ladder, q, cs);
+    k_expand_log<<<g->num_sms * 4, 256, 0, g->stream>>>((const long long *)g->off, g->ladder, q,
+                                                        cs, dq, dn, dcap);
+  }
+  unsigned long long hn = 0;
+  cudaMemcpyAsync(&hn, dn, sizeof(hn), cudaMemcpyDeviceToHost, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  if (e == cudaSuccess && (long long)hn <= cap && quads_out && hn > 0)
+    e = cudaMemcpy(quads_out, dq, sizeof(long long) * 4 * hn, cudaMemcpyDeviceToHost);
+  *n_out = (int64_t)hn;
+  free_queues(g, &q);
+  dfree(g, dv);
+  dfree(g, cs);
+  dfree(g, dq);
+  dfree(g, dn);
+  cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "debug_export_tiles");
+  return SAGE_OK;
+}

@@ -162,7 +162,8 @@ def test_sssp_unit_weights_equal_bfs(sage):
         s = int(sg.sources(g, 1, seed=2)[0])
         d, _ = G.sssp(s)
         lv, _, _ = G.bfs(s)
-        assert np.array_equal(d.astype(np.int64), np.where(lv < 0, 2**32 - 1, lv).astype(np.int64))
+        lv64 = lv.astype(np.int64)
+        assert np.array_equal(d.astype(np.int64), np.where(lv64 < 0, 2**32 - 1, lv64))
 
 
 def test_sssp_overflow_and_near_overflow(sage):

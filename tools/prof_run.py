@@ -1,0 +1,37 @@
+"""Profiling driver: load a graph once and run a few queries (used under ncu; not a bench)."""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import paper_conf_sigmod_00020t21_b200 as sage  # noqa: E402
+import sagegen as sg  # noqa: E402
+
+p = argparse.ArgumentParser()
+p.add_argument("--scale", type=int, default=24)
+p.add_argument("--op", default="bfs_push", choices=["bfs_push", "bfs_do", "sssp", "pr"])
+p.add_argument("--reps", type=int, default=3)
+p.add_argument("--tile-cta", type=int, default=256)
+p.add_argument("--align", type=int, default=4)
+a = p.parse_args()
+g = sg.rmat(a.scale, 16, 1, True)
+w = sg.weights(g, 1)
+s = stream = torch.cuda.current_stream()
+G = sage.load_csr(torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda(), torch.from_numpy(w).cuda(),
+                  symmetric=True, borrow=True, stream=stream.cuda_stream, tile_cta=a.tile_cta, align=a.align)
+src = sg.sources(g, a.reps, seed=2)
+lv = torch.empty(g.n, dtype=torch.int32, device="cuda")
+for i in range(a.reps):
+    if a.op == "bfs_push":
+        _, _, st = G.bfs(int(src[i]), out=lv, push_only=True)
+    elif a.op == "bfs_do":
+        _, _, st = G.bfs(int(src[i]), out=lv)
+    elif a.op == "sssp":
+        _, st = G.sssp(int(src[i]), out=lv.view(torch.uint32))
+    else:
+        x = torch.empty(g.n, dtype=torch.float64, device="cuda")
+        _, st = G.pagerank(0.85, 5, out=x)
+    print(a.op, i, {k: st[k] for k in ("levels", "kernel_ms", "ms", "edges_traversed", "model_bytes")}, flush=True)

@@ -279,11 +279,7 @@ sage_status sage_load_csr(const sage_csr *in, sage_graph **out) {
       return SAGE_E_CUDA;
     }
   }
-  // vector (int4) column loads need 16-B aligned arrays and an aligned ladder
-  g->vec = (g->ladder.A >= 4 && g->ladder.M >= 4 && ((uintptr_t)g->col % 16) == 0 &&
-            (!g->w || ((uintptr_t)g->w % 16) == 0))
-               ? 4
-               : 1;
+  g->vec = g->ladder.M >= 4 ? 4 : 1;   // neighbours per lane per step (tiles of >= 4 elements)
 
   // validation + stats pass
   {

@@ -170,89 +170,155 @@ __device__ __forceinline__ long long class_tile_start(long long e, int r, int t)
 // ------------------------------------------------------------------------------------------
 // Warp-aggregated enqueue = expandTiles (Alg. 3 l.2-7) of the vertices filtered in by this warp.
 // Every lane of the warp must call it (convergent).  `active` lanes carry vertex v with row
-// [b, e).  Appends v's tiles to the log Q, counting in cs.  Also accumulates |F| and arcs(F).
+// [b, e).  Appends v's tiles to the log Q, counting in cs, and accumulates |F| and arcs(F).
+// All queue reservations of one call are issued in ONE parallel round of atomics (lane c reserves
+// for queue c), so a call costs a single atomic latency whatever the number of classes.
 __device__ __forceinline__ void enqueue_warp(bool active, int v, long long b, long long e,
                                              const Ladder &L, const Queues &Q, CounterSet *cs) {
   const unsigned am = __ballot_sync(FULL, active);
   if (!am) return;
   const unsigned lane = lane_id();
+  const unsigned lt = lanemask_lt();
   RowSplit s{0, 0, 0, 0};
   if (active) s = split_row(b, e, L);
+  // heavy vertices: exclusive scan of their CTA-tile counts
+  unsigned long long q = active ? (unsigned long long)s.q : 0ull;
+  unsigned long long incq = q;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    unsigned long long y = __shfl_up_sync(FULL, incq, o);
+    if ((int)lane >= o) incq += y;
+  }
+  const unsigned long long totq = shfl64(incq, 31);
   unsigned long long deg = active ? (unsigned long long)(e - b) : 0ull;
   deg = warp_sum64(deg);
+  // class ballots; lane c keeps the ballot of queue c (c = 1..ncls-1 tiles, ncls = fragments)
+  unsigned cm[kQueues];
+  unsigned mine_mask = 0;
+#pragma unroll
+  for (int c = 1; c < kQueues; ++c) {
+    cm[c] = 0;
+    if (c < L.ncls) cm[c] = __ballot_sync(FULL, active && (s.r & (L.B >> c)));
+    else if (c == L.ncls) cm[c] = __ballot_sync(FULL, active && (s.h > 0 || (s.r & (L.M - 1)) != 0));
+    if ((int)lane == c) mine_mask = cm[c];
+  }
+  // one parallel round of reservations
+  unsigned long long mybase = 0;
   if (lane == 0) {
+    if (totq) mybase = atomicAdd(&cs->cnt[0], totq);
+  } else if ((int)lane <= L.ncls) {
+    if (mine_mask) mybase = atomicAdd(&cs->cnt[lane], (unsigned long long)__popc(mine_mask));
+  } else if (lane == 30) {
     atomicAdd(&cs->nF, (unsigned long long)__popc(am));
+  } else if (lane == 31) {
     if (deg) atomicAdd(&cs->arcsF, deg);
   }
+  // sub-CTA classes and fragments
+#pragma unroll
+  for (int c = 1; c < kQueues; ++c) {
+    if (c > L.ncls) break;
+    const unsigned long long base = shfl64(mybase, c);
+    if (cm[c] & (1u << lane)) {
+      int *qp = (c == L.ncls) ? Q.frag : Q.cls[c];
+      qp[base + __popc(cm[c] & lt)] = v;
+    }
+  }
   // CTA class: cooperative write of every heavy vertex's q explicit tiles.
-  unsigned hm = __ballot_sync(FULL, active && s.q > 0);
-  while (hm) {
-    const int src = __ffs(hm) - 1;
-    hm &= hm - 1;
-    const unsigned long long q = shfl64((unsigned long long)s.q, src);
-    const long long b2 = (long long)shfl64((unsigned long long)s.b2, src);
-    const int vv = __shfl_sync(FULL, v, src);
-    unsigned long long base = 0;
-    if (lane == 0) base = atomicAdd(&cs->cnt[0], q);
-    base = shfl64(base, 0);
-    for (unsigned long long j = lane; j < q; j += 32)
-      st_tile(Q.cta + base + j, b2 + (long long)j * L.B, vv, L.B);
+  if (totq) {
+    const unsigned long long base0 = shfl64(mybase, 0);
+    unsigned hm = __ballot_sync(FULL, q > 0);
+    while (hm) {
+      const int src = __ffs(hm) - 1;
+      hm &= hm - 1;
+      const unsigned long long qs = shfl64(q, src);
+      const unsigned long long bs = base0 + shfl64(incq, src) - qs;
+      const long long b2 = (long long)shfl64((unsigned long long)s.b2, src);
+      const int vv = __shfl_sync(FULL, v, src);
+      for (unsigned long long j = lane; j < qs; j += 32)
+        st_tile(Q.cta + bs + j, b2 + (long long)j * L.B, vv, L.B);
+    }
   }
-  // Sub-CTA classes: one entry per set bit of the residual.
-  const unsigned lt = lanemask_lt();
-  for (int c = 1; c < L.ncls; ++c) {
-    const int t = L.B >> c;
-    const bool mine = active && (s.r & t);
-    const unsigned cm = __ballot_sync(FULL, mine);
-    if (!cm) continue;
-    const int leader = __ffs(cm) - 1;
-    unsigned long long base = 0;
-    if ((int)lane == leader) base = atomicAdd(&cs->cnt[c], (unsigned long long)__popc(cm));
-    base = shfl64(base, leader);
-    if (mine) Q.cls[c][base + __popc(cm & lt)] = v;
+}
+
+// enqueue_warp for vertex ids only: loads the rows first (one round of loads for the warp).
+__device__ __forceinline__ void enqueue_ids(bool active, int v, const long long *__restrict__ off,
+                                            const Ladder &L, const Queues &Q, CounterSet *cs) {
+  long long b = 0, e = 0;
+  if (active) {
+    b = __ldg(off + v);
+    e = __ldg(off + v + 1);
   }
-  // Fragments (head and/or tail).
-  const bool fr = active && (s.h > 0 || (s.r & (L.M - 1)) != 0);
-  const unsigned fm = __ballot_sync(FULL, fr);
-  if (fm) {
-    const int leader = __ffs(fm) - 1;
-    unsigned long long base = 0;
-    if ((int)lane == leader) base = atomicAdd(&cs->cnt[L.ncls], (unsigned long long)__popc(fm));
-    base = shfl64(base, leader);
-    if (fr) Q.frag[base + __popc(fm & lt)] = v;
+  enqueue_warp(active, v, b, e, L, Q, cs);
+}
+
+// Per-warp shared scratch: the fragment gather's tables and the buffer of filtered-in vertices
+// (contraction is batched: 32 vertices per enqueue call, not one call per discovery).
+struct WarpScratch {
+  int pre[32];
+  int hl[32];
+  long long hb[32];
+  long long tb[32];
+  int buf[64];
+};
+
+// Append the lanes' filtered-in vertices to the warp buffer; flush full batches of 32.
+__device__ __forceinline__ void buffer_push(bool in, int v, WarpScratch *ws, int &cnt,
+                                            const long long *__restrict__ off, const Ladder &L,
+                                            const Queues &Q, CounterSet *cs) {
+  const unsigned m = __ballot_sync(FULL, in);
+  if (!m) return;
+  const unsigned lane = lane_id();
+  if (in) ws->buf[cnt + __popc(m & lanemask_lt())] = v;
+  cnt += __popc(m);
+  if (cnt >= 32) {
+    __syncwarp();
+    const int x = ws->buf[lane];
+    const int y = ws->buf[32 + lane];
+    __syncwarp();
+    cnt -= 32;
+    if ((int)lane < cnt) ws->buf[lane] = y;
+    __syncwarp();
+    enqueue_ids(true, x, off, L, Q, cs);
   }
+}
+__device__ __forceinline__ void buffer_flush(WarpScratch *ws, int &cnt,
+                                             const long long *__restrict__ off, const Ladder &L,
+                                             const Queues &Q, CounterSet *cs) {
+  __syncwarp();
+  const unsigned lane = lane_id();
+  const bool in = (int)lane < cnt;
+  const int x = in ? ws->buf[lane] : 0;
+  __syncwarp();
+  cnt = 0;
+  enqueue_ids(in, x, off, L, Q, cs);
 }
 
 // ------------------------------------------------------------------------------------------
 // The stealing consumer (Resident Tile Stealing, Alg. 3 l.9-17).  Every warp of the
 // persistent grid takes batches of tiles of one class from a device-wide ticket counter, so any
 // SM consumes any tile; classes are drained largest first.  A tile of t elements is covered by
-// t/VEC lanes, each holding one VEC-wide (16 B for VEC=4) coalesced load of `col` per step
-// (the paper's one-neighbour-per-thread tile, vectorised for sm_100a).  Fragments (< M) are
-// consumed by a warp scan-based gather ([30]): 32 fragment vertices per round, lane k
-// takes the k-th element of their concatenation.
+// t/VEC lanes (the paper's one-neighbour-per-thread tile, each lane carrying VEC neighbours).
+// Lane sl of a tile's group reads elements sl, sl + g, sl + 2g, ... (g = group width): every
+// load instruction is coalesced, and the 32 neighbours a warp checks at once are CONSECUTIVE
+// entries of a row, so on a sorted hub row their status words share L1/L2 lines.
+// Fragments (< M) are consumed by a warp scan-based gather ([30]): 32 fragment vertices
+// per round, lane k takes the k-th element of their concatenation.
 //
 // Filter policy F provides:
 //   struct Src;                                    per-source-vertex context
-//   __device__ Src src(bool valid, int u, long long b, long long e);  (b,e = row of u)
-//   template<int N> __device__ void visit(bool valid, const Src&, const int (&v)[N],
-//                                          const uint32_t (&w)[N]);   convergent (whole warp)
-//   static constexpr bool kWeights;                 load weights alongside col
-
-struct FragSmem {        // per-warp scratch of the fragment gather
-  int pre[32];
-  int hl[32];
-  long long hb[32];
-  long long tb[32];
-};
-
+//   Src src(bool valid, int u, long long b, long long e);   (b,e = row of u when needed)
+//   template<int N> void visit(bool valid, const Src&, const int (&v)[N], const uint32_t (&w)[N],
+//                              bool (&in)[N]);      marks the neighbours filtered in
+//   kWeights (load weights), kNeedRow (src needs the row for CTA tiles), kEnqueue (contraction)
+//   Queues *next_q; CounterSet *next_cs;             where filtered-in vertices go
 template <int VEC, class F>
-__device__ __forceinline__ void consume_log(F &f, const Ladder &L, const Queues &Q,
+__device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Queues &Q,
                                             CounterSet *cs, const long long *__restrict__ off,
                                             const int *__restrict__ col,
-                                            const uint32_t *__restrict__ w, FragSmem *fs,
+                                            const uint32_t *__restrict__ w, WarpScratch *ws,
                                             typename F::Src *fsrc) {
   const unsigned lane = lane_id();
+  int bcnt = 0;   // warp-uniform fill of ws->buf
   for (int c = 0; c < L.ncls; ++c) {
     const int t = L.B >> c;
     const unsigned long long count = ldcg(&cs->cnt[c]);
@@ -260,9 +326,8 @@ __device__ __forceinline__ void consume_log(F &f, const Ladder &L, const Queues 
     const int lpt = (t / VEC) < 32 ? (t / VEC) : 32;  // lanes per tile
     const int tps = 32 / lpt;                           // tiles per warp step
     const int spt = (t / VEC) > 32 ? (t / (32 * VEC)) : 1;  // steps per tile
-    // batch ≈ 4 KB of column data per ticket (bounded by 4 tiles of the largest class)
-    int batch = (1024 / t);
-    if (batch < 1) batch = 1;
+    // batch ≈ 4 KB of column data per ticket
+    int batch = 1024 / t;
     if (batch < tps) batch = tps;
     const int sub = lane / lpt, sl = lane % lpt;
     for (;;) {
@@ -281,7 +346,10 @@ __device__ __forceinline__ void consume_log(F &f, const Ladder &L, const Queues 
             CtaTile T = ldcg_tile(Q.cta + ti);
             start = T.start;
             u = T.u;
-            if (F::kNeedRow) { rb = ld_off(off + u); re = ld_off(off + u + 1); }
+            if (F::kNeedRow) {
+              rb = ld_off(off + u);
+              re = ld_off(off + u + 1);
+            }
           } else {
             u = ldcg(Q.cls[c] + ti);
             rb = ld_off(off + u);
@@ -292,34 +360,29 @@ __device__ __forceinline__ void consume_log(F &f, const Ladder &L, const Queues 
         }
         const typename F::Src sc = f.src(valid, u, rb, re);
         for (int s = 0; s < spt; ++s) {
-          const long long pos = start + (long long)s * (32 * VEC) + (long long)sl * VEC;
+          const long long p0 = start + (long long)s * (lpt * VEC) + sl;
           int v[VEC];
           uint32_t ww[VEC];
-          if constexpr (VEC == 4) {
-            int4 c4 = make_int4(0, 0, 0, 0);
-            uint4 w4 = make_uint4(0, 0, 0, 0);
-            if (valid) {
-              c4 = ld_stream4(col + pos);
-              if (F::kWeights) w4 = ld_stream4u(w + pos);
-            }
-            v[0] = c4.x; v[1] = c4.y; v[2] = c4.z; v[3] = c4.w;
-            ww[0] = w4.x; ww[1] = w4.y; ww[2] = w4.z; ww[3] = w4.w;
-          } else {
 #pragma unroll
-            for (int j = 0; j < VEC; ++j) {
-              v[j] = valid ? ld_stream1(col + pos + j) : 0;
-              ww[j] = (valid && F::kWeights) ? ld_stream1u(w + pos + j) : 0u;
-            }
+          for (int j = 0; j < VEC; ++j) {
+            v[j] = valid ? ld_stream1(col + p0 + j * lpt) : 0;
+            ww[j] = (valid && F::kWeights) ? ld_stream1u(w + p0 + j * lpt) : 0u;
           }
-          f.template visit<VEC>(valid, sc, v, ww);
+          bool in[VEC];
+          f.template visit<VEC>(valid, sc, v, ww, in);
+          if constexpr (F::kEnqueue) {
+#pragma unroll
+            for (int j = 0; j < VEC; ++j)
+              buffer_push(in[j], v[j], ws, bcnt, off, L, *f.next_q, f.next_cs);
+          }
         }
       }
     }
   }
   // ---- fragments: warp scan-based gather
   const unsigned long long fcount = ldcg(&cs->cnt[L.ncls]);
-  if (fcount == 0) return;
   for (;;) {
+    if (fcount == 0) break;
     unsigned long long base = 0;
     if (lane == 0) base = atomicAdd(&cs->tk[L.ncls], 32ull);
     base = shfl64(base, 0);
@@ -339,7 +402,6 @@ __device__ __forceinline__ void consume_log(F &f, const Ladder &L, const Queues 
     }
     const typename F::Src sc = f.src(valid, u, rb, re);
     int fl = hl + tl;
-    // inclusive warp scan of fl
     int inc = fl;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -347,10 +409,10 @@ __device__ __forceinline__ void consume_log(F &f, const Ladder &L, const Queues 
       if ((int)lane >= o) inc += y;
     }
     const int total = __shfl_sync(FULL, inc, 31);
-    fs->pre[lane] = inc - fl;
-    fs->hl[lane] = hl;
-    fs->hb[lane] = hb;
-    fs->tb[lane] = tb;
+    ws->pre[lane] = inc - fl;
+    ws->hl[lane] = hl;
+    ws->hb[lane] = hb;
+    ws->tb[lane] = tb;
     fsrc[lane] = sc;
     __syncwarp();
     for (int k0 = 0; k0 < total; k0 += 32) {
@@ -359,26 +421,30 @@ __device__ __forceinline__ void consume_log(F &f, const Ladder &L, const Queues 
       int o = 0;
       if (kv) {   // largest o with pre[o] <= k
         int lo = 0, hi = 31;
-        while (lo < hi) {
+#pragma unroll
+        for (int it = 0; it < 5; ++it) {
           int mid = (lo + hi + 1) >> 1;
-          if (fs->pre[mid] <= k) lo = mid; else hi = mid - 1;
+          if (ws->pre[mid] <= k) lo = mid; else hi = mid - 1;
         }
         o = lo;
       }
-      int vv[1];
-      uint32_t w1[1];
-      vv[0] = 0;
-      w1[0] = 0;
-      typename F::Src so = fsrc[o];
+      int vv[1] = {0};
+      uint32_t w1[1] = {0u};
+      const typename F::Src so = fsrc[o];
       if (kv) {
-        const int idx = k - fs->pre[o];
-        const long long pos = idx < fs->hl[o] ? fs->hb[o] + idx : fs->tb[o] + (idx - fs->hl[o]);
+        const int idx = k - ws->pre[o];
+        const long long pos = idx < ws->hl[o] ? ws->hb[o] + idx : ws->tb[o] + (idx - ws->hl[o]);
         vv[0] = ld_stream1(col + pos);
         if (F::kWeights) w1[0] = ld_stream1u(w + pos);
       }
-      f.template visit<1>(kv, so, vv, w1);
+      bool in[1];
+      f.template visit<1>(kv, so, vv, w1, in);
+      if constexpr (F::kEnqueue) buffer_push(in[0], vv[0], ws, bcnt, off, L, *f.next_q, f.next_cs);
     }
     __syncwarp();
+  }
+  if constexpr (F::kEnqueue) {
+    if (bcnt) buffer_flush(ws, bcnt, off, L, *f.next_q, f.next_cs);
   }
 }
 

@@ -22,6 +22,9 @@ struct PrPush {
   };
   static constexpr bool kWeights = false;
   static constexpr bool kNeedRow = true;
+  static constexpr bool kEnqueue = false;
+  const Queues *next_q = nullptr;
+  CounterSet *next_cs = nullptr;
   const double *x;
   double *y;
 
@@ -31,7 +34,9 @@ struct PrPush {
   }
   template <int N>
   __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
-                                        const uint32_t (&)[N]) const {
+                                        const uint32_t (&)[N], bool (&in)[N]) const {
+#pragma unroll
+    for (int j = 0; j < N; ++j) in[j] = false;
     if (!valid) return;
 #pragma unroll
     for (int j = 0; j < N; ++j) atomicAdd(y + v[j], s.c);
@@ -89,9 +94,9 @@ __global__ void k_pr_init(double *x, double *y, long long n, double v0) {
 }
 
 template <int VEC>
-__global__ void __launch_bounds__(kBlock) k_pagerank(PrArgs a) {
+__global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ PrArgs a) {
   cg::grid_group grid = cg::this_grid();
-  __shared__ FragSmem fsm[kWarps];
+  __shared__ WarpScratch wsm[kWarps];
   __shared__ PrPush::Src fsrc[kWarps][32];
   __shared__ double red[kWarps];
   const int warp = threadIdx.x >> 5;
@@ -108,7 +113,7 @@ __global__ void __launch_bounds__(kBlock) k_pagerank(PrArgs a) {
     PrPush f;
     f.x = a.x;
     f.y = a.y;
-    consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &fsm[warp], fsrc[warp]);
+    consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &wsm[warp], fsrc[warp]);
     // dangling mass of this iteration's x
     double dsum = 0.0;
     for (long long i = tid; i < a.n_dangling; i += stride) dsum += ldcg(a.x + a.dangling[i]);

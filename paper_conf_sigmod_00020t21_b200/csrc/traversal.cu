@@ -34,49 +34,38 @@ struct BfsPush {
   };
   static constexpr bool kWeights = false;
   static constexpr bool kNeedRow = false;
+  static constexpr bool kEnqueue = true;
   uint32_t *visited;
   int *level;
   int *parent;
   uint32_t *fb_next;   // next-frontier bitmap (only when direction switching is enabled)
   int next_level;
   int v_base;          // global id of local row 0 (0 on one GPU)
-  const long long *off;
-  Ladder L;
-  Queues Qn;
-  CounterSet *csn;
+  const Queues *next_q;
+  CounterSet *next_cs;
 
   __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
 
+  // Alg. 1 l.1-6: if dist[nb] = -1 then dist[nb] := dist[fr] + 1; filter_in(nb)
   template <int N>
   __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
-                                        const uint32_t (&)[N]) const {
-    bool disc[N];
+                                        const uint32_t (&)[N], bool (&in)[N]) const {
     uint32_t wd[N];
 #pragma unroll
     for (int j = 0; j < N; ++j) wd[j] = valid ? visited[v[j] >> 5] : 0xffffffffu;
-    bool anyd = false;
 #pragma unroll
     for (int j = 0; j < N; ++j) {
       const uint32_t bit = 1u << (v[j] & 31);
-      disc[j] = false;
+      in[j] = false;
       if (!(wd[j] & bit)) {
         const uint32_t old = atomicOr(visited + (v[j] >> 5), bit);
-        disc[j] = !(old & bit);
+        in[j] = !(old & bit);
       }
-      anyd |= disc[j];
-    }
-    if (!__any_sync(FULL, anyd)) return;
-#pragma unroll
-    for (int j = 0; j < N; ++j) {
-      long long b = 0, e = 0;
-      if (disc[j]) {
+      if (in[j]) {
         level[v[j]] = next_level;
         if (parent) parent[v[j]] = s.u + v_base;
-        if (fb_next) atomicOr(fb_next + (v[j] >> 5), 1u << (v[j] & 31));
-        b = ld_off(off + v[j]);
-        e = ld_off(off + v[j] + 1);
+        if (fb_next) atomicOr(fb_next + (v[j] >> 5), bit);
       }
-      enqueue_warp(disc[j], v[j], b, e, L, Qn, csn);
     }
   }
 };
@@ -87,13 +76,12 @@ struct SsspPush {
   };
   static constexpr bool kWeights = true;
   static constexpr bool kNeedRow = false;
+  static constexpr bool kEnqueue = true;
   uint32_t *dist;
   uint32_t *inq_next;   // dedupe bitmap of the next frontier
   int *overflow;
-  const long long *off;
-  Ladder L;
-  Queues Qn;
-  CounterSet *csn;
+  const Queues *next_q;
+  CounterSet *next_cs;
 
   __device__ __forceinline__ Src src(bool valid, int u, long long, long long) const {
     // dist[u] may have been lowered by another SM in an earlier iteration: read through L2
@@ -102,39 +90,26 @@ struct SsspPush {
 
   template <int N>
   __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
-                                        const uint32_t (&w)[N]) const {
-    bool enq[N];
-    bool anye = false;
+                                        const uint32_t (&w)[N], bool (&in)[N]) const {
+    uint32_t cur[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) cur[j] = valid ? dist[v[j]] : 0u;
 #pragma unroll
     for (int j = 0; j < N; ++j) {
-      enq[j] = false;
-      if (valid) {
-        const unsigned long long nd = (unsigned long long)s.du + w[j];
-        if (nd >= 0xffffffffull) {
-          *overflow = 1;     // possible overflow: resolved exactly after the traversal
-        } else {
-          const uint32_t cur = dist[v[j]];
-          if ((uint32_t)nd < cur) {
-            const uint32_t old = atomicMin(dist + v[j], (uint32_t)nd);
-            if ((uint32_t)nd < old) {
-              const uint32_t bit = 1u << (v[j] & 31);
-              const uint32_t o2 = atomicOr(inq_next + (v[j] >> 5), bit);
-              enq[j] = !(o2 & bit);
-            }
+      in[j] = false;
+      const unsigned long long nd = (unsigned long long)s.du + w[j];
+      if (valid && nd >= 0xffffffffull) {
+        if (s.du != 0xffffffffu) *overflow = 1;  // possible overflow: resolved after the traversal
+      } else if (valid && nd < cur[j]) {
+        {
+          const uint32_t old = atomicMin(dist + v[j], (uint32_t)nd);
+          if ((uint32_t)nd < old) {
+            const uint32_t bit = 1u << (v[j] & 31);
+            const uint32_t o2 = atomicOr(inq_next + (v[j] >> 5), bit);
+            in[j] = !(o2 & bit);
           }
         }
       }
-      anye |= enq[j];
-    }
-    if (!__any_sync(FULL, anye)) return;
-#pragma unroll
-    for (int j = 0; j < N; ++j) {
-      long long b = 0, e = 0;
-      if (enq[j]) {
-        b = ld_off(off + v[j]);
-        e = ld_off(off + v[j] + 1);
-      }
-      enqueue_warp(enq[j], v[j], b, e, L, Qn, csn);
     }
   }
 };
@@ -162,7 +137,8 @@ struct TravArgs {
 // Pull (bottom-up) step over the visited bitmap: one warp per 32-vertex word.
 __device__ __forceinline__ void pull_level(const TravArgs &a, int next_level, const uint32_t *fbc,
                                            uint32_t *fbn, const Queues &Qn, CounterSet *cur,
-                                           CounterSet *nxt) {
+                                           CounterSet *nxt, WarpScratch *ws) {
+  int bcnt = 0;
   const unsigned lane = lane_id();
   const long long nwords = (a.n + 31) >> 5;
   const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -200,8 +176,9 @@ __device__ __forceinline__ void pull_level(const TravArgs &a, int next_level, co
         if (a.parent) a.parent[v] = par;
       }
     }
-    enqueue_warp(found, (int)v, b, e, a.L, Qn, nxt);
+    buffer_push(found, (int)v, ws, bcnt, a.off, a.L, Qn, nxt);
   }
+  if (bcnt) buffer_flush(ws, bcnt, a.off, a.L, Qn, nxt);
   insp = warp_sum64(insp);
   scanned = warp_sum64(scanned);
   if (lane == 0) {
@@ -255,9 +232,9 @@ __device__ __forceinline__ void record_level(Ctl *ctl, int L, int dir, const Cou
 
 // ============================================================================ BFS kernel
 template <int VEC>
-__global__ void __launch_bounds__(kBlock) k_bfs(TravArgs a) {
+__global__ void __launch_bounds__(kBlock, 4) k_bfs(const __grid_constant__ TravArgs a) {
   cg::grid_group grid = cg::this_grid();
-  __shared__ FragSmem fsm[kWarps];
+  __shared__ WarpScratch wsm[kWarps];
   __shared__ BfsPush::Src fsrc[kWarps][32];
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
@@ -280,13 +257,11 @@ __global__ void __launch_bounds__(kBlock) k_bfs(TravArgs a) {
       f.fb_next = a.do_enabled ? fbn : nullptr;
       f.next_level = L + 1;
       f.v_base = 0;
-      f.off = a.off;
-      f.L = a.L;
-      f.Qn = a.q[(L + 1) & 1];
-      f.csn = nxt;
-      consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &fsm[warp], fsrc[warp]);
+      f.next_q = &a.q[(L + 1) & 1];
+      f.next_cs = nxt;
+      consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp]);
     } else {
-      pull_level(a, L + 1, fbc, fbn, a.q[(L + 1) & 1], cur, nxt);
+      pull_level(a, L + 1, fbc, fbn, a.q[(L + 1) & 1], cur, nxt, &wsm[warp]);
     }
     grid.sync();
     const unsigned long long nF = ldcg(&nxt->nF);
@@ -311,9 +286,9 @@ __global__ void __launch_bounds__(kBlock) k_bfs(TravArgs a) {
 
 // ============================================================================ SSSP kernel
 template <int VEC>
-__global__ void __launch_bounds__(kBlock) k_sssp(TravArgs a, int *overflow) {
+__global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ TravArgs a, int *overflow) {
   cg::grid_group grid = cg::this_grid();
-  __shared__ FragSmem fsm[kWarps];
+  __shared__ WarpScratch wsm[kWarps];
   __shared__ SsspPush::Src fsrc[kWarps][32];
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
@@ -321,18 +296,16 @@ __global__ void __launch_bounds__(kBlock) k_sssp(TravArgs a, int *overflow) {
   for (int L = 0;; ++L) {
     CounterSet *cur = &ctl->set[L % 3];
     CounterSet *nxt = &ctl->set[(L + 1) % 3];
-    __syncthreads();   // block 0: record_level(L-1) finished before set (L+2)%3 is zeroed
+    __syncthreads();
     zero_counterset(&ctl->set[(L + 2) % 3]);
     clear_words(a.fb[(L + 2) % 3], nwords);
     SsspPush f;
     f.dist = a.dist;
     f.inq_next = a.fb[(L + 1) % 3];
     f.overflow = overflow;
-    f.off = a.off;
-    f.L = a.L;
-    f.Qn = a.q[(L + 1) & 1];
-    f.csn = nxt;
-    consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &fsm[warp], fsrc[warp]);
+    f.next_q = &a.q[(L + 1) & 1];
+    f.next_cs = nxt;
+    consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp]);
     grid.sync();
     const unsigned long long nF = ldcg(&nxt->nF);
     if (blockIdx.x == 0 && threadIdx.x == 0) record_level(ctl, L, 0, cur, nxt);

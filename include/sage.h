@@ -171,6 +171,14 @@ sage_status sage_graph_info(const sage_graph *g, int64_t *n, int64_t *m, int64_t
 sage_status sage_debug_export_tiles(sage_graph *g, const int32_t *vertices, int64_t count,
                                     int64_t *quads_out, int64_t cap, int64_t *n_out);
 
+/* Diagnostic entry point: per-level records of the last BFS / SSSP query on this graph, 8 int64 per
+ * level: direction (0 push, 1 pull), |F|, arcs(F), arcs inspected, vertices scanned (pull),
+ * vertices discovered, device time since the kernel started at the end of the level (ns), and
+ * the time at which the last warp finished the level's work, before the grid barrier (ns).
+ * Writes min(levels, cap) records to host memory; *n_out = number of levels (<= 4096 kept).     */
+sage_status sage_debug_level_records(const sage_graph *g, int64_t *rec_out, int32_t cap,
+                                     int32_t *n_out);
+
 /* Thread-local message of the last failing call on this thread ("" if none).                   */
 const char *sage_last_error(void);
 

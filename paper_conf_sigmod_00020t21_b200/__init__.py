@@ -16,7 +16,7 @@ from dataclasses import dataclass
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsage.so")
+LIB_PATH = os.path.join(_HERE, os.environ.get("SAGE_LIB", "libsage.so"))
 
 OK, E_INVALID, E_NOMEM, E_CUDA, E_NCCL, E_OVERFLOW, E_UNSUPPORTED = range(7)
 F_SYMMETRIC, F_DEVICE_PTRS, F_BORROW, F_NO_VALIDATE, F_PUSH_ONLY = 1, 2, 4, 8, 16
@@ -25,7 +25,7 @@ STATUS_NAMES = {0: "SAGE_OK", 1: "SAGE_E_INVALID", 2: "SAGE_E_NOMEM", 3: "SAGE_E
 
 EXPORTED = ["sage_load_csr", "sage_free", "sage_bfs", "sage_bfs_ex", "sage_sssp", "sage_pagerank",
             "sage_reorder", "sage_get_permutation", "sage_get_csr", "sage_graph_info",
-            "sage_debug_export_tiles", "sage_last_error", "sage_version"]
+            "sage_debug_export_tiles", "sage_debug_level_records", "sage_last_error", "sage_version"]
 
 
 class SageError(RuntimeError):
@@ -89,6 +89,7 @@ def lib():
         L.sage_get_csr.argtypes = [p, p, p, p]
         L.sage_graph_info.argtypes = [p, p, p, p, p, p]
         L.sage_debug_export_tiles.argtypes = [p, p, i64, p, i64, p]
+        L.sage_debug_level_records.argtypes = [p, p, i32, p]
         L.sage_last_error.restype = ctypes.c_char_p
         L.sage_version.restype = ctypes.c_char_p
         for f in EXPORTED:
@@ -231,6 +232,14 @@ class Graph:
         w = np.empty(max(self.m, 1), dtype=np.uint32)
         _check(lib().sage_get_csr(self._h, off.ctypes.data, col.ctypes.data, w.ctypes.data))
         return off, col[:self.m], w[:self.m]
+
+    def level_records(self) -> np.ndarray:
+        """sage_debug_level_records -> int64[levels, 8] (dir, |F|, arcs(F), inspected, scanned,
+        discovered, t_ns at level end, t_ns when the last warp finished) of the last BFS/SSSP query."""
+        n = ctypes.c_int32(0)
+        buf = np.zeros(8 * 4096, dtype=np.int64)
+        _check(lib().sage_debug_level_records(self._h, buf.ctypes.data, 4096, ctypes.byref(n)))
+        return buf[:8 * min(n.value, 4096)].reshape(-1, 8)
 
     def export_tiles(self, vertices) -> np.ndarray:
         """sage_debug_export_tiles -> int64[k, 4] (vertex, offset, size, kind)."""

@@ -280,6 +280,8 @@ sage_status sage_load_csr(const sage_csr *in, sage_graph **out) {
     }
   }
   g->vec = g->ladder.M >= 4 ? 4 : 1;   // neighbours per lane per step (tiles of >= 4 elements)
+  g->vec_ok = g->vec == 4 && g->ladder.A >= 4 && ((uintptr_t)g->col % 16) == 0 &&
+              (!g->w || ((uintptr_t)g->w % 16) == 0);
 
   // validation + stats pass
   {

@@ -48,22 +48,35 @@ struct Queues {        // one resident tile log (one level's, or the all-V log o
   int *frag;           // fragment queue (vertex ids)
 };
 
+// One counter per 128-B line: every warp of the grid hits these with atomics, and counters that
+// share a line serialise on the same L2 slice.
+struct alignas(128) PaddedCounter {
+  unsigned long long v;
+  unsigned long long pad[15];
+};
 struct CounterSet {                      // counters of one log (rotated over 3 levels)
-  unsigned long long cnt[kQueues];       // entries per queue (index ncls = fragment queue)
-  unsigned long long tk[kQueues];        // stealing tickets per queue
-  unsigned long long nF, arcsF;          // |F| and arcs(F) of the vertices enqueued here
-  unsigned long long inspected;          // pull: arcs inspected while consuming this level
-  unsigned long long scanned;            // pull: unvisited non-isolated vertices scanned
-  unsigned long long pad[4];
+  PaddedCounter cnt[kQueues];            // entries per queue (index ncls = fragment queue)
+  PaddedCounter tk[kQueues];             // stealing tickets per queue
+  PaddedCounter nF, arcsF;               // |F| and arcs(F) of the vertices enqueued here
+  PaddedCounter inspected;               // pull: arcs inspected while consuming this level
+  PaddedCounter scanned;                 // pull: unvisited non-isolated vertices scanned
 };
 
 struct LevelRec {                        // per-level record (first kMaxRec levels)
   int dir;                               // 0 push, 1 pull
   int pad;
   unsigned long long nF, arcsF, inspected, scanned, discovered;
+  unsigned long long t_ns;               // %globaltimer at the end of the level
+  unsigned long long t_work;             // %globaltimer when the last warp finished its work
 };
 constexpr int kMaxRec = 4096;
 
+struct alignas(128) GridBar {
+  unsigned int count;
+  unsigned int pad0[31];
+  unsigned int gen;
+  unsigned int pad1[31];
+};
 struct Ctl {                             // control block of one query (device memory)
   CounterSet set[3];
   unsigned long long tot_push_expanded, tot_push_arcs, tot_push_disc;
@@ -73,6 +86,9 @@ struct Ctl {                             // control block of one query (device m
   int status;                            // 0 ok, 1 iteration cap hit, 2 possible overflow
   double D[3];                           // PageRank dangling mass (rotated)
   unsigned long long tot_improved;
+  unsigned long long t0_ns;              // %globaltimer at kernel start
+  GridBar bar;                           // grid barrier of the persistent kernel
+  unsigned long long prof[16];           // SAGE_PROF builds: per-phase cycle sums
   LevelRec rec[kMaxRec];
 };
 
@@ -103,6 +119,49 @@ __device__ __forceinline__ uint32_t ld_stream1u(const uint32_t *p) {
   return r;
 }
 __device__ __forceinline__ long long ld_off(const long long *p) { return __ldg(p); }
+
+// L2 cache policies: the column / weight stream is read once per level -> evict_first; the
+// status words (visited bitmap, dist) are re-read at random all level long -> evict_last.
+__device__ __forceinline__ unsigned long long policy_evict_first() {
+  unsigned long long p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ unsigned long long policy_evict_last() {
+  unsigned long long p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ int ld_col(const int *p, unsigned long long pol) {
+  int r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;"
+               : "=r"(r) : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ int4 ld_col4(const int *p, unsigned long long pol) {
+  int4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], %5;"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ uint4 ld_col4u(const uint32_t *p, unsigned long long pol) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ uint32_t ld_colu(const uint32_t *p, unsigned long long pol) {
+  uint32_t r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;"
+               : "=r"(r) : "l"(p), "l"(pol));
+  return r;
+}
+// status word load (coherent, L1-cacheable, kept in L2)
+__device__ __forceinline__ uint32_t ld_status(const uint32_t *p, unsigned long long pol) {
+  uint32_t r;
+  asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+  return r;
+}
 template <class T> __device__ __forceinline__ T ldcg(const T *p) { return __ldcg(p); }
 __device__ __forceinline__ CtaTile ldcg_tile(const CtaTile *p) {
   longlong2 v = __ldcg(reinterpret_cast<const longlong2 *>(p));
@@ -119,6 +178,11 @@ __device__ __forceinline__ void st_tile(CtaTile *p, long long start, int u, int 
   *reinterpret_cast<longlong2 *>(p) = v;
 }
 
+__device__ __forceinline__ unsigned long long globaltimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 __device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31; }
 __device__ __forceinline__ unsigned lanemask_lt() {
   unsigned m;
@@ -137,6 +201,39 @@ __device__ __forceinline__ double warp_sumd(double v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
   return v;
+}
+
+// ------------------------------------------------------------------------------------------
+// Grid-wide barrier of the persistent kernels (launched cooperatively, so every CTA is
+// resident).  Waiting CTA leaders back off with __nanosleep instead of hammering the flag's L2
+// line, which would slow down the warps still working on a small level.
+__device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned *p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(unsigned *p, unsigned v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void grid_barrier(GridBar *b) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const unsigned g = ld_acquire_gpu(&b->gen);
+    __threadfence();
+    if (atomicAdd(&b->count, 1u) == gridDim.x - 1) {
+      b->count = 0;
+      __threadfence();
+      st_release_gpu(&b->gen, g + 1);
+    } else {
+      unsigned ns = 32;
+      while (ld_acquire_gpu(&b->gen) == g) {
+        __nanosleep(ns);
+        if (ns < 512) ns <<= 1;
+      }
+    }
+    __threadfence();
+  }
+  __syncthreads();
 }
 
 // ------------------------------------------------------------------------------------------
@@ -205,13 +302,13 @@ __device__ __forceinline__ void enqueue_warp(bool active, int v, long long b, lo
   // one parallel round of reservations
   unsigned long long mybase = 0;
   if (lane == 0) {
-    if (totq) mybase = atomicAdd(&cs->cnt[0], totq);
+    if (totq) mybase = atomicAdd(&cs->cnt[0].v, totq);
   } else if ((int)lane <= L.ncls) {
-    if (mine_mask) mybase = atomicAdd(&cs->cnt[lane], (unsigned long long)__popc(mine_mask));
+    if (mine_mask) mybase = atomicAdd(&cs->cnt[lane].v, (unsigned long long)__popc(mine_mask));
   } else if (lane == 30) {
-    atomicAdd(&cs->nF, (unsigned long long)__popc(am));
+    atomicAdd(&cs->nF.v, (unsigned long long)__popc(am));
   } else if (lane == 31) {
-    if (deg) atomicAdd(&cs->arcsF, deg);
+    if (deg) atomicAdd(&cs->arcsF.v, deg);
   }
   // sub-CTA classes and fragments
 #pragma unroll
@@ -241,7 +338,9 @@ __device__ __forceinline__ void enqueue_warp(bool active, int v, long long b, lo
 }
 
 // enqueue_warp for vertex ids only: loads the rows first (one round of loads for the warp).
-__device__ __forceinline__ void enqueue_ids(bool active, int v, const long long *__restrict__ off,
+// Not inlined: it is the cold path of the consumer (once per 32 filtered-in vertices) and
+// inlining it at every call site multiplies the kernel's code size (I-cache misses).
+static __device__ __noinline__ void enqueue_ids(bool active, int v, const long long *__restrict__ off,
                                             const Ladder &L, const Queues &Q, CounterSet *cs) {
   long long b = 0, e = 0;
   if (active) {
@@ -261,6 +360,15 @@ struct WarpScratch {
   int buf[64];
 };
 
+#ifdef SAGE_PROF
+__device__ unsigned long long g_prof[16];
+#define PROF_T(x) long long x = clock64()
+#define PROF_ADD(i, v) if (lane_id() == 0) atomicAdd(&g_prof[i], (unsigned long long)(v))
+#else
+#define PROF_T(x)
+#define PROF_ADD(i, v)
+#endif
+
 // Append the lanes' filtered-in vertices to the warp buffer; flush full batches of 32.
 __device__ __forceinline__ void buffer_push(bool in, int v, WarpScratch *ws, int &cnt,
                                             const long long *__restrict__ off, const Ladder &L,
@@ -271,6 +379,7 @@ __device__ __forceinline__ void buffer_push(bool in, int v, WarpScratch *ws, int
   if (in) ws->buf[cnt + __popc(m & lanemask_lt())] = v;
   cnt += __popc(m);
   if (cnt >= 32) {
+    PROF_T(tf0);
     __syncwarp();
     const int x = ws->buf[lane];
     const int y = ws->buf[32 + lane];
@@ -279,6 +388,9 @@ __device__ __forceinline__ void buffer_push(bool in, int v, WarpScratch *ws, int
     if ((int)lane < cnt) ws->buf[lane] = y;
     __syncwarp();
     enqueue_ids(true, x, off, L, Q, cs);
+    PROF_T(tf1);
+    PROF_ADD(0, tf1 - tf0);
+    PROF_ADD(1, 1);
   }
 }
 __device__ __forceinline__ void buffer_flush(WarpScratch *ws, int &cnt,
@@ -316,24 +428,39 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
                                             CounterSet *cs, const long long *__restrict__ off,
                                             const int *__restrict__ col,
                                             const uint32_t *__restrict__ w, WarpScratch *ws,
-                                            typename F::Src *fsrc) {
+                                            typename F::Src *fsrc, bool vec_ok) {
   const unsigned lane = lane_id();
+  const unsigned long long pol = policy_evict_first();
+  const long long gwarp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
+  // all queue sizes in one round of loads (lane c holds cnt[c])
+  const unsigned long long my_cnt = (int)lane <= L.ncls ? ldcg(&cs->cnt[lane].v) : 0ull;
   int bcnt = 0;   // warp-uniform fill of ws->buf
   for (int c = 0; c < L.ncls; ++c) {
     const int t = L.B >> c;
-    const unsigned long long count = ldcg(&cs->cnt[c]);
+    const unsigned long long count = shfl64(my_cnt, c);
     if (count == 0) continue;
     const int lpt = (t / VEC) < 32 ? (t / VEC) : 32;  // lanes per tile
     const int tps = 32 / lpt;                           // tiles per warp step
     const int spt = (t / VEC) > 32 ? (t / (32 * VEC)) : 1;  // steps per tile
-    // batch ≈ 4 KB of column data per ticket
-    int batch = 1024 / t;
-    if (batch < tps) batch = tps;
+    // adaptive ticket batch: ~2 grabs per warp, <= 16 KB of columns per grab; warps beyond the
+    // number of grabs skip the class (no ticket traffic on small levels)
+    unsigned long long batch = (count + 2 * nwarps - 1) / (2 * nwarps);
+    const unsigned long long bmax = (4096 / t) > (unsigned)tps ? (4096 / t) : tps;
+    if (batch > bmax) batch = bmax;
+    batch = ((batch + tps - 1) / tps) * tps;
+    const unsigned long long grabs = (count + batch - 1) / batch;
+    if ((unsigned long long)gwarp >= grabs) continue;
     const int sub = lane / lpt, sl = lane % lpt;
+    const bool contiguous = lpt < 32 && vec_ok && VEC == 4;
     for (;;) {
+      PROF_T(tt0);
       unsigned long long base = 0;
-      if (lane == 0) base = atomicAdd(&cs->tk[c], (unsigned long long)batch);
+      if (lane == 0) base = atomicAdd(&cs->tk[c].v, batch);
       base = shfl64(base, 0);
+      PROF_T(tt1);
+      PROF_ADD(5, tt1 - tt0);
+      PROF_ADD(6, 1);
       if (base >= count) break;
       const unsigned long long end = (base + batch < count) ? base + batch : count;
       for (unsigned long long i = base; i < end; i += tps) {
@@ -359,32 +486,62 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
           }
         }
         const typename F::Src sc = f.src(valid, u, rb, re);
-        for (int s = 0; s < spt; ++s) {
-          const long long p0 = start + (long long)s * (lpt * VEC) + sl;
+        PROF_T(tv0);
+        if (contiguous) {
+          // sub-warp tiles: each lane reads VEC consecutive elements (one 16-B load)
+          const long long p0 = start + (long long)sl * VEC;
           int v[VEC];
           uint32_t ww[VEC];
-#pragma unroll
-          for (int j = 0; j < VEC; ++j) {
-            v[j] = valid ? ld_stream1(col + p0 + j * lpt) : 0;
-            ww[j] = (valid && F::kWeights) ? ld_stream1u(w + p0 + j * lpt) : 0u;
+          int4 c4 = make_int4(0, 0, 0, 0);
+          uint4 w4 = make_uint4(0, 0, 0, 0);
+          if (valid) {
+            c4 = ld_col4(col + p0, pol);
+            if (F::kWeights) w4 = ld_col4u(w + p0, pol);
           }
+          v[0] = c4.x; v[1 % VEC] = c4.y; v[2 % VEC] = c4.z; v[3 % VEC] = c4.w;
+          ww[0] = w4.x; ww[1 % VEC] = w4.y; ww[2 % VEC] = w4.z; ww[3 % VEC] = w4.w;
           bool in[VEC];
           f.template visit<VEC>(valid, sc, v, ww, in);
+          PROF_T(tv1);
+          PROF_ADD(2, tv1 - tv0);
           if constexpr (F::kEnqueue) {
 #pragma unroll
             for (int j = 0; j < VEC; ++j)
               buffer_push(in[j], v[j], ws, bcnt, off, L, *f.next_q, f.next_cs);
+          }
+        } else {
+          // strided: lane sl reads elements sl, sl+lpt, ... (coalesced, consecutive per load)
+          for (int s = 0; s < spt; ++s) {
+            const long long p0 = start + (long long)s * (lpt * VEC) + sl;
+            int v[VEC];
+            uint32_t ww[VEC];
+#pragma unroll
+            for (int j = 0; j < VEC; ++j) {
+              v[j] = valid ? ld_col(col + p0 + j * lpt, pol) : 0;
+              ww[j] = (valid && F::kWeights) ? ld_colu(w + p0 + j * lpt, pol) : 0u;
+            }
+            bool in[VEC];
+            f.template visit<VEC>(valid, sc, v, ww, in);
+            PROF_T(tv2);
+            PROF_ADD(3, tv2 - tv0);
+            PROF_ADD(4, 1);
+            if constexpr (F::kEnqueue) {
+#pragma unroll
+              for (int j = 0; j < VEC; ++j)
+                buffer_push(in[j], v[j], ws, bcnt, off, L, *f.next_q, f.next_cs);
+            }
           }
         }
       }
     }
   }
   // ---- fragments: warp scan-based gather
-  const unsigned long long fcount = ldcg(&cs->cnt[L.ncls]);
+  const unsigned long long fcount = shfl64(my_cnt, L.ncls);
+  const unsigned long long fgrabs = (fcount + 31) / 32;
   for (;;) {
-    if (fcount == 0) break;
+    if (fcount == 0 || (unsigned long long)gwarp >= fgrabs) break;
     unsigned long long base = 0;
-    if (lane == 0) base = atomicAdd(&cs->tk[L.ncls], 32ull);
+    if (lane == 0) base = atomicAdd(&cs->tk[L.ncls].v, 32ull);
     base = shfl64(base, 0);
     if (base >= fcount) break;
     const bool valid = base + lane < fcount;
@@ -434,8 +591,8 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
       if (kv) {
         const int idx = k - ws->pre[o];
         const long long pos = idx < ws->hl[o] ? ws->hb[o] + idx : ws->tb[o] + (idx - ws->hl[o]);
-        vv[0] = ld_stream1(col + pos);
-        if (F::kWeights) w1[0] = ld_stream1u(w + pos);
+        vv[0] = ld_col(col + pos, pol);
+        if (F::kWeights) w1[0] = ld_colu(w + pos, pol);
       }
       bool in[1];
       f.template visit<1>(kv, so, vv, w1, in);

@@ -65,7 +65,8 @@ struct sage_graph {
   int64_t n_isolated = 0;
   sage::Ladder ladder{};
   double alpha = 15.0, beta = 18.0;
-  int vec = 4;                // 4 = int4 column loads, 1 = scalar (paper mode / unaligned)
+  int vec = 4;                // neighbours per lane per step (4; 1 when tile_min < 4)
+  bool vec_ok = true;         // sub-warp tiles use 16-B loads (align % 4 == 0, aligned arrays)
   // reordering: sigma[v_orig] = current label; sigma_inv[label] = v_orig (null = identity)
   int32_t *sigma = nullptr, *sigma_inv = nullptr;
   bool reordered = false;

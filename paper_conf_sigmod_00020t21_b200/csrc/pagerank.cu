@@ -57,6 +57,7 @@ struct PrArgs {
   long long n_dangling;
   double *x, *y;
   Ctl *ctl;
+  int vec_ok;
 };
 
 // Build the all-V resident log: one thread per vertex, warp-aggregated classification.
@@ -95,7 +96,6 @@ __global__ void k_pr_init(double *x, double *y, long long n, double v0) {
 
 template <int VEC>
 __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ PrArgs a) {
-  cg::grid_group grid = cg::this_grid();
   __shared__ WarpScratch wsm[kWarps];
   __shared__ PrPush::Src fsrc[kWarps][32];
   __shared__ double red[kWarps];
@@ -107,13 +107,13 @@ __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ 
   for (int it = 0; it < a.iters; ++it) {
     CounterSet *cs = &a.sets[it % 3];
     __syncthreads();
-    if (blockIdx.x == 0 && threadIdx.x < kQueues) a.sets[(it + 2) % 3].tk[threadIdx.x] = 0ull;
+    if (blockIdx.x == 0 && threadIdx.x < kQueues) a.sets[(it + 2) % 3].tk[threadIdx.x].v = 0ull;
     if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->D[(it + 2) % 3] = 0.0;
     // push phase over the resident log
     PrPush f;
     f.x = a.x;
     f.y = a.y;
-    consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &wsm[warp], fsrc[warp]);
+    consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &wsm[warp], fsrc[warp], a.vec_ok);
     // dangling mass of this iteration's x
     double dsum = 0.0;
     for (long long i = tid; i < a.n_dangling; i += stride) dsum += ldcg(a.x + a.dangling[i]);
@@ -125,7 +125,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ 
       for (int k = 0; k < kWarps; ++k) s += red[k];
       if (s != 0.0) atomicAdd(&a.ctl->D[it % 3], s);
     }
-    grid.sync();
+    grid_barrier(&a.ctl->bar);
     // finalize: x = (1-d)/N + d*(y + D/N); y = 0
     const double D = ldcg(&a.ctl->D[it % 3]);
     const double add = base + a.d * D / a.N;
@@ -134,7 +134,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ 
       a.x[v] = add + a.d * yv;
       a.y[v] = 0.0;
     }
-    grid.sync();
+    grid_barrier(&a.ctl->bar);
   }
 }
 
@@ -173,13 +173,13 @@ sage_status ensure_pagerank_log(sage_graph *g) {
   // replicate the counts into the two other rotating sets
   cudaMemcpyAsync(p.cs + 1, p.cs, sizeof(CounterSet), cudaMemcpyDeviceToDevice, g->stream);
   cudaMemcpyAsync(p.cs + 2, p.cs, sizeof(CounterSet), cudaMemcpyDeviceToDevice, g->stream);
-  CounterSet h;
+  static CounterSet h;
   unsigned long long hnd = 0;
   cudaMemcpyAsync(&h, p.cs, sizeof(h), cudaMemcpyDeviceToHost, g->stream);
   cudaMemcpyAsync(&hnd, nd, sizeof(hnd), cudaMemcpyDeviceToHost, g->stream);
   cudaError_t e = cudaStreamSynchronize(g->stream);
   if (e != cudaSuccess) return cuda_fail(g, e, "PageRank log build");
-  memcpy(p.cnt, h.cnt, sizeof(p.cnt));
+  for (int i = 0; i < kQueues; ++i) p.cnt[i] = h.cnt[i].v;
   p.n_dangling = (long long)hnd;
   p.valid = true;
   return SAGE_OK;
@@ -235,6 +235,7 @@ extern "C" sage_status sage_pagerank(sage_graph *g, double damping, int32_t iter
   a.x = p.x;
   a.y = p.y;
   a.ctl = g->ts.ctl;
+  a.vec_ok = g->vec_ok ? 1 : 0;
   if (iterations > 0) {
     const void *fn = g->vec == 4 ? (const void *)k_pagerank<4> : (const void *)k_pagerank<1>;
     const int grid = coop_grid(g, fn, &g->grid_pr);

@@ -51,8 +51,9 @@ struct BfsPush {
   __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
                                         const uint32_t (&)[N], bool (&in)[N]) const {
     uint32_t wd[N];
+    const unsigned long long keep = policy_evict_last();
 #pragma unroll
-    for (int j = 0; j < N; ++j) wd[j] = valid ? visited[v[j] >> 5] : 0xffffffffu;
+    for (int j = 0; j < N; ++j) wd[j] = valid ? ld_status(visited + (v[j] >> 5), keep) : 0xffffffffu;
 #pragma unroll
     for (int j = 0; j < N; ++j) {
       const uint32_t bit = 1u << (v[j] & 31);
@@ -92,8 +93,9 @@ struct SsspPush {
   __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
                                         const uint32_t (&w)[N], bool (&in)[N]) const {
     uint32_t cur[N];
+    const unsigned long long keep = policy_evict_last();
 #pragma unroll
-    for (int j = 0; j < N; ++j) cur[j] = valid ? dist[v[j]] : 0u;
+    for (int j = 0; j < N; ++j) cur[j] = valid ? ld_status(dist + v[j], keep) : 0u;
 #pragma unroll
     for (int j = 0; j < N; ++j) {
       in[j] = false;
@@ -130,6 +132,7 @@ struct TravArgs {
   uint32_t *dist;
   Ctl *ctl;
   int do_enabled;       // direction switching allowed
+  int vec_ok;           // 16-B vector loads allowed (A % 4 == 0 and 16-B aligned col / w)
   double alpha, beta;
   int max_levels;
 };
@@ -182,15 +185,15 @@ __device__ __forceinline__ void pull_level(const TravArgs &a, int next_level, co
   insp = warp_sum64(insp);
   scanned = warp_sum64(scanned);
   if (lane == 0) {
-    if (insp) atomicAdd(&cur->inspected, insp);
-    if (scanned) atomicAdd(&cur->scanned, scanned);
+    if (insp) atomicAdd(&cur->inspected.v, insp);
+    if (scanned) atomicAdd(&cur->scanned.v, scanned);
   }
 }
 
 __device__ __forceinline__ void zero_counterset(CounterSet *s) {
-  constexpr int words = sizeof(CounterSet) / 8;
-  if (blockIdx.x == 0 && threadIdx.x < words)
-    reinterpret_cast<unsigned long long *>(s)[threadIdx.x] = 0ull;
+  constexpr int nctr = sizeof(CounterSet) / sizeof(PaddedCounter);
+  if (blockIdx.x == 0 && threadIdx.x < nctr)
+    reinterpret_cast<PaddedCounter *>(s)[threadIdx.x].v = 0ull;
 }
 
 __device__ __forceinline__ void clear_words(uint32_t *p, long long nwords) {
@@ -202,9 +205,9 @@ __device__ __forceinline__ void clear_words(uint32_t *p, long long nwords) {
 // Record level L's statistics (single thread).
 __device__ __forceinline__ void record_level(Ctl *ctl, int L, int dir, const CounterSet *cur,
                                              const CounterSet *nxt) {
-  const unsigned long long nF = ldcg(&cur->nF), aF = ldcg(&cur->arcsF);
-  const unsigned long long disc = ldcg(&nxt->nF), aN = ldcg(&nxt->arcsF);
-  const unsigned long long insp = ldcg(&cur->inspected), sc = ldcg(&cur->scanned);
+  const unsigned long long nF = ldcg(&cur->nF.v), aF = ldcg(&cur->arcsF.v);
+  const unsigned long long disc = ldcg(&nxt->nF.v), aN = ldcg(&nxt->arcsF.v);
+  const unsigned long long insp = ldcg(&cur->inspected.v), sc = ldcg(&cur->scanned.v);
   if (dir == 0) {
     ctl->tot_push_expanded += nF;
     ctl->tot_push_arcs += aF;
@@ -226,6 +229,7 @@ __device__ __forceinline__ void record_level(Ctl *ctl, int L, int dir, const Cou
     r.inspected = dir == 0 ? aF : insp;
     r.scanned = sc;
     r.discovered = disc;
+    r.t_ns = globaltimer();
   }
   ctl->levels = L + 1;
 }
@@ -233,12 +237,12 @@ __device__ __forceinline__ void record_level(Ctl *ctl, int L, int dir, const Cou
 // ============================================================================ BFS kernel
 template <int VEC>
 __global__ void __launch_bounds__(kBlock, 4) k_bfs(const __grid_constant__ TravArgs a) {
-  cg::grid_group grid = cg::this_grid();
   __shared__ WarpScratch wsm[kWarps];
   __shared__ BfsPush::Src fsrc[kWarps][32];
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
-  double mU = (double)a.m - (double)ldcg(&ctl->set[0].arcsF);
+  double mU = (double)a.m - (double)ldcg(&ctl->set[0].arcsF.v);
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t0_ns = globaltimer();
   int dir = 0;
   unsigned long long prev_nF = 1;
   const long long nwords = (a.n + 31) >> 5;
@@ -259,13 +263,14 @@ __global__ void __launch_bounds__(kBlock, 4) k_bfs(const __grid_constant__ TravA
       f.v_base = 0;
       f.next_q = &a.q[(L + 1) & 1];
       f.next_cs = nxt;
-      consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp]);
+      consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok);
     } else {
       pull_level(a, L + 1, fbc, fbn, a.q[(L + 1) & 1], cur, nxt, &wsm[warp]);
     }
-    grid.sync();
-    const unsigned long long nF = ldcg(&nxt->nF);
-    const unsigned long long aF = ldcg(&nxt->arcsF);
+    if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
+    grid_barrier(&ctl->bar);
+    const unsigned long long nF = ldcg(&nxt->nF.v);
+    const unsigned long long aF = ldcg(&nxt->arcsF.v);
     if (blockIdx.x == 0 && threadIdx.x == 0) record_level(ctl, L, dir, cur, nxt);
     if (nF == 0) break;
     if (L + 1 >= a.max_levels) {
@@ -287,12 +292,12 @@ __global__ void __launch_bounds__(kBlock, 4) k_bfs(const __grid_constant__ TravA
 // ============================================================================ SSSP kernel
 template <int VEC>
 __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ TravArgs a, int *overflow) {
-  cg::grid_group grid = cg::this_grid();
   __shared__ WarpScratch wsm[kWarps];
   __shared__ SsspPush::Src fsrc[kWarps][32];
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
   const long long nwords = (a.n + 31) >> 5;
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t0_ns = globaltimer();
   for (int L = 0;; ++L) {
     CounterSet *cur = &ctl->set[L % 3];
     CounterSet *nxt = &ctl->set[(L + 1) % 3];
@@ -305,9 +310,10 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
     f.overflow = overflow;
     f.next_q = &a.q[(L + 1) & 1];
     f.next_cs = nxt;
-    consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp]);
-    grid.sync();
-    const unsigned long long nF = ldcg(&nxt->nF);
+    consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok);
+    if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
+    grid_barrier(&ctl->bar);
+    const unsigned long long nF = ldcg(&nxt->nF.v);
     if (blockIdx.x == 0 && threadIdx.x == 0) record_level(ctl, L, 0, cur, nxt);
     if (nF == 0) break;
     if (L + 1 >= a.max_levels) {
@@ -417,20 +423,20 @@ __global__ void k_expand_log(const long long *__restrict__ off, Ladder L, Queues
       quads[4 * k + 3] = kind;
     }
   };
-  for (long long i = tid; i < (long long)cs->cnt[0]; i += stride) {
+  for (long long i = tid; i < (long long)cs->cnt[0].v; i += stride) {
     CtaTile T = Q.cta[i];
     emit(T.u, T.start, T.len, 0);
   }
   for (int c = 1; c < L.ncls; ++c) {
     const int t = L.B >> c;
-    for (long long i = tid; i < (long long)cs->cnt[c]; i += stride) {
+    for (long long i = tid; i < (long long)cs->cnt[c].v; i += stride) {
       const int u = Q.cls[c][i];
       const long long b = off[u], e = off[u + 1];
       RowSplit s = split_row(b, e, L);
       emit(u, class_tile_start(e, s.r, t), t, 0);
     }
   }
-  for (long long i = tid; i < (long long)cs->cnt[L.ncls]; i += stride) {
+  for (long long i = tid; i < (long long)cs->cnt[L.ncls].v; i += stride) {
     const int u = Q.frag[i];
     const long long b = off[u], e = off[u + 1];
     RowSplit s = split_row(b, e, L);
@@ -567,6 +573,7 @@ static TravArgs make_args(sage_graph *g) {
   a.alpha = g->alpha;
   a.beta = g->beta;
   a.max_levels = (int)std::min<long long>(g->n + 1, 0x7fffffffll);
+  a.vec_ok = g->vec_ok ? 1 : 0;
   return a;
 }
 
@@ -651,7 +658,7 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   if (parent_out) cudaMemsetAsync(t.parent, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
   cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
   for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
-  cudaMemsetAsync(t.ctl, 0, offsetof(Ctl, rec), g->stream);
+  cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);
   TravArgs a = make_args(g);
   a.parent = parent_out ? t.parent : nullptr;
   a.do_enabled = (symmetric && !push_only) ? 1 : 0;
@@ -724,7 +731,7 @@ extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_o
   cudaMemsetAsync(t.dist, 0xff, sizeof(uint32_t) * (size_t)g->n_local, g->stream);
   cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
   for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
-  cudaMemsetAsync(t.ctl, 0, offsetof(Ctl, rec), g->stream);
+  cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);
   TravArgs a = make_args(g);
   k_seed<<<1, 32, 0, g->stream>>>(a, src, 1);
   cudaEventRecord(e1, g->stream);
@@ -847,3 +854,51 @@ extern "C" sage_status sage_debug_export_tiles(sage_graph *g, const int32_t *ver
   if (e != cudaSuccess) return cuda_fail(g, e, "debug_export_tiles");
   return SAGE_OK;
 }
+
+extern "C" sage_status sage_debug_level_records(const sage_graph *gc, int64_t *rec_out, int32_t cap,
+                                                int32_t *n_out) {
+  // 8 int64 per level (the 8th = device time at which the last warp finished the level's work)
+  clear_error();
+  sage_graph *g = const_cast<sage_graph *>(gc);
+  if (!g || !n_out || (cap > 0 && !rec_out)) {
+    set_error("null argument");
+    return SAGE_E_INVALID;
+  }
+  if (!g->ts.ready) {
+    *n_out = 0;
+    return SAGE_OK;
+  }
+  Ctl *h = new Ctl;
+  cudaError_t e = cudaMemcpy(h, g->ts.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) {
+    delete h;
+    return cuda_fail(g, e, "level records");
+  }
+  const int nl = std::min(h->levels, kMaxRec);
+  *n_out = h->levels;
+  for (int i = 0; i < nl && i < cap; ++i) {
+    const LevelRec &r = h->rec[i];
+    int64_t *o = rec_out + 8 * i;
+    o[0] = r.dir;
+    o[1] = (int64_t)r.nF;
+    o[2] = (int64_t)r.arcsF;
+    o[3] = (int64_t)r.inspected;
+    o[4] = (int64_t)r.scanned;
+    o[5] = (int64_t)r.discovered;
+    o[6] = (int64_t)(r.t_ns - h->t0_ns);
+    o[7] = r.t_work ? (int64_t)(r.t_work - h->t0_ns) : 0;
+  }
+  delete h;
+  return SAGE_OK;
+}
+
+#ifdef SAGE_PROF
+extern "C" int sage_prof_read(unsigned long long *out16, int reset) {
+  cudaMemcpyFromSymbol(out16, sage::g_prof, sizeof(unsigned long long) * 16);
+  if (reset) {
+    unsigned long long z[16] = {0};
+    cudaMemcpyToSymbol(sage::g_prof, z, sizeof(z));
+  }
+  return 0;
+}
+#endif

@@ -71,15 +71,16 @@ def build_sage(force=False, verbose=False):
     csrc = os.path.join(PKG, "csrc")
     cus = sorted(glob.glob(os.path.join(csrc, "*.cu")))
     hdrs = sorted(glob.glob(os.path.join(csrc, "*.cuh"))) + [os.path.join(ROOT, "include", "sage.h")]
-    out = os.path.join(PKG, "libsage.so")
+    prof = os.environ.get("SAGE_PROF") == "1"
+    out = os.path.join(PKG, "libsage_prof.so" if prof else "libsage.so")
     if not (force or _stale(out, cus + hdrs)):
         return out
     nccl_inc, nccl_lib = _nccl_paths()
-    objdir = os.path.join(PKG, "build")
+    objdir = os.path.join(PKG, "build_prof" if prof else "build")
     os.makedirs(objdir, exist_ok=True)
     common = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC",
               "-I", os.path.join(ROOT, "include"), "-I", csrc, "-I", nccl_inc,
-              "--expt-relaxed-constexpr", "-Xptxas", "-v" if verbose else "-O3"]
+              "--expt-relaxed-constexpr", "-Xptxas", "-v" if verbose else "-O3"] + (["-DSAGE_PROF=1"] if prof else [])
     objs = []
     for cu in cus:
         obj = os.path.join(objdir, os.path.basename(cu)[:-3] + ".o")

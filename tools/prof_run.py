@@ -35,3 +35,18 @@ for i in range(a.reps):
         x = torch.empty(g.n, dtype=torch.float64, device="cuda")
         _, st = G.pagerank(0.85, 5, out=x)
     print(a.op, i, {k: st[k] for k in ("levels", "kernel_ms", "ms", "edges_traversed", "model_bytes")}, flush=True)
+    if a.op != "pr":
+        prev = 0
+        for r in G.level_records():
+            print("   L dir=%d |F|=%9d arcsF=%11d insp=%11d disc=%9d  %8.1f us (work done at +%8.1f)" % (
+                r[0], r[1], r[2], r[3], r[5], (r[6] - prev) / 1e3, (r[7] - prev) / 1e3))
+            prev = r[6]
+    if os.environ.get("SAGE_PROF") == "1":
+        import ctypes
+        buf = (ctypes.c_ulonglong * 16)()
+        sage.lib().sage_prof_read(buf, 1)
+        names = ["flush_cyc", "flushes", "visit_contig_cyc", "visit_strided_cyc", "strided_steps", "ticket_cyc", "tickets"]
+        d = {nm: buf[k] for k, nm in enumerate(names)}
+        print("   prof:", d, {"cyc/flush": d["flush_cyc"] / max(1, d["flushes"]),
+                               "cyc/strided_step": d["visit_strided_cyc"] / max(1, d["strided_steps"]),
+                               "cyc/ticket": d["ticket_cyc"] / max(1, d["tickets"])})

@@ -108,8 +108,8 @@ typedef struct {
 
 typedef struct {
   int32_t sector_width;        /* S: node ids per sector (R17); power of two; default 8             */
-  const int32_t *candidates;   /* optional (host) list of CURRENT labels allowed to move in the
-                                  first round (Fig. 5's "only consider node-8"); NULL = all   */
+  const int32_t *candidates;   /* optional (host) list of ORIGINAL vertex ids allowed to move, in
+                                  every round (Fig. 5's "only consider node-8"); NULL = all   */
   int64_t n_candidates;
 } sage_reorder_opts;
 
@@ -152,6 +152,11 @@ sage_status sage_pagerank(sage_graph *g, double damping, int32_t iterations, dou
 sage_status sage_reorder(sage_graph *g, int32_t rounds, const sage_reorder_opts *opt,
                          sage_stats *st);
 
+/* Objective of §6 on the current labels: the sum over the tile sample (every tile of
+ * every vertex under the graph's ladder, readings R19/R20) of the number of distinct sectors
+ * floor(label / sector_width) among the tile's members.  Lower = better locality.              */
+sage_status sage_reorder_objective(sage_graph *g, int32_t sector_width, int64_t *out);
+
 /* new_id_of_old[v] = current label of original vertex v (n entries; identity before reorder). */
 sage_status sage_get_permutation(const sage_graph *g, int32_t *new_id_of_old);
 
@@ -170,6 +175,13 @@ sage_status sage_graph_info(const sage_graph *g, int64_t *n, int64_t *m, int64_t
  * small nothing is written and *n_out is the required count.                                   */
 sage_status sage_debug_export_tiles(sage_graph *g, const int32_t *vertices, int64_t count,
                                     int64_t *quads_out, int64_t cap, int64_t *n_out);
+
+/* Test entry point: stages 1-3 of one reorder round on the current labels, without relabelling:
+ * per vertex (current labels) loc1, target sector, loc3 (int64, n each) and mover flag (uint8, n),
+ * host buffers.  candidates: optional ORIGINAL ids allowed to move.                              */
+sage_status sage_debug_reorder_stages(sage_graph *g, int32_t sector_width, const int32_t *candidates,
+                                      int64_t n_candidates, int64_t *loc1_out, int64_t *target_out,
+                                      int64_t *loc3_out, uint8_t *mover_out);
 
 /* Diagnostic entry point: per-level records of the last BFS / SSSP query on this graph, 8 int64 per
  * level: direction (0 push, 1 pull), |F|, arcs(F), arcs inspected, vertices scanned (pull),

@@ -24,8 +24,8 @@ STATUS_NAMES = {0: "SAGE_OK", 1: "SAGE_E_INVALID", 2: "SAGE_E_NOMEM", 3: "SAGE_E
                 4: "SAGE_E_NCCL", 5: "SAGE_E_OVERFLOW", 6: "SAGE_E_UNSUPPORTED"}
 
 EXPORTED = ["sage_load_csr", "sage_free", "sage_bfs", "sage_bfs_ex", "sage_sssp", "sage_pagerank",
-            "sage_reorder", "sage_get_permutation", "sage_get_csr", "sage_graph_info",
-            "sage_debug_export_tiles", "sage_debug_level_records", "sage_last_error", "sage_version"]
+            "sage_reorder", "sage_reorder_objective", "sage_get_permutation", "sage_get_csr", "sage_graph_info",
+            "sage_debug_export_tiles", "sage_debug_reorder_stages", "sage_debug_level_records", "sage_last_error", "sage_version"]
 
 
 class SageError(RuntimeError):
@@ -86,6 +86,8 @@ def lib():
         L.sage_pagerank.argtypes = [p, dbl, i32, p, ctypes.POINTER(Stats)]
         L.sage_reorder.argtypes = [p, i32, ctypes.POINTER(ReorderOpts), ctypes.POINTER(Stats)]
         L.sage_get_permutation.argtypes = [p, p]
+        L.sage_reorder_objective.argtypes = [p, i32, p]
+        L.sage_debug_reorder_stages.argtypes = [p, i32, p, i64, p, p, p, p]
         L.sage_get_csr.argtypes = [p, p, p, p]
         L.sage_graph_info.argtypes = [p, p, p, p, p, p]
         L.sage_debug_export_tiles.argtypes = [p, p, i64, p, i64, p]
@@ -220,6 +222,25 @@ class Graph:
         st = Stats()
         _check(lib().sage_reorder(self._h, int(rounds), ctypes.byref(ro), ctypes.byref(st)))
         return st.as_dict()
+
+    def objective(self, sector_width: int = 8) -> int:
+        """sage_reorder_objective: sum over sampled tiles of distinct sectors."""
+        out = ctypes.c_int64(0)
+        _check(lib().sage_reorder_objective(self._h, int(sector_width), ctypes.byref(out)))
+        return out.value
+
+    def reorder_stages(self, sector_width: int = 8, candidates=None) -> dict:
+        """sage_debug_reorder_stages -> {loc1, target, loc3, mover} of one round (no relabel)."""
+        n = self.n
+        out = {k: np.zeros(n, dtype=np.int64) for k in ("loc1", "target", "loc3")}
+        mover = np.zeros(n, dtype=np.uint8)
+        c = None if candidates is None else np.ascontiguousarray(candidates, dtype=np.int32)
+        _check(lib().sage_debug_reorder_stages(self._h, int(sector_width), c.ctypes.data if c is not None else None,
+                                               0 if c is None else len(c), out["loc1"].ctypes.data,
+                                               out["target"].ctypes.data, out["loc3"].ctypes.data,
+                                               mover.ctypes.data))
+        out["mover"] = mover
+        return out
 
     def permutation(self) -> np.ndarray:
         out = np.empty(self.n, dtype=np.int32)

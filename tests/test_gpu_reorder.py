@@ -1,0 +1,149 @@
+"""GPU parity of Sampling-based Reordering (§6) against the oracle.
+
+Every count of the three stages is an integer and every tie-break is fixed (DESIGN.md readings
+R17-R25), so the GPU's stage vectors, permutation and relabelled CSR must equal the oracle's
+exactly; queries after reordering must return the same answers in original ids.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import sagegen as sg
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def sage():
+    import torch
+    assert torch.cuda.is_available()
+    from __graft_entry__ import build
+    build()
+    import paper_conf_sigmod_00020t21_b200 as s
+    return s
+
+
+def _fig5(golden_dir):
+    fx = json.load(open(os.path.join(golden_dir, "fig5_reorder.json")))
+    owners = [6, 7, 11, 13]
+    edges = [(o, v) for o, t in zip(owners, fx["tiles"]) for v in t]
+    return fx, sg.from_edges(fx["n"], edges)
+
+
+def test_figure5_stages_on_device(sage, golden_dir):
+    fx, g = _fig5(golden_dir)
+    with sage.load_csr(g.off, g.col, tile_cta=4, tile_min=4, align=0) as G:
+        st = G.reorder_stages(fx["S"], candidates=[8])
+        assert st["loc1"].tolist() == fx["stage1_locality"]
+        assert st["target"][8] == fx["node8_target_sector"]
+        assert st["loc3"][8] == fx["node8_loc3"]
+        assert st["mover"].nonzero()[0].tolist() == [8]
+        assert G.objective(fx["S"]) == fx["objective_round1"]
+        full = G.reorder_stages(fx["S"])
+        assert full["mover"].nonzero()[0].tolist() == fx["reading_full_run"]["movers"]
+
+
+def test_figure5_round_on_device(sage, golden_dir):
+    fx, g = _fig5(golden_dir)
+    with sage.load_csr(g.off, g.col, tile_cta=4, tile_min=4, align=0) as G:
+        st = G.reorder(1, sector_width=fx["S"], candidates=[8])
+        sigma = G.permutation()
+        assert sigma[8] == fx["node8_only_new_label"] and sigma[3] == 8
+        assert st["vertices_discovered"] == 1        # one swap
+        off2, col2, _ = G.csr()
+        tiles = sorted(sorted(col2[off2[u]:off2[u + 1]].tolist()) for u in range(g.n) if off2[u + 1] > off2[u])
+        assert tiles == sorted(fx["round2_tiles_node8_only"])
+        assert G.objective(fx["S"]) == fx["objective_round2_node8_only"]
+    with sage.load_csr(g.off, g.col, tile_cta=4, tile_min=4, align=0) as G:
+        G.reorder(1, sector_width=fx["S"])
+        sigma = G.permutation()
+        pairs = sorted(tuple(sorted((v, int(sigma[v])))) for v in range(g.n) if sigma[v] != v)
+        assert sorted(set(pairs)) == [tuple(p) for p in fx["reading_full_run"]["swaps"]]
+        assert G.objective(fx["S"]) == fx["reading_full_run"]["objective_after"]
+
+
+CASES = [dict(scale=11, sym=True, B=256, M=8, A=4, S=8),
+         dict(scale=12, sym=False, B=32, M=8, A=4, S=8),
+         dict(scale=11, sym=True, B=64, M=4, A=0, S=32),
+         dict(scale=10, sym=False, B=16, M=8, A=0, S=4)]
+
+
+@pytest.mark.parametrize("case", CASES, ids=lambda c: "s{scale}{sym}B{B}M{M}A{A}S{S}".format(**c))
+def test_stage_vectors_equal_oracle(sage, case):
+    g = sg.rmat(case["scale"], 16, seed=5, symmetric=case["sym"])
+    tp, mem = oracle.sample_tiles(g.off, g.col, case["B"], case["M"], case["A"])
+    ref = oracle.reorder_stages(g.n, tp, mem, case["S"])
+    with sage.load_csr(g.off, g.col, tile_cta=case["B"], tile_min=case["M"], align=case["A"]) as G:
+        got = G.reorder_stages(case["S"])
+        assert G.objective(case["S"]) == oracle.objective_tiles(tp, mem, case["S"])
+    for k in ("loc1", "target", "loc3"):
+        assert np.array_equal(got[k], ref[k]), k
+    assert np.array_equal(got["mover"], ref["mover"])
+
+
+def test_unsorted_rows_stage_vectors(sage):
+    """Rows in arbitrary order: the GPU sorts each tile in shared memory; counts are per tile."""
+    g = sg.rmat(11, 16, seed=8, symmetric=False)
+    rng = np.random.default_rng(1)
+    col = g.col.copy()
+    for u in range(g.n):
+        rng.shuffle(col[g.off[u]:g.off[u + 1]])
+    tp, mem = oracle.sample_tiles(g.off, col, 64, 8, 4)
+    ref = oracle.reorder_stages(g.n, tp, mem, 8)
+    with sage.load_csr(g.off, col, tile_cta=64, tile_min=8, align=4) as G:
+        assert not G.rows_sorted
+        got = G.reorder_stages(8)
+    for k in ("loc1", "target", "loc3"):
+        assert np.array_equal(got[k], ref[k]), k
+
+
+@pytest.mark.parametrize("case", CASES[:3], ids=lambda c: "s{scale}{sym}B{B}M{M}A{A}S{S}".format(**c))
+def test_reorder_rounds_equal_oracle(sage, case):
+    g = sg.rmat(case["scale"], 16, seed=7, symmetric=case["sym"])
+    w = sg.weights(g, 2)
+    rounds = 3
+    off2, col2, w2, sigma, info = oracle.reorder(g.off, g.col, w, rounds=rounds, B=case["B"], M=case["M"],
+                                                 A=case["A"], S=case["S"])
+    with sage.load_csr(g.off, g.col, w, symmetric=case["sym"], tile_cta=case["B"], tile_min=case["M"],
+                       align=case["A"]) as G:
+        st = G.reorder(rounds, sector_width=case["S"])
+        assert st["levels"] == len(info)
+        assert np.array_equal(G.permutation(), sigma)
+        o, c, ww = G.csr()
+        assert np.array_equal(o, off2) and np.array_equal(c, col2) and np.array_equal(ww, w2)
+        # queries after reordering: original ids, unchanged answers
+        for s in sg.sources(g, 3, seed=2):
+            s = int(s)
+            lv, par, _ = G.bfs(s, parents=True)
+            ref = oracle.bfs(g.off, g.col, s)
+            assert np.array_equal(lv, ref)
+            ok = lv > 0
+            assert np.all(ref[par[ok]] == ref[ok] - 1)
+            d, _ = G.sssp(s)
+            assert np.array_equal(d, oracle.sssp(g.off, g.col, w, s)[0])
+        x, _ = G.pagerank(0.85, 20)
+        xr = oracle.pagerank(g.off, g.col, 0.85, 20)
+        assert np.max(np.abs(x - xr) / xr) <= 1e-6
+
+
+def test_reorder_candidates_every_round(sage):
+    g = sg.rmat(11, 16, seed=3, symmetric=True)
+    cand = sg.sources(g, 200, seed=9)
+    off2, col2, _, sigma, info = oracle.reorder(g.off, g.col, None, rounds=2, candidates=cand)
+    with sage.load_csr(g.off, g.col, symmetric=True) as G:
+        G.reorder(2, candidates=cand)
+        assert np.array_equal(G.permutation(), sigma)
+
+
+def test_reorder_objective_improves_and_errors(sage):
+    g = sg.rmat(13, 16, seed=1, symmetric=True)
+    with sage.load_csr(g.off, g.col, symmetric=True) as G:
+        before = G.objective(8)
+        st = G.reorder(2)
+        assert st["vertices_discovered"] > 0 and G.objective(8) < before
+        with pytest.raises(sage.SageError) as ei:
+            G.reorder(1, sector_width=3)
+        assert ei.value.status == sage.E_INVALID

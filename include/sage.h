@@ -68,7 +68,7 @@ typedef struct {
 /* Tile ladder used by every kernel and by the reorder's sample (Alg. 2; readings
  * R9-R14 of DESIGN.md).  NULL = defaults.                                                      */
 typedef struct {
-  int32_t tile_cta;  /* B: largest ("CTA") tile, power of two in [8, 4096]; default 256   */
+  int32_t tile_cta;  /* B: largest ("CTA") tile, power of two in [1, 4096]; default 256   */
   int32_t tile_min;  /* M: MIN_TILE_SIZE, power of two in [1, B]; default 8 (Fig. 3)        */
   int32_t align;     /* A: tile alignment in elements: 0 = paper mode (no head fragment),
                         else a power of two in [1, 64]; default 4 (16 B, one int4 load)          */

@@ -125,8 +125,8 @@ static sage_status make_ladder(const sage_options *o, sage_graph *g) {
     alpha = o->alpha;
     beta = o->beta;
   }
-  if (!is_pow2(B) || B < 8 || B > 4096) {
-    set_error("tile_cta must be a power of two in [8, 4096]");
+  if (!is_pow2(B) || B > 4096) {
+    set_error("tile_cta must be a power of two in [1, 4096]");
     return SAGE_E_INVALID;
   }
   if (!is_pow2(M) || M > B || (B / M) > 4096) {

@@ -663,6 +663,7 @@ extern "C" sage_status sage_debug_reorder_stages(sage_graph *g, int32_t sector_w
   if (s == SAGE_OK) s = one_round(g, b, lgS, b.cand, &mv, &sw, true);
   if (s == SAGE_OK) {
     const size_t n = (size_t)g->n;
+    cudaStreamSynchronize(g->stream);   // the stages ran on the graph's (non-blocking) stream
     std::vector<unsigned long long> l1(n), l3(n);
     std::vector<int> tg(n);
     cudaMemcpy(l1.data(), b.loc1, 8 * n, cudaMemcpyDeviceToHost);

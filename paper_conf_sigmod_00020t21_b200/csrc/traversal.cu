@@ -814,6 +814,7 @@ extern "C" sage_status sage_debug_export_tiles(sage_graph *g, const int32_t *ver
   long long msum = 0;
   {
     std::vector<long long> hoff((size_t)g->n_local + 1);
+    cudaStreamSynchronize(g->stream);
     cudaMemcpy(hoff.data(), g->off, sizeof(long long) * hoff.size(), cudaMemcpyDeviceToHost);
     for (int64_t i = 0; i < count; ++i) msum += hoff[vertices[i] + 1] - hoff[vertices[i]];
   }
@@ -869,6 +870,7 @@ extern "C" sage_status sage_debug_level_records(const sage_graph *gc, int64_t *r
     return SAGE_OK;
   }
   Ctl *h = new Ctl;
+  cudaStreamSynchronize(g->stream);
   cudaError_t e = cudaMemcpy(h, g->ts.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost);
   if (e != cudaSuccess) {
     delete h;

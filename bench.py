@@ -301,15 +301,32 @@ def _extras(a, G, g, srcs, level, flush, stream, sage):
     ex["e2e"] = {"value": len(e2e) / sum(t * 1e9 / e for t, e in e2e), "unit": "GTEPS",
                  "h2d_bytes_per_step": int(g.off.nbytes + g.col.nbytes), "d2h_bytes_per_step": int(4 * g.n),
                  "includes": "sage_load_csr from pinned host CSR (copy + validation) + sage_bfs + level D2H"}
-    # timed CPU oracle on a bounded sample of the same workload
+    # timed CPU oracle on a bounded sample of the same workload (also the full-size parity check)
+    G.bfs(int(srcs[0]), out=level, push_only=True)
+    gpu_lv = level.cpu().numpy()
     t0 = time.perf_counter()
     lv = oracle.bfs(g.off, g.col, int(srcs[0]))
     dt = time.perf_counter() - t0
     e = int(np.diff(g.off)[lv >= 0].sum()) // 2
-    assert np.array_equal(lv, level.cpu().numpy()) or True
     ex["cpu_baseline"] = {"value": e / dt / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
                           "sample": "1 serial oracle BFS (oracle/oracle.c FIFO queue) from the first warm-up source",
                           "seconds": dt, "host_cpus": os.cpu_count()}
+    G.sssp(int(srcs[0]), out=dist)
+    ex["parity"] = {"bfs_levels_equal_oracle": bool(np.array_equal(lv, gpu_lv)),
+                    "sssp_certificate_ok": oracle.check_sssp(g.off, g.col, g.w, int(srcs[0]),
+                                                              dist.cpu().numpy().view(np.uint32)) == 0,
+                    "source": int(srcs[0])}
+    # one Sampling-based Reordering round on a copy of the graph (C3-style reorder on/off)
+    with sage.load_csr(torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda(), symmetric=True,
+                       stream=stream.cuda_stream) as H:
+        ob0 = H.objective(8)
+        _, _, b0 = H.bfs(int(srcs[1]), out=level, push_only=True)
+        st = H.reorder(1)
+        ob1 = H.objective(8)
+        _, _, b1 = H.bfs(int(srcs[1]), out=level, push_only=True)
+        ex["reorder"] = {"round_ms": st["ms"], "swaps": st["vertices_discovered"], "movers": st["vertices_expanded"],
+                         "objective_before": ob0, "objective_after": ob1,
+                         "bfs_push_ms_before": b0["kernel_ms"], "bfs_push_ms_after": b1["kernel_ms"]}
     return ex
 
 

@@ -34,6 +34,7 @@ def _lib():
         lib.ora_sssp.argtypes = [i64, p, p, p, i32, p]
         lib.ora_check_sssp.argtypes = [i64, p, p, p, i32, p]
         lib.ora_pagerank.argtypes = [i64, p, p, dbl, i32, p]
+        lib.ora_pagerank_step.argtypes = [i64, p, p, dbl, p, p]
         lib.ora_tiles_row.argtypes = [i64, i64, i32, i32, i32, p]
         lib.ora_tiles_row.restype = i64
         lib.ora_tile_log.argtypes = [p, p, i64, i32, i32, i32, p]
@@ -106,6 +107,18 @@ def pagerank(off, col, damping: float = 0.85, iters: int = 20) -> np.ndarray:
     if _lib().ora_pagerank(n, po, pc, float(damping), int(iters), x.ctypes.data) != 0:
         raise ValueError("empty graph")
     return x
+
+
+def pagerank_step(off, col, x, damping: float = 0.85) -> np.ndarray:
+    """One power-iteration step of c3 from the iterate ``x`` (same arithmetic as ``pagerank``)."""
+    off, po = _c(off, np.int64)
+    col, pc = _c(col, np.int32)
+    x, px = _c(x, np.float64)
+    n = len(off) - 1
+    out = np.empty(n, dtype=np.float64)
+    if _lib().ora_pagerank_step(n, po, pc, float(damping), px, out.ctypes.data) != 0:
+        raise ValueError("empty graph")
+    return out
 
 
 # ---------------------------------------------------------------- c4 tiles (Alg. 2/3, Fig. 3)

@@ -197,6 +197,27 @@ int ora_pagerank(int64_t n, const int64_t *off, const int32_t *col, double d, in
   return 0;
 }
 
+/* One iteration of c3 from a given iterate x (n doubles) -> x_next: the same three lines of the
+ * power iteration above (D, y, x update), so that a GPU result at full size can be checked vertex
+ * by vertex against x_K = step(x_{K-1}) without re-running the whole serial iteration.          */
+int ora_pagerank_step(int64_t n, const int64_t *off, const int32_t *col, double d, const double *x,
+                      double *x_next) {
+  if (n <= 0) return 1;
+  double *y = (double *)calloc((size_t)n, sizeof(double));
+  if (!y) return 2;
+  const double N = (double)n;
+  double D = 0.0;
+  for (int64_t u = 0; u < n; ++u) {
+    int64_t deg = off[u + 1] - off[u];
+    if (deg == 0) { D += x[u]; continue; }
+    double inc = x[u] / (double)deg;
+    for (int64_t k = off[u]; k < off[u + 1]; ++k) y[col[k]] += inc;
+  }
+  for (int64_t v = 0; v < n; ++v) x_next[v] = (1.0 - d) / N + d * (y[v] + D / N);
+  free(y);
+  return 0;
+}
+
 /* ===================================================================================== */
 /* c4. Tiled Partitioning of one row [b, e) — Alg. 2 as the resident tile log of
  * Alg. 3 l.2-7.  The block-sized tile consumes full tile-size chunks of the row

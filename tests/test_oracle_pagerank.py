@@ -79,3 +79,18 @@ def test_sums_to_one():
     x = oracle.pagerank(g.off, g.col, 0.85, 20)
     assert abs(x.sum() - 1.0) < 1e-12
     assert np.all(x >= 0.15 / g.n * (1 - 1e-12))
+
+
+def test_pagerank_step_composes_to_pagerank():
+    """pagerank_step applied K times from x0 = 1/N reproduces pagerank(K) bit for bit (same
+    arithmetic in the same order), and a hand-computed step on a 3-vertex graph."""
+    g = sg.rmat(9, 8, seed=4, symmetric=False)
+    x = np.full(g.n, 1.0 / g.n)
+    for _ in range(7):
+        x = oracle.pagerank_step(g.off, g.col, x, 0.85)
+    assert np.array_equal(x, oracle.pagerank(g.off, g.col, 0.85, 7))
+    h = sg.from_edges(3, [(0, 1), (0, 2), (1, 2)], False, "tri")     # vertex 2 dangles
+    x0 = np.array([0.5, 0.3, 0.2])
+    d = 0.85
+    exp = np.array([0.0, 0.5 / 2, 0.5 / 2 + 0.3]) * d + (1 - d) / 3 + d * 0.2 / 3
+    assert np.allclose(oracle.pagerank_step(h.off, h.col, x0, d), exp, rtol=0, atol=1e-15)

@@ -56,7 +56,10 @@ enum {
                               expansion (Alg. 2/3).  Can also be set per call (sage_bfs_ex).     */
 };
 
-/* Multi-GPU description (1D vertex partition).  NULL in sage_csr = single GPU.  */
+/* Multi-GPU description (1D vertex partition).  NULL in sage_csr = single GPU.
+ * Non-NULL selects the NCCL path (also with world == 1: a 1-rank communicator).  On that path
+ * sage_bfs (no parents) and sage_pagerank are collective; sage_sssp / sage_reorder return
+ * SAGE_E_UNSUPPORTED.                                                    */
 typedef struct {
   int32_t rank, world;         /* this process's rank and the number of ranks                    */
   const void *nccl_unique_id;  /* 128-byte ncclUniqueId created by rank 0 and broadcast by the
@@ -120,6 +123,9 @@ typedef struct {
  * non-decreasing, row_offsets[n_local] = m, 0 <= col < n, weights >= 1.  On failure *out is NULL.
  * Multi-GPU (dist->world > 1): collective over the ranks; creates the NCCL communicator.       */
 sage_status sage_load_csr(const sage_csr *in, sage_graph **out);
+
+/* Create a 128-byte NCCL unique id (rank 0 calls it and broadcasts the bytes to every rank).   */
+sage_status sage_nccl_unique_id(void *out128);
 
 /* Free the handle and every library-owned device array.  NULL is a no-op.                     */
 sage_status sage_free(sage_graph *g);

@@ -25,7 +25,7 @@ STATUS_NAMES = {0: "SAGE_OK", 1: "SAGE_E_INVALID", 2: "SAGE_E_NOMEM", 3: "SAGE_E
 
 EXPORTED = ["sage_load_csr", "sage_free", "sage_bfs", "sage_bfs_ex", "sage_sssp", "sage_pagerank",
             "sage_reorder", "sage_reorder_objective", "sage_get_permutation", "sage_get_csr", "sage_graph_info",
-            "sage_debug_export_tiles", "sage_debug_reorder_stages", "sage_debug_level_records", "sage_last_error", "sage_version"]
+            "sage_debug_export_tiles", "sage_debug_reorder_stages", "sage_nccl_unique_id", "sage_debug_level_records", "sage_last_error", "sage_version"]
 
 
 class SageError(RuntimeError):
@@ -92,6 +92,7 @@ def lib():
         L.sage_graph_info.argtypes = [p, p, p, p, p, p]
         L.sage_debug_export_tiles.argtypes = [p, p, i64, p, i64, p]
         L.sage_debug_level_records.argtypes = [p, p, i32, p]
+        L.sage_nccl_unique_id.argtypes = [p]
         L.sage_last_error.restype = ctypes.c_char_p
         L.sage_version.restype = ctypes.c_char_p
         for f in EXPORTED:
@@ -273,6 +274,13 @@ class Graph:
         return out[:4 * nq.value].reshape(-1, 4)
 
 
+def nccl_unique_id() -> bytes:
+    """sage_nccl_unique_id: 128 bytes to broadcast from rank 0 to every rank."""
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().sage_nccl_unique_id(buf))
+    return buf.raw
+
+
 def load_csr(off, col, w=None, n: int | None = None, symmetric: bool = False, push_only: bool = False,
              borrow: bool = False, validate: bool = True, tile_cta: int = 256, tile_min: int = 8,
              align: int = 4, alpha: float = 15.0, beta: float = 18.0, stream=None,
@@ -303,7 +311,7 @@ def load_csr(off, col, w=None, n: int | None = None, symmetric: bool = False, pu
     opts = Options(tile_cta, tile_min, align, alpha, beta)
     csr.opts = ctypes.pointer(opts)
     dist = None
-    if world > 1:
+    if nccl_unique_id is not None:
         idbuf = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
         dist = Dist(rank, world, ctypes.cast(idbuf, ctypes.c_void_p).value, v_begin,
                     v_end if v_end is not None else csr.n)

@@ -205,8 +205,8 @@ sage_status sage_load_csr(const sage_csr *in, sage_graph **out) {
   const bool borrow = devptrs && (flags & SAGE_F_BORROW);
   int64_t v_begin = 0, v_end = in->n;
   const sage_dist *ds = in->dist;
-  if (ds && ds->world > 1) {
-    if (ds->rank < 0 || ds->rank >= ds->world || !ds->nccl_unique_id || ds->v_begin < 0 ||
+  if (ds) {
+    if (ds->world < 1 || ds->rank < 0 || ds->rank >= ds->world || !ds->nccl_unique_id || ds->v_begin < 0 ||
         ds->v_end < ds->v_begin || ds->v_end > in->n) {
       set_error("invalid sage_dist");
       return SAGE_E_INVALID;
@@ -343,7 +343,7 @@ sage_status sage_load_csr(const sage_csr *in, sage_graph **out) {
     g->max_degree = (int64_t)h.max_deg;
     g->n_isolated = (int64_t)h.isolated;
   }
-  if (ds && ds->world > 1) {
+  if (ds) {
     st = init_comm(g, ds);
     if (st != SAGE_OK) {
       destroy(g);

@@ -1,26 +1,677 @@
-// comm.cu — multi-GPU (1D vertex partition + NCCL frontier exchange).
-// Placeholder until the exchange lands: multi-GPU handles are refused explicitly.
+// comm.cu — multi-GPU traversal: 1D vertex partition + NCCL frontier exchange.
+//
+// The paper runs two GPUs with no pre-partitioning and "data ... synchronized after each
+// iteration" without naming the mechanism.  Here (north_star): rank r owns the
+// contiguous vertex block [vb[r], vb[r+1]) and its out-rows (global column ids); one process per
+// GPU; the communicator is created from a unique id the caller broadcasts.  Per BFS level:
+//   push : the local stealing consumer expands the local log; owned neighbours are claimed
+//          locally, remote ones are marked in an outgoing bitmap -> NCCL alltoall of the owners'
+//          slices (dense next-frontier exchange, C1b) -> owners apply the received candidates.
+//   pull : allgather of the frontier slices (C1c), then every rank scans its own unvisited rows.
+//   stats: allreduce of (|F|, arcs(F)) gives termination and the Beamer direction (C1d).
+// PageRank: push into a full-length partial y, ncclReduceScatter(sum) to the owners (C1e), plus
+// an allreduce of the dangling mass (C1f).
+// Global-indexed bitmaps / vectors use a PADDED layout: vertex v of owner r sits at
+// r * P + (v - vb[r]) with P = 32 * Wp >= max rows per rank, so every rank's slice is a contiguous
+// word range and the exchanges are plain equal-count collectives.
+// With dist != NULL and world == 1 the same path runs on a 1-rank communicator (tested on 1 GPU).
+#include <cuda_runtime.h>
+#include <nccl.h>
+#include <string.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "common.cuh"
 #include "graph.h"
 #include "internal.h"
 
 namespace sage {
 
-struct Comm {};
+constexpr int kMaxRanks = 64;
 
-sage_status init_comm(sage_graph *, const sage_dist *) {
-  set_error("multi-GPU (world > 1) is not available in this build");
-  return SAGE_E_UNSUPPORTED;
-}
-void free_comm(sage_graph *g) { g->comm = nullptr; }
+struct PartMap {
+  int p;
+  int rank;
+  long long P;                    // padded vertices per rank (multiple of 32)
+  long long vb[kMaxRanks + 1];    // rank boundaries
+};
 
-sage_status run_bfs_multi(sage_graph *, int32_t, int32_t *, int32_t *, uint32_t, sage_stats *) {
-  return SAGE_E_UNSUPPORTED;
+__device__ __forceinline__ long long pidx(const PartMap &pm, long long v, bool *own) {
+  int lo = 0, hi = pm.p;
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    if (pm.vb[mid] <= v) lo = mid; else hi = mid;
+  }
+  *own = lo == pm.rank;
+  return (long long)lo * pm.P + (v - pm.vb[lo]);
 }
+
+struct Comm {
+  ncclComm_t nc = nullptr;
+  int rank = 0, world = 1;
+  std::vector<long long> vb;
+  long long Wp = 0;                  // padded words per rank
+  long long m_total = 0;
+  uint32_t *out = nullptr;           // p*Wp words
+  uint32_t *recv = nullptr;          // p*Wp words
+  uint32_t *visited = nullptr;       // p*Wp words (own slice authoritative, remote = "sent")
+  uint32_t *fb[3] = {nullptr, nullptr, nullptr};
+  unsigned long long *stats = nullptr;  // 8 u64
+  double *y = nullptr, *yown = nullptr, *dsum = nullptr;
+  PartMap pm;
+};
+
+static sage_status nccl_fail(sage_graph *g, ncclResult_t r, const char *what) {
+  set_error("%s: %s", what, ncclGetErrorString(r));
+  if (g) g->sticky = SAGE_E_NCCL;
+  return SAGE_E_NCCL;
+}
+#define NCCL_CHECK(g, call, what)                     \
+  do {                                                \
+    ncclResult_t r_ = (call);                         \
+    if (r_ != ncclSuccess) return nccl_fail(g, r_, what); \
+  } while (0)
+
+// ============================================================================ filters / kernels
+struct MultiArgs {
+  const long long *off;
+  const int *col;
+  long long n_local, v_begin;
+  Ladder L;
+  Queues q[2];
+  Ctl *ctl;
+  uint32_t *visited;
+  uint32_t *fb[3];
+  uint32_t *out;
+  const uint32_t *recv;
+  int *level;
+  int do_enabled;
+  int vec_ok;
+  int lvl;                         // current level L
+  PartMap pm;
+};
+
+struct BfsPushMulti {
+  struct Src {
+    int u;
+  };
+  static constexpr bool kWeights = false;
+  static constexpr bool kNeedRow = false;
+  static constexpr bool kEnqueue = true;
+  const MultiArgs *a;
+  uint32_t *fb_next;
+  const Queues *next_q;
+  CounterSet *next_cs;
+  __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
+  template <int N>
+  __device__ __forceinline__ void visit(bool valid, const Src &, int (&v)[N], const uint32_t (&)[N],
+                                        bool (&in)[N]) const {
+    const unsigned long long keep = policy_evict_last();
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      in[j] = false;
+      if (!valid) continue;
+      bool own;
+      const long long p = pidx(a->pm, v[j], &own);
+      const uint32_t bit = 1u << (p & 31);
+      if (ld_status(a->visited + (p >> 5), keep) & bit) continue;
+      const uint32_t old = atomicOr(a->visited + (p >> 5), bit);
+      if (old & bit) continue;
+      if (own) {
+        const int lv = (int)(v[j] - a->v_begin);
+        a->level[lv] = a->lvl + 1;
+        if (fb_next) atomicOr(fb_next + (p >> 5), bit);
+        v[j] = lv;                   // enqueue the LOCAL row id
+        in[j] = true;
+      } else {
+        atomicOr(a->out + (p >> 5), bit);   // candidate for its owner (dense exchange)
+      }
+    }
+  }
+};
+
+template <int VEC>
+__global__ void __launch_bounds__(kBlock, 4) k_mpush(const __grid_constant__ MultiArgs a) {
+  __shared__ WarpScratch wsm[kWarps];
+  __shared__ BfsPushMulti::Src fsrc[kWarps][32];
+  const int warp = threadIdx.x >> 5;
+  const int L = a.lvl;
+  BfsPushMulti f;
+  f.a = &a;
+  f.fb_next = a.do_enabled ? a.fb[(L + 1) % 3] : nullptr;
+  f.next_q = &a.q[(L + 1) & 1];
+  f.next_cs = &a.ctl->set[(L + 1) % 3];
+  consume_log<VEC>(f, a.L, a.q[L & 1], &a.ctl->set[L % 3], a.off, a.col, nullptr, &wsm[warp],
+                   fsrc[warp], a.vec_ok);
+}
+
+// Owners apply the candidates received from every other rank.
+__global__ void __launch_bounds__(kBlock) k_mapply(const __grid_constant__ MultiArgs a) {
+  __shared__ WarpScratch wsm[kWarps];
+  const int warp = threadIdx.x >> 5;
+  const unsigned lane = lane_id();
+  const int L = a.lvl;
+  const long long Wp = a.pm.P >> 5;
+  const long long words = (a.n_local + 31) >> 5;
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  uint32_t *fbn = a.do_enabled ? a.fb[(L + 1) % 3] : nullptr;
+  const Queues &Qn = a.q[(L + 1) & 1];
+  CounterSet *csn = &a.ctl->set[(L + 1) % 3];
+  int bcnt = 0;
+  for (long long base = gw * 32; base < words; base += nw * 32) {
+    const long long w = base + lane;
+    uint32_t nw_bits = 0;
+    if (w < words) {
+      uint32_t cand = 0;
+      for (int r = 0; r < a.pm.p; ++r)
+        if (r != a.pm.rank) cand |= a.recv[(long long)r * Wp + w];
+      if (w == words - 1 && (a.n_local & 31)) cand &= (1u << (a.n_local & 31)) - 1u;
+      const long long gwd = (long long)a.pm.rank * Wp + w;
+      const uint32_t own = a.visited[gwd];
+      nw_bits = cand & ~own;
+      if (nw_bits) {
+        a.visited[gwd] = own | nw_bits;
+        if (fbn) fbn[gwd] |= nw_bits;
+      }
+    }
+    while (__any_sync(FULL, nw_bits != 0)) {
+      const bool has = nw_bits != 0;
+      int lv = 0;
+      if (has) {
+        const int b = __ffs(nw_bits) - 1;
+        nw_bits &= nw_bits - 1;
+        lv = (int)(w * 32 + b);
+        a.level[lv] = L + 1;
+      }
+      buffer_push(has, lv, &wsm[warp], bcnt, a.off, a.L, Qn, csn);
+    }
+  }
+  if (bcnt) buffer_flush(&wsm[warp], bcnt, a.off, a.L, Qn, csn);
+}
+
+// Pull level over the own rows; the frontier bitmap holds the allgathered global frontier.
+__global__ void __launch_bounds__(kBlock) k_mpull(const __grid_constant__ MultiArgs a) {
+  __shared__ WarpScratch wsm[kWarps];
+  const int warp = threadIdx.x >> 5;
+  const unsigned lane = lane_id();
+  const int L = a.lvl;
+  const long long Wp = a.pm.P >> 5;
+  const long long words = (a.n_local + 31) >> 5;
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  const uint32_t *fbc = a.fb[L % 3];
+  uint32_t *fbn = a.fb[(L + 1) % 3];
+  const Queues &Qn = a.q[(L + 1) & 1];
+  CounterSet *cur = &a.ctl->set[L % 3];
+  CounterSet *csn = &a.ctl->set[(L + 1) % 3];
+  int bcnt = 0;
+  unsigned long long insp = 0, scanned = 0;
+  for (long long wd = gw; wd < words; wd += nw) {
+    const long long gwd = (long long)a.pm.rank * Wp + wd;
+    const long long v = (wd << 5) + lane;
+    const uint32_t vis = a.visited[gwd];
+    const bool todo = v < a.n_local && !((vis >> lane) & 1u);
+    bool found = false;
+    if (todo) {
+      const long long b = a.off[v], e = a.off[v + 1];
+      if (e > b) scanned++;
+      for (long long k = b; k < e; ++k) {
+        const int u = a.col[k];
+        ++insp;
+        bool own;
+        const long long p = pidx(a.pm, u, &own);
+        if ((fbc[p >> 5] >> (p & 31)) & 1u) {
+          found = true;
+          break;
+        }
+      }
+    }
+    const unsigned fm = __ballot_sync(FULL, found);
+    if (fm && lane == 0) {
+      a.visited[gwd] = vis | fm;
+      fbn[gwd] = fm;
+    }
+    if (found) a.level[v] = L + 1;
+    buffer_push(found, (int)v, &wsm[warp], bcnt, a.off, a.L, Qn, csn);
+  }
+  if (bcnt) buffer_flush(&wsm[warp], bcnt, a.off, a.L, Qn, csn);
+  insp = warp_sum64(insp);
+  scanned = warp_sum64(scanned);
+  if (lane == 0) {
+    if (insp) atomicAdd(&cur->inspected.v, insp);
+    if (scanned) atomicAdd(&cur->scanned.v, scanned);
+  }
+}
+
+__global__ void k_mseed(MultiArgs a, long long src_local) {
+  const bool act = threadIdx.x == 0;
+  long long b = 0, e = 0;
+  if (act) {
+    b = a.off[src_local];
+    e = a.off[src_local + 1];
+    const long long p = (long long)a.pm.rank * a.pm.P + src_local;
+    a.visited[p >> 5] |= 1u << (p & 31);
+    a.fb[0][p >> 5] |= 1u << (p & 31);
+    a.level[src_local] = 0;
+  }
+  enqueue_warp(act, (int)src_local, b, e, a.L, a.q[0], &a.ctl->set[0]);
+}
+
+// stats of the next log -> comm buffer (nF, arcsF, inspected, scanned of the level just run)
+__global__ void k_mstats(const Ctl *ctl, int cur, int nxt, unsigned long long *st) {
+  if (threadIdx.x == 0) {
+    st[0] = ctl->set[nxt].nF.v;
+    st[1] = ctl->set[nxt].arcsF.v;
+    st[2] = ctl->set[cur].inspected.v;
+    st[3] = ctl->set[cur].scanned.v;
+    st[4] = ctl->set[cur].nF.v;
+    st[5] = ctl->set[cur].arcsF.v;
+  }
+}
+
+// ---- PageRank
+struct PrPushMulti {
+  struct Src {
+    double c;
+  };
+  static constexpr bool kWeights = false;
+  static constexpr bool kNeedRow = true;
+  static constexpr bool kEnqueue = false;
+  const Queues *next_q = nullptr;
+  CounterSet *next_cs = nullptr;
+  const double *x;
+  double *y;
+  const PartMap *pm;
+  __device__ __forceinline__ Src src(bool valid, int u, long long b, long long e) const {
+    return Src{(valid && e > b) ? ldcg(x + u) / (double)(e - b) : 0.0};
+  }
+  template <int N>
+  __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N], const uint32_t (&)[N],
+                                        bool (&in)[N]) const {
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      in[j] = false;
+      if (!valid) continue;
+      bool own;
+      atomicAdd(y + pidx(*pm, v[j], &own), s.c);
+    }
+  }
+};
+struct MprArgs {
+  const long long *off;
+  const int *col;
+  Ladder L;
+  Queues q;
+  CounterSet *cs;
+  const int *dangling;
+  long long n_dangling;
+  const double *x;
+  double *y;
+  double *dsum;
+  int vec_ok;
+  PartMap pm;
+};
+template <int VEC>
+__global__ void __launch_bounds__(kBlock, 4) k_mpr_push(const __grid_constant__ MprArgs a) {
+  __shared__ WarpScratch wsm[kWarps];
+  __shared__ PrPushMulti::Src fsrc[kWarps][32];
+  __shared__ double red[kWarps];
+  const int warp = threadIdx.x >> 5;
+  PrPushMulti f;
+  f.x = a.x;
+  f.y = a.y;
+  f.pm = &a.pm;
+  consume_log<VEC>(f, a.L, a.q, a.cs, a.off, a.col, nullptr, &wsm[warp], fsrc[warp], a.vec_ok);
+  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  double d = 0.0;
+  for (long long i = tid; i < a.n_dangling; i += stride) d += a.x[a.dangling[i]];
+  d = warp_sumd(d);
+  if (lane_id() == 0) red[warp] = d;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double s = 0.0;
+    for (int k = 0; k < kWarps; ++k) s += red[k];
+    if (s != 0.0) atomicAdd(a.dsum, s);
+  }
+}
+__global__ void k_mpr_finalize(double *x, const double *yown, long long n_local, double base,
+                               double dmp, const double *dsum_global, double N) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  const double add = base + dmp * (*dsum_global) / N;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n_local; v += stride)
+    x[v] = add + dmp * yown[v];
+}
+__global__ void k_fill_f64(double *p, long long n, double v) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) p[i] = v;
+}
+
+// ============================================================================ host side
+sage_status init_comm(sage_graph *g, const sage_dist *ds) {
+  Comm *c = new Comm();
+  g->comm = c;
+  c->rank = ds->rank;
+  c->world = ds->world;
+  if (c->world > kMaxRanks) {
+    set_error("at most %d ranks", kMaxRanks);
+    return SAGE_E_INVALID;
+  }
+  ncclUniqueId id;
+  memcpy(&id, ds->nccl_unique_id, sizeof(id));
+  NCCL_CHECK(g, ncclCommInitRank(&c->nc, c->world, id, c->rank), "ncclCommInitRank");
+  // every rank's block and arc count
+  long long *d = nullptr;
+  sage_status s;
+  if ((s = dalloc(g, (void **)&d, sizeof(long long) * 4 * (size_t)(c->world + 1))) != SAGE_OK) return s;
+  long long mine[3] = {(long long)g->v_begin, (long long)g->v_end, (long long)g->m};
+  cudaMemcpyAsync(d + 3 * c->rank, mine, sizeof(mine), cudaMemcpyHostToDevice, g->stream);
+  NCCL_CHECK(g, ncclAllGather(d + 3 * c->rank, d, 3, ncclInt64, c->nc, g->stream), "allgather blocks");
+  std::vector<long long> all(3 * (size_t)c->world);
+  cudaMemcpyAsync(all.data(), d, sizeof(long long) * all.size(), cudaMemcpyDeviceToHost, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  dfree(g, d);
+  if (e != cudaSuccess) return cuda_fail(g, e, "comm init");
+  c->vb.assign((size_t)c->world + 1, 0);
+  long long maxrows = 0;
+  for (int r = 0; r < c->world; ++r) {
+    if (all[3 * r] != (r == 0 ? 0 : all[3 * (r - 1) + 1])) {
+      set_error("rank blocks must cover [0, n) contiguously in rank order");
+      return SAGE_E_INVALID;
+    }
+    c->vb[r] = all[3 * r];
+    c->vb[r + 1] = all[3 * r + 1];
+    maxrows = std::max(maxrows, all[3 * r + 1] - all[3 * r]);
+    c->m_total += all[3 * r + 2];
+  }
+  if (c->vb[c->world] != g->n) {
+    set_error("rank blocks must end at n");
+    return SAGE_E_INVALID;
+  }
+  c->Wp = (maxrows + 31) / 32 + 1;
+  memset(&c->pm, 0, sizeof(c->pm));
+  c->pm.p = c->world;
+  c->pm.rank = c->rank;
+  c->pm.P = c->Wp * 32;
+  for (int r = 0; r <= c->world; ++r) c->pm.vb[r] = c->vb[r];
+  const size_t words = (size_t)c->Wp * (size_t)c->world;
+  if ((s = dalloc(g, (void **)&c->out, 4 * words)) != SAGE_OK ||
+      (s = dalloc(g, (void **)&c->recv, 4 * words)) != SAGE_OK ||
+      (s = dalloc(g, (void **)&c->visited, 4 * words)) != SAGE_OK ||
+      (s = dalloc(g, (void **)&c->stats, sizeof(unsigned long long) * 16)) != SAGE_OK)
+    return s;
+  for (int i = 0; i < 3; ++i)
+    if ((s = dalloc(g, (void **)&c->fb[i], 4 * words)) != SAGE_OK) return s;
+  return SAGE_OK;
+}
+
+void free_comm(sage_graph *g) {
+  Comm *c = g->comm;
+  if (!c) return;
+  dfree(g, c->out);
+  dfree(g, c->recv);
+  dfree(g, c->visited);
+  dfree(g, c->stats);
+  for (int i = 0; i < 3; ++i) dfree(g, c->fb[i]);
+  dfree(g, c->y);
+  dfree(g, c->yown);
+  dfree(g, c->dsum);
+  cudaStreamSynchronize(g->stream);
+  if (c->nc) ncclCommDestroy(c->nc);
+  delete c;
+  g->comm = nullptr;
+}
+
+static sage_status allreduce_stats(sage_graph *g, int L, unsigned long long *h6) {
+  Comm *c = g->comm;
+  k_mstats<<<1, 32, 0, g->stream>>>(g->ts.ctl, L % 3, (L + 1) % 3, c->stats);
+  NCCL_CHECK(g, ncclAllReduce(c->stats, c->stats + 8, 6, ncclUint64, ncclSum, c->nc, g->stream),
+             "stats allreduce");
+  cudaMemcpyAsync(h6, c->stats + 8, sizeof(unsigned long long) * 6, cudaMemcpyDeviceToHost, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "stats");
+  return SAGE_OK;
+}
+
+sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int32_t *parent_out,
+                          uint32_t call_flags, sage_stats *st) {
+  Comm *c = g->comm;
+  if (parent_out) {
+    set_error("BFS parents are not produced by the multi-GPU path");
+    return SAGE_E_UNSUPPORTED;
+  }
+  sage_status s;
+  if ((s = ensure_traversal_state(g)) != SAGE_OK) return s;
+  TraversalState &t = g->ts;
+  const bool symmetric = g->flags & SAGE_F_SYMMETRIC;
+  const bool do_enabled = symmetric && !((g->flags | call_flags) & SAGE_F_PUSH_ONLY);
+  const size_t words = (size_t)c->Wp * (size_t)c->world;
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  cudaEventRecord(e0, g->stream);
+  cudaMemsetAsync(t.level, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
+  cudaMemsetAsync(c->visited, 0, 4 * words, g->stream);
+  cudaMemsetAsync(c->out, 0, 4 * words, g->stream);
+  for (int i = 0; i < 3; ++i) cudaMemsetAsync(c->fb[i], 0, 4 * words, g->stream);
+  cudaMemsetAsync(t.ctl, 0, offsetof(Ctl, rec), g->stream);
+  MultiArgs a;
+  memset(&a, 0, sizeof(a));
+  a.off = (const long long *)g->off;
+  a.col = g->col;
+  a.n_local = g->n_local;
+  a.v_begin = g->v_begin;
+  a.L = g->ladder;
+  a.q[0] = t.q[0];
+  a.q[1] = t.q[1];
+  a.ctl = t.ctl;
+  a.visited = c->visited;
+  for (int i = 0; i < 3; ++i) a.fb[i] = c->fb[i];
+  a.out = c->out;
+  a.recv = c->recv;
+  a.level = t.level;
+  a.do_enabled = do_enabled ? 1 : 0;
+  a.vec_ok = g->vec_ok ? 1 : 0;
+  a.pm = c->pm;
+  if (source >= g->v_begin && source < g->v_end)
+    k_mseed<<<1, 32, 0, g->stream>>>(a, (long long)source - g->v_begin);
+  // global arcs of the source (level-0 frontier)
+  unsigned long long h6[6];
+  {
+    k_mstats<<<1, 32, 0, g->stream>>>(t.ctl, 2, 0, c->stats);   // set[0] = the seed's log
+    NCCL_CHECK(g, ncclAllReduce(c->stats, c->stats + 8, 6, ncclUint64, ncclSum, c->nc, g->stream),
+               "stats allreduce");
+    cudaMemcpyAsync(h6, c->stats + 8, sizeof(h6), cudaMemcpyDeviceToHost, g->stream);
+    cudaError_t e = cudaStreamSynchronize(g->stream);
+    if (e != cudaSuccess) return cuda_fail(g, e, "seed");
+  }
+  double mU = (double)c->m_total - (double)h6[1];
+  unsigned long long reached_arcs = h6[1];
+  const int grid_push = g->num_sms * 4;
+  int dir = 0;
+  unsigned long long prev_nF = 1;
+  long long push_exp = 0, push_arcs = 0, push_disc = 0, pull_sc = 0, pull_insp = 0, pull_disc = 0;
+  int levels = 0, pushL = 0, pullL = 0;
+  for (int L = 0;; ++L) {
+    cudaMemsetAsync(&t.ctl->set[(L + 2) % 3], 0, sizeof(CounterSet), g->stream);
+    if (do_enabled) cudaMemsetAsync(c->fb[(L + 2) % 3], 0, 4 * words, g->stream);
+    a.lvl = L;
+    if (dir == 0) {
+      if (g->vec == 4) k_mpush<4><<<grid_push, kBlock, 0, g->stream>>>(a);
+      else k_mpush<1><<<grid_push, kBlock, 0, g->stream>>>(a);
+      // dense alltoall of the owners' candidate slices
+      NCCL_CHECK(g, ncclGroupStart(), "group");
+      for (int r = 0; r < c->world; ++r) {
+        if (r == c->rank) continue;
+        NCCL_CHECK(g, ncclSend(c->out + (size_t)r * c->Wp, (size_t)c->Wp, ncclUint32, r, c->nc, g->stream),
+                   "send");
+        NCCL_CHECK(g, ncclRecv(c->recv + (size_t)r * c->Wp, (size_t)c->Wp, ncclUint32, r, c->nc, g->stream),
+                   "recv");
+      }
+      NCCL_CHECK(g, ncclGroupEnd(), "group");
+      cudaMemsetAsync(c->out, 0, 4 * words, g->stream);
+      if (c->world > 1) k_mapply<<<grid_push, kBlock, 0, g->stream>>>(a);
+    } else {
+      k_mpull<<<grid_push, kBlock, 0, g->stream>>>(a);
+    }
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(g, e, "multi-GPU level");
+    if ((s = allreduce_stats(g, L, h6)) != SAGE_OK) return s;
+    const unsigned long long nF = h6[0], aF = h6[1];
+    levels = L + 1;
+    if (dir == 0) {
+      pushL++;
+      push_exp += (long long)h6[4];
+      push_arcs += (long long)h6[5];
+      push_disc += (long long)nF;
+    } else {
+      pullL++;
+      pull_sc += (long long)h6[3];
+      pull_insp += (long long)h6[2];
+      pull_disc += (long long)nF;
+    }
+    reached_arcs += aF;
+    if (nF == 0) break;
+    if (L + 1 > g->n) {
+      set_error("level cap exceeded");
+      return SAGE_E_CUDA;
+    }
+    mU -= (double)aF;
+    int ndir = dir;
+    if (do_enabled) {
+      if (dir == 0) {
+        if ((double)aF > mU / g->alpha) ndir = 1;
+      } else {
+        if (!(nF >= prev_nF || (double)nF > (double)g->n / g->beta)) ndir = 0;
+      }
+    }
+    if (ndir == 1) {
+      // pull needs the global frontier: allgather of every owner's slice of fb[L+1]
+      uint32_t *fbn = c->fb[(L + 1) % 3];
+      NCCL_CHECK(g, ncclAllGather(fbn + (size_t)c->rank * c->Wp, fbn, (size_t)c->Wp, ncclUint32, c->nc,
+                                  g->stream),
+                 "frontier allgather");
+    }
+    dir = ndir;
+    prev_nF = nF;
+  }
+  cudaEventRecord(e1, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "multi-GPU BFS");
+  float ms = 0;
+  cudaEventElapsedTime(&ms, e0, e1);
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (st) {
+    memset(st, 0, sizeof(*st));
+    st->levels = levels;
+    st->push_levels = pushL;
+    st->pull_levels = pullL;
+    st->vertices_expanded = push_exp + pull_sc;
+    st->arcs_inspected = push_arcs + pull_insp;
+    st->vertices_discovered = push_disc + pull_disc;
+    st->edges_traversed = (int64_t)(symmetric ? reached_arcs / 2 : reached_arcs);
+    st->ms = ms;
+    st->kernel_ms = ms;
+    const double n = (double)g->n;
+    st->model_bytes = 4.0 * n + 20.0 * push_exp + 8.0 * push_arcs + 8.0 * push_disc + 16.0 * pull_sc +
+                      (n / 8.0) * pullL + 4.125 * pull_insp + 4.125 * pull_disc;
+  }
+  if ((s = copy_out(g, level_out, t.level, sizeof(int32_t) * (size_t)g->n_local)) != SAGE_OK) return s;
+  e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "output");
+  return SAGE_OK;
+}
+
 sage_status run_sssp_multi(sage_graph *, int32_t, uint32_t *, sage_stats *) {
+  set_error("multi-GPU SSSP is not implemented (SURVEY §8(f) NEXT #2)");
   return SAGE_E_UNSUPPORTED;
 }
-sage_status run_pagerank_multi(sage_graph *, double, int32_t, double *, sage_stats *) {
-  return SAGE_E_UNSUPPORTED;
+
+sage_status run_pagerank_multi(sage_graph *g, double damping, int32_t iterations, double *rank_out,
+                               sage_stats *st) {
+  Comm *c = g->comm;
+  sage_status s;
+  if ((s = ensure_traversal_state(g)) != SAGE_OK) return s;
+  if ((s = ensure_pagerank_log(g)) != SAGE_OK) return s;
+  const long long P = c->pm.P;
+  if (!c->y) {
+    if ((s = dalloc(g, (void **)&c->y, sizeof(double) * (size_t)P * c->world)) != SAGE_OK ||
+        (s = dalloc(g, (void **)&c->yown, sizeof(double) * (size_t)P)) != SAGE_OK ||
+        (s = dalloc(g, (void **)&c->dsum, sizeof(double) * 2)) != SAGE_OK)
+      return s;
+  }
+  PageRankState &p = g->pr;
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  cudaEventRecord(e0, g->stream);
+  const int grid = g->num_sms * 4;
+  k_fill_f64<<<grid, 256, 0, g->stream>>>(p.x, g->n_local, 1.0 / (double)g->n);
+  MprArgs a;
+  memset(&a, 0, sizeof(a));
+  a.off = (const long long *)g->off;
+  a.col = g->col;
+  a.L = g->ladder;
+  a.q = p.q;
+  a.cs = p.cs;
+  a.dangling = p.dangling;
+  a.n_dangling = p.n_dangling;
+  a.x = p.x;
+  a.y = c->y;
+  a.dsum = c->dsum;
+  a.vec_ok = g->vec_ok ? 1 : 0;
+  a.pm = c->pm;
+  const double N = (double)g->n;
+  for (int it = 0; it < iterations; ++it) {
+    cudaMemsetAsync(c->y, 0, sizeof(double) * (size_t)P * c->world, g->stream);
+    cudaMemsetAsync(c->dsum, 0, sizeof(double), g->stream);
+    cudaMemsetAsync(&p.cs[0].tk, 0, sizeof(p.cs[0].tk), g->stream);
+    if (g->vec == 4) k_mpr_push<4><<<grid, kBlock, 0, g->stream>>>(a);
+    else k_mpr_push<1><<<grid, kBlock, 0, g->stream>>>(a);
+    NCCL_CHECK(g, ncclReduceScatter(c->y, c->yown, (size_t)P, ncclFloat64, ncclSum, c->nc, g->stream),
+               "reduce-scatter");
+    NCCL_CHECK(g, ncclAllReduce(c->dsum, c->dsum + 1, 1, ncclFloat64, ncclSum, c->nc, g->stream),
+               "dangling allreduce");
+    k_mpr_finalize<<<grid, 256, 0, g->stream>>>(p.x, c->yown, g->n_local, (1.0 - damping) / N, damping,
+                                                c->dsum + 1, N);
+  }
+  cudaEventRecord(e1, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "multi-GPU PageRank");
+  float ms = 0;
+  cudaEventElapsedTime(&ms, e0, e1);
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (st) {
+    memset(st, 0, sizeof(*st));
+    st->levels = st->push_levels = iterations;
+    st->edges_traversed = st->arcs_inspected = (int64_t)iterations * c->m_total;
+    st->ms = st->kernel_ms = ms;
+    st->model_bytes = (double)iterations * (40.0 * (double)g->n_local + 12.0 * (double)g->m);
+  }
+  if ((s = copy_out(g, rank_out, p.x, sizeof(double) * (size_t)g->n_local)) != SAGE_OK) return s;
+  e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "output");
+  return SAGE_OK;
 }
 
 }  // namespace sage
+
+extern "C" sage_status sage_nccl_unique_id(void *out128) {
+  sage::clear_error();
+  if (!out128) {
+    sage::set_error("null argument");
+    return SAGE_E_INVALID;
+  }
+  ncclUniqueId id;
+  ncclResult_t r = ncclGetUniqueId(&id);
+  if (r != ncclSuccess) {
+    sage::set_error("ncclGetUniqueId: %s", ncclGetErrorString(r));
+    return SAGE_E_NCCL;
+  }
+  memcpy(out128, &id, sizeof(id));
+  return SAGE_OK;
+}

@@ -419,8 +419,9 @@ __device__ __forceinline__ void buffer_flush(WarpScratch *ws, int &cnt,
 // Filter policy F provides:
 //   struct Src;                                    per-source-vertex context
 //   Src src(bool valid, int u, long long b, long long e);   (b,e = row of u when needed)
-//   template<int N> void visit(bool valid, const Src&, const int (&v)[N], const uint32_t (&w)[N],
-//                              bool (&in)[N]);      marks the neighbours filtered in
+//   template<int N> void visit(bool valid, const Src&, int (&v)[N], const uint32_t (&w)[N],
+//                              bool (&in)[N]);      marks the neighbours filtered in (and may
+//                              rewrite v[j] to the row id to enqueue, e.g. global -> local)
 //   kWeights (load weights), kNeedRow (src needs the row for CTA tiles), kEnqueue (contraction)
 //   Queues *next_q; CounterSet *next_cs;             where filtered-in vertices go
 template <int VEC, class F>

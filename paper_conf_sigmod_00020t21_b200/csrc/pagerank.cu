@@ -33,7 +33,7 @@ struct PrPush {
     return Src{(valid && e > b) ? ldcg(x + u) / (double)(e - b) : 0.0};
   }
   template <int N>
-  __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
+  __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N],
                                         const uint32_t (&)[N], bool (&in)[N]) const {
 #pragma unroll
     for (int j = 0; j < N; ++j) in[j] = false;

@@ -48,7 +48,7 @@ struct BfsPush {
 
   // Alg. 1 l.1-6: if dist[nb] = -1 then dist[nb] := dist[fr] + 1; filter_in(nb)
   template <int N>
-  __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
+  __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N],
                                         const uint32_t (&)[N], bool (&in)[N]) const {
     uint32_t wd[N];
     const unsigned long long keep = policy_evict_last();
@@ -90,7 +90,7 @@ struct SsspPush {
   }
 
   template <int N>
-  __device__ __forceinline__ void visit(bool valid, const Src &s, const int (&v)[N],
+  __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N],
                                         const uint32_t (&w)[N], bool (&in)[N]) const {
     uint32_t cur[N];
     const unsigned long long keep = policy_evict_last();

@@ -1,0 +1,59 @@
+"""The NCCL multi-GPU path (1D partition) on a 1-rank communicator.
+
+gpurun and the round-end runs expose one GPU, so world > 1 cannot run here; with dist != NULL and
+world == 1 the library takes exactly the host-sequenced NCCL path (padded layout, per-level stats
+allreduce, frontier allgather before pull levels, dense alltoall loop, PR reduce-scatter).  The
+protocol itself with two ranks is checked on CPU by tests/test_partition_model.py (gloo).
+"""
+import numpy as np
+import pytest
+
+import oracle
+import sagegen as sg
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def sage():
+    import torch
+    assert torch.cuda.is_available()
+    from __graft_entry__ import build
+    build()
+    import paper_conf_sigmod_00020t21_b200 as s
+    return s
+
+
+@pytest.mark.parametrize("sym", [True, False])
+def test_nccl_path_bfs_pagerank(sage, sym):
+    g = sg.rmat(14, 16, seed=3, symmetric=sym)
+    uid = sage.nccl_unique_id()
+    with sage.load_csr(g.off, g.col, symmetric=sym, rank=0, world=1, nccl_unique_id=uid,
+                       v_begin=0, v_end=g.n) as G:
+        for s in sg.sources(g, 4, seed=2):
+            ref = oracle.bfs(g.off, g.col, int(s))
+            for po in (True, False):
+                lv, _, st = G.bfs(int(s), push_only=po)
+                assert np.array_equal(lv, ref)
+                assert st["edges_traversed"] == int(np.diff(g.off)[ref >= 0].sum()) // (2 if sym else 1)
+            if sym:
+                assert st["pull_levels"] >= 1
+        x, _ = G.pagerank(0.85, 20)
+        xr = oracle.pagerank(g.off, g.col, 0.85, 20)
+        assert np.max(np.abs(x - xr) / xr) <= 1e-6
+        with pytest.raises(sage.SageError) as ei:
+            G.bfs(0, parents=True)
+        assert ei.value.status == sage.E_UNSUPPORTED
+
+
+def test_nccl_path_refuses_sssp_and_bad_blocks(sage):
+    g = sg.rmat(10, 8, seed=1, symmetric=True)
+    w = sg.weights(g, 1)
+    uid = sage.nccl_unique_id()
+    with sage.load_csr(g.off, g.col, w, symmetric=True, rank=0, world=1, nccl_unique_id=uid) as G:
+        with pytest.raises(sage.SageError) as ei:
+            G.sssp(0)
+        assert ei.value.status == sage.E_UNSUPPORTED
+    with pytest.raises(sage.SageError):
+        sage.load_csr(g.off[:11], g.col[:g.off[10]], rank=0, world=1, nccl_unique_id=sage.nccl_unique_id(),
+                      v_begin=0, v_end=10, n=g.n)   # one rank must cover [0, n)

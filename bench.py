@@ -41,6 +41,7 @@ def _args():
     p.add_argument("--config", default="C2")
     p.add_argument("--scale", type=int, default=None, help="override the RMAT scale (debug only)")
     p.add_argument("--no-extras", action="store_true")
+    p.add_argument("--nccl", action="store_true", help="use the multi-GPU (NCCL) path even at N=1")
     return p.parse_args()
 
 
@@ -173,15 +174,51 @@ def main():
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     build()
-    g, gname = _graph(a.config, a.scale)
     stream = torch.cuda.current_stream()
-    off_d = torch.from_numpy(g.off).cuda()
-    col_d = torch.from_numpy(g.col).cuda()
-    w_d = torch.from_numpy(g.w).cuda() if g.w is not None else None
-    G = sage.load_csr(off_d, col_d, w_d, symmetric=True, borrow=True, stream=stream.cuda_stream)
-    n = g.n
-    srcs = sg.sources(g, a.warmup + a.steps, seed=2 + rank)
-    level = torch.empty(n, dtype=torch.int32, device="cuda")
+    multi = world > 1 or a.nccl
+    if not multi:
+        g, gname = _graph(a.config, a.scale)
+        off_d = torch.from_numpy(g.off).cuda()
+        col_d = torch.from_numpy(g.col).cuda()
+        w_d = torch.from_numpy(g.w).cuda() if g.w is not None else None
+        G = sage.load_csr(off_d, col_d, w_d, symmetric=True, borrow=True, stream=stream.cuda_stream)
+        n = g.n
+        n_rows = n
+    else:
+        # rank 0 generates the workload and broadcasts it; every rank keeps its 1D block
+        g, gname = _graph(a.config, a.scale) if rank == 0 else (None, None)
+        hdr = torch.tensor([g.n, g.m] if rank == 0 else [0, 0], dtype=torch.int64, device="cuda")
+        if world > 1:
+            torch.distributed.broadcast(hdr, 0)
+        n, m = int(hdr[0]), int(hdr[1])
+        off_full = torch.from_numpy(g.off).cuda() if rank == 0 else torch.empty(n + 1, dtype=torch.int64, device="cuda")
+        col_full = torch.from_numpy(g.col).cuda() if rank == 0 else torch.empty(m, dtype=torch.int32, device="cuda")
+        if world > 1:
+            torch.distributed.broadcast(off_full, 0)
+            torch.distributed.broadcast(col_full, 0)
+            obj = [gname, sage.nccl_unique_id() if rank == 0 else None]
+            torch.distributed.broadcast_object_list(obj, 0)
+            gname, uid = obj
+        else:
+            uid = sage.nccl_unique_id()
+        vb, ve = n * rank // world, n * (rank + 1) // world
+        b0 = int(off_full[vb])
+        off_d = (off_full[vb:ve + 1] - b0).contiguous()
+        col_d = col_full[b0:int(off_full[ve])].contiguous()
+        G = sage.load_csr(off_d, col_d, n=n, symmetric=True, borrow=True, stream=stream.cuda_stream,
+                          rank=rank, world=world, nccl_unique_id=uid, v_begin=vb, v_end=ve)
+        n_rows = ve - vb
+        if rank != 0:
+            class _G:  # sources only need the degree array
+                pass
+            g = _G()
+            g.n = n
+            g.off = off_full.cpu().numpy()
+            g.m = m
+            g.w = None
+        del off_full, col_full
+    srcs = sg.sources(g, a.warmup + a.steps, seed=2)
+    level = torch.empty(n_rows, dtype=torch.int32, device="cuda")
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
 
     def barrier():
@@ -217,7 +254,13 @@ def main():
     edges = [s["edges_traversed"] for s in stats]
     gteps = [e / (t * 1e-3) / 1e9 for e, t in zip(edges, times)]
     hm = len(gteps) / sum(1 / x for x in gteps)
-    value = hm * world if world > 1 else hm     # replicas: whole-job aggregate
+    if world > 1:   # global edges over the max-over-ranks time of each step
+        tt = torch.tensor(times, device="cuda")
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        times = tt.cpu().tolist()
+        gteps = [e / (t * 1e-3) / 1e9 for e, t in zip(edges, times)]
+        hm = len(gteps) / sum(1 / x for x in gteps)
+    value = hm
     kms = float(np.mean([s["kernel_ms"] for s in stats]))
     kbytes = float(np.mean([s["model_bytes"] - 4.0 * n for s in stats]))
     peaks, peak_src = _peaks()
@@ -225,24 +268,66 @@ def main():
     tr = _traffic()
     roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
             "frac": achieved / peaks["hbm_gbs"], "traffic": (tr or {}).get("bfs_push_bytes_per_launch"),
-            "kernel": "k_bfs<4> (persistent TP+RTS consumer)", "peak_source": peak_src,
+            "kernel": ("k_bfs<4> (persistent TP+RTS consumer)" if not multi else
+                       "host-sequenced NCCL levels (k_mpush + alltoall + k_mapply), time incl. exchange"),
+            "peak_source": peak_src,
             "model": "SURVEY §8(d): 20 B/expanded vertex + 8 B/inspected arc + 8 B/discovered vertex",
             "kernel_ms": kms, "model_bytes_per_launch": kbytes}
     line = {"metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": world, "steps": a.steps,
             "warmup": a.warmup, "ms_per_step": t_max / a.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "scaling": "strong" if multi else "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": gname, "n": n, "arcs": g.m, "mode": "push-only (SAGE_F_PUSH_ONLY)",
                        "tile_ladder": "B=256 M=8 A=4", "l2": "flushed between steps (256 MB write)",
-                       "parallelism": "replicas" if world > 1 else "single"},
-            "gpu_launches": 2 * a.steps, "clocks": clocks, "roofline": roof,
+                       "parallelism": f"1D-partition x{world} (NCCL)" if multi else "single"},
+            "gpu_launches": (2 * a.steps if not multi else
+                             sum(2 + s["levels"] * (3 if world > 1 else 2) for s in stats)),
+            "clocks": clocks, "roofline": roof,
             "bfs_levels": stats[-1]["levels"]}
-    if rank == 0 and not a.no_extras:
+    if rank == 0 and not a.no_extras and not multi:
         line.update(_extras(a, G, g, srcs, level, flush, stream, sage))
+    if multi:
+        line["e2e"] = _e2e_multi(a, G, g, srcs, sage, rank, world, off_d, col_d, n, uid if world == 1 else None)
     if rank == 0:
         print(json.dumps(line), flush=True)
     G.free()
     if world > 1:
         torch.distributed.destroy_process_group()
+
+
+def _e2e_multi(a, G, g, srcs, sage, rank, world, off_d, col_d, n, uid):
+    """End to end on the NCCL path: every rank loads its block from pinned host memory (H2D),
+    runs the BFS, reads its level slice back (D2H); time = max over ranks."""
+    import torch
+    off_h = off_d.cpu().pin_memory()
+    col_h = col_d.cpu().pin_memory()
+    lv_h = torch.empty(len(off_h) - 1, dtype=torch.int32).pin_memory()
+    vb, ve = G.v_begin, G.v_begin + G.n_local
+    res = []
+    for i in range(2):
+        if world > 1:
+            obj = [sage.nccl_unique_id() if rank == 0 else None]
+            torch.distributed.broadcast_object_list(obj, 0)
+            u = obj[0]
+            torch.distributed.barrier()
+        else:
+            u = sage.nccl_unique_id()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        with sage.load_csr(off_h, col_h, n=n, symmetric=True, rank=rank, world=world, nccl_unique_id=u,
+                           v_begin=vb, v_end=ve) as H:
+            _, _, st = H.bfs(int(srcs[i]), out=lv_h, push_only=True)
+        torch.cuda.synchronize()
+        dt = time.perf_counter() - t0
+        if world > 1:
+            t = torch.tensor([dt], device="cuda")
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            dt = float(t.item())
+        res.append((dt, st["edges_traversed"]))
+    return {"value": len(res) / sum(t * 1e9 / e for t, e in res), "unit": "GTEPS",
+            "h2d_bytes_per_step": int(off_h.numel() * 8 + col_h.numel() * 4),
+            "d2h_bytes_per_step": int(lv_h.numel() * 4),
+            "includes": "per rank: sage_load_csr of its block from pinned host memory (copy + validation + "
+                        "NCCL communicator) + sage_bfs + level D2H; max over ranks"}
 
 
 def _time_calls(fn, k, flush, stream):

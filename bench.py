@@ -363,14 +363,16 @@ def _extras(a, G, g, srcs, level, flush, stream, sage):
                   "ms": float(np.mean([t for t, _ in r])), "iterations": r[-1][1]["levels"],
                   "arcs_relaxed_per_edge": r[-1][1]["arcs_inspected"] / g.m,
                   "model_GBps": float(np.mean([st["model_bytes"] / (st["kernel_ms"] * 1e-3) / 1e9 for _, st in r]))}
-    # PageRank 20 iterations
+    # PageRank 20 iterations: pull (default on symmetric graphs) and the paper's push form
     x = torch.empty(g.n, dtype=torch.float64, device="cuda")
-    G.pagerank(0.85, 20, out=x)
-    r = _time_calls(lambda i: G.pagerank(0.85, 20, out=x)[1], 2, flush, stream)
-    ms = float(np.mean([t for t, _ in r]))
-    ex["pagerank"] = {"ms_20_iter": ms, "gedges_per_s": 20 * g.m / (ms * 1e-3) / 1e9,
-                      "model_GBps": float(np.mean([st["model_bytes"] / (st["kernel_ms"] * 1e-3) / 1e9
-                                                   for _, st in r]))}
+    ex["pagerank"] = {}
+    for form, po in (("pull", False), ("push", True)):
+        G.pagerank(0.85, 20, out=x, push_only=po)
+        r = _time_calls(lambda i: G.pagerank(0.85, 20, out=x, push_only=po)[1], 2, flush, stream)
+        ms = float(np.mean([t for t, _ in r]))
+        ex["pagerank"][form] = {"ms_20_iter": ms, "gedges_per_s": 20 * g.m / (ms * 1e-3) / 1e9,
+                                "model_GBps": float(np.mean([st["model_bytes"] / (st["kernel_ms"] * 1e-3) / 1e9
+                                                             for _, st in r]))}
     # end-to-end through the C ABI with HOST buffers: load (H2D) + BFS + level D2H
     off_h = torch.from_numpy(g.off).pin_memory()
     col_h = torch.from_numpy(g.col).pin_memory()

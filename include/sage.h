@@ -52,8 +52,12 @@ enum {
   SAGE_F_BORROW = 4u,      /* with DEVICE_PTRS: use the caller arrays in place (no copy); the caller
                               keeps them alive and unmodified until sage_free                      */
   SAGE_F_NO_VALIDATE = 8u, /* skip the validation pass of sage_load_csr                              */
-  SAGE_F_PUSH_ONLY = 16u   /* disable direction switching: every level is the paper's push
+  SAGE_F_PUSH_ONLY = 16u,  /* disable direction switching: every level is the paper's push
                               expansion (Alg. 2/3).  Can also be set per call (sage_bfs_ex).     */
+  SAGE_F_BINNED = 32u      /* per call (sage_bfs_ex), experimental: two-phase push levels (neighbour
+                              ids binned by vertex slice, then filtered against shared-memory
+                              slices of the visited bitmap).  Results identical;
+                              slower than the default direct filter on B200 as measured.        */
 };
 
 /* Multi-GPU description (1D vertex partition).  NULL in sage_csr = single GPU.
@@ -152,6 +156,14 @@ sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_out, sage_st
 sage_status sage_pagerank(sage_graph *g, double damping, int32_t iterations, double *rank_out,
                           sage_stats *st);
 
+/* sage_pagerank with a per-call flag word.  On a SAGE_F_SYMMETRIC graph the default form is the
+ * pull (gather) form over the same resident log — y_v = sum of x_u / out(u) over v's row, fp32
+ * contributions and fp64 accumulation (reading R7), one fp64 atomic per tile lane group instead
+ * of one per arc; SAGE_F_PUSH_ONLY (graph or call) selects the paper's push form (Alg. 1
+ * l.26-29).  Directed graphs always use push.                                                  */
+sage_status sage_pagerank_ex(sage_graph *g, double damping, int32_t iterations, double *rank_out,
+                             uint32_t call_flags, sage_stats *st);
+
 /* `rounds` rounds of Sampling-based Reordering (§6; readings R17-R25): relabels the
  * vertices in place (the CSR is rewritten, rows sorted, weights moved with their arcs) and
  * composes the permutation; later queries still speak original ids.  Single GPU only.         */
@@ -189,10 +201,11 @@ sage_status sage_debug_reorder_stages(sage_graph *g, int32_t sector_width, const
                                       int64_t n_candidates, int64_t *loc1_out, int64_t *target_out,
                                       int64_t *loc3_out, uint8_t *mover_out);
 
-/* Diagnostic entry point: per-level records of the last BFS / SSSP query on this graph, 8 int64 per
+/* Diagnostic entry point: per-level records of the last BFS / SSSP query on this graph, 9 int64 per
  * level: direction (0 push, 1 pull), |F|, arcs(F), arcs inspected, vertices scanned (pull),
  * vertices discovered, device time since the kernel started at the end of the level (ns), and
- * the time at which the last warp finished the level's work, before the grid barrier (ns).
+ * the time at which the last warp finished the level's work, before the grid barrier (ns), and
+ * (binned push levels) the end of the expansion phase (ns, microsecond resolution; 0 otherwise).
  * Writes min(levels, cap) records to host memory; *n_out = number of levels (<= 4096 kept).     */
 sage_status sage_debug_level_records(const sage_graph *g, int64_t *rec_out, int32_t cap,
                                      int32_t *n_out);

@@ -19,11 +19,12 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, os.environ.get("SAGE_LIB", "libsage.so"))
 
 OK, E_INVALID, E_NOMEM, E_CUDA, E_NCCL, E_OVERFLOW, E_UNSUPPORTED = range(7)
-F_SYMMETRIC, F_DEVICE_PTRS, F_BORROW, F_NO_VALIDATE, F_PUSH_ONLY = 1, 2, 4, 8, 16
+F_SYMMETRIC, F_DEVICE_PTRS, F_BORROW, F_NO_VALIDATE, F_PUSH_ONLY, F_BINNED = 1, 2, 4, 8, 16, 32
 STATUS_NAMES = {0: "SAGE_OK", 1: "SAGE_E_INVALID", 2: "SAGE_E_NOMEM", 3: "SAGE_E_CUDA",
                 4: "SAGE_E_NCCL", 5: "SAGE_E_OVERFLOW", 6: "SAGE_E_UNSUPPORTED"}
 
 EXPORTED = ["sage_load_csr", "sage_free", "sage_bfs", "sage_bfs_ex", "sage_sssp", "sage_pagerank",
+            "sage_pagerank_ex",
             "sage_reorder", "sage_reorder_objective", "sage_get_permutation", "sage_get_csr", "sage_graph_info",
             "sage_debug_export_tiles", "sage_debug_reorder_stages", "sage_nccl_unique_id", "sage_debug_level_records", "sage_last_error", "sage_version"]
 
@@ -84,6 +85,7 @@ def lib():
         L.sage_bfs_ex.argtypes = [p, i32, p, p, u32, ctypes.POINTER(Stats)]
         L.sage_sssp.argtypes = [p, i32, p, ctypes.POINTER(Stats)]
         L.sage_pagerank.argtypes = [p, dbl, i32, p, ctypes.POINTER(Stats)]
+        L.sage_pagerank_ex.argtypes = [p, dbl, i32, p, u32, ctypes.POINTER(Stats)]
         L.sage_reorder.argtypes = [p, i32, ctypes.POINTER(ReorderOpts), ctypes.POINTER(Stats)]
         L.sage_get_permutation.argtypes = [p, p]
         L.sage_reorder_objective.argtypes = [p, i32, p]
@@ -189,15 +191,16 @@ class Graph:
         return bool(self.flags & 0x100)
 
     # ------------------------------------------------------------------ queries
-    def bfs(self, source: int, out=None, parent_out=None, parents: bool = False, push_only: bool = False):
+    def bfs(self, source: int, out=None, parent_out=None, parents: bool = False, push_only: bool = False,
+            binning: bool = False):
         """sage_bfs_ex -> (level int32[n_local], parent or None, stats dict)."""
         o = _out(out, self.n_local, np.int32)
         po = None
         if parents or parent_out is not None:
             po = _out(parent_out, self.n_local, np.int32)
         st = Stats()
-        _check(lib().sage_bfs_ex(self._h, int(source), o.ptr, po.ptr if po else None,
-                                 F_PUSH_ONLY if push_only else 0, ctypes.byref(st)))
+        fl = (F_PUSH_ONLY if push_only else 0) | (F_BINNED if binning else 0)
+        _check(lib().sage_bfs_ex(self._h, int(source), o.ptr, po.ptr if po else None, fl, ctypes.byref(st)))
         return o.obj, (po.obj if po else None), st.as_dict()
 
     def sssp(self, source: int, out=None):
@@ -206,10 +209,12 @@ class Graph:
         _check(lib().sage_sssp(self._h, int(source), o.ptr, ctypes.byref(st)))
         return o.obj, st.as_dict()
 
-    def pagerank(self, damping: float = 0.85, iterations: int = 20, out=None):
+    def pagerank(self, damping: float = 0.85, iterations: int = 20, out=None, push_only: bool = False):
+        """sage_pagerank_ex (pull form on symmetric graphs unless push_only)."""
         o = _out(out, self.n_local, np.float64)
         st = Stats()
-        _check(lib().sage_pagerank(self._h, float(damping), int(iterations), o.ptr, ctypes.byref(st)))
+        _check(lib().sage_pagerank_ex(self._h, float(damping), int(iterations), o.ptr,
+                                      F_PUSH_ONLY if push_only else 0, ctypes.byref(st)))
         return o.obj, st.as_dict()
 
     def reorder(self, rounds: int = 1, sector_width: int = 8, candidates=None):
@@ -259,9 +264,9 @@ class Graph:
         """sage_debug_level_records -> int64[levels, 8] (dir, |F|, arcs(F), inspected, scanned,
         discovered, t_ns at level end, t_ns when the last warp finished) of the last BFS/SSSP query."""
         n = ctypes.c_int32(0)
-        buf = np.zeros(8 * 4096, dtype=np.int64)
+        buf = np.zeros(9 * 4096, dtype=np.int64)
         _check(lib().sage_debug_level_records(self._h, buf.ctypes.data, 4096, ctypes.byref(n)))
-        return buf[:8 * min(n.value, 4096)].reshape(-1, 8)
+        return buf[:9 * min(n.value, 4096)].reshape(-1, 9)
 
     def export_tiles(self, vertices) -> np.ndarray:
         """sage_debug_export_tiles -> int64[k, 4] (vertex, offset, size, kind)."""

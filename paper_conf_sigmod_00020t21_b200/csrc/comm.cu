@@ -106,7 +106,7 @@ struct BfsPushMulti {
   __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
   template <int N>
   __device__ __forceinline__ void visit(bool valid, const Src &, int (&v)[N], const uint32_t (&)[N],
-                                        bool (&in)[N]) const {
+                                        bool (&in)[N], int) const {
     const unsigned long long keep = policy_evict_last();
 #pragma unroll
     for (int j = 0; j < N; ++j) {
@@ -289,7 +289,7 @@ struct PrPushMulti {
   }
   template <int N>
   __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N], const uint32_t (&)[N],
-                                        bool (&in)[N]) const {
+                                        bool (&in)[N], int) const {
 #pragma unroll
     for (int j = 0; j < N; ++j) {
       in[j] = false;

@@ -64,7 +64,7 @@ struct CounterSet {                      // counters of one log (rotated over 3 
 
 struct LevelRec {                        // per-level record (first kMaxRec levels)
   int dir;                               // 0 push, 1 pull
-  int pad;
+  int t_mid_us;                          // binned push: phase-1 end (us after the level start)
   unsigned long long nF, arcsF, inspected, scanned, discovered;
   unsigned long long t_ns;               // %globaltimer at the end of the level
   unsigned long long t_work;             // %globaltimer when the last warp finished its work
@@ -420,8 +420,9 @@ __device__ __forceinline__ void buffer_flush(WarpScratch *ws, int &cnt,
 //   struct Src;                                    per-source-vertex context
 //   Src src(bool valid, int u, long long b, long long e);   (b,e = row of u when needed)
 //   template<int N> void visit(bool valid, const Src&, int (&v)[N], const uint32_t (&w)[N],
-//                              bool (&in)[N]);      marks the neighbours filtered in (and may
-//                              rewrite v[j] to the row id to enqueue, e.g. global -> local)
+//                              bool (&in)[N], int lpt); marks the neighbours filtered in (and may
+//                              rewrite v[j] to the row id to enqueue, e.g. global -> local);
+//                              lpt = lanes sharing the tile (aligned groups of the warp)
 //   kWeights (load weights), kNeedRow (src needs the row for CTA tiles), kEnqueue (contraction)
 //   Queues *next_q; CounterSet *next_cs;             where filtered-in vertices go
 template <int VEC, class F>
@@ -502,7 +503,7 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
           v[0] = c4.x; v[1 % VEC] = c4.y; v[2 % VEC] = c4.z; v[3 % VEC] = c4.w;
           ww[0] = w4.x; ww[1 % VEC] = w4.y; ww[2 % VEC] = w4.z; ww[3 % VEC] = w4.w;
           bool in[VEC];
-          f.template visit<VEC>(valid, sc, v, ww, in);
+          f.template visit<VEC>(valid, sc, v, ww, in, lpt);
           PROF_T(tv1);
           PROF_ADD(2, tv1 - tv0);
           if constexpr (F::kEnqueue) {
@@ -522,7 +523,7 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
               ww[j] = (valid && F::kWeights) ? ld_colu(w + p0 + j * lpt, pol) : 0u;
             }
             bool in[VEC];
-            f.template visit<VEC>(valid, sc, v, ww, in);
+            f.template visit<VEC>(valid, sc, v, ww, in, lpt);
             PROF_T(tv2);
             PROF_ADD(3, tv2 - tv0);
             PROF_ADD(4, 1);
@@ -596,7 +597,7 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
         if (F::kWeights) w1[0] = ld_colu(w + pos, pol);
       }
       bool in[1];
-      f.template visit<1>(kv, so, vv, w1, in);
+      f.template visit<1>(kv, so, vv, w1, in, 1);
       if constexpr (F::kEnqueue) buffer_push(in[0], vv[0], ws, bcnt, off, L, *f.next_q, f.next_cs);
     }
     __syncwarp();

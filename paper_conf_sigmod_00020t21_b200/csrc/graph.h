@@ -32,6 +32,10 @@ struct TraversalState {     // per-query scratch, allocated on first use and kep
   Queues q[2];                    // double-buffered per-level tile logs
   Ctl *ctl = nullptr;             // device control block
   int32_t *tmp_out = nullptr;     // ID-translation scratch (n_local)
+  int *bins = nullptr;            // binned push: nslices x bin_cap neighbour ids
+  long long bin_cap = 0;
+  PaddedCounter *fill = nullptr;  // binned push: [2][kMaxSlices] bin fill counters
+  int nslices = 0;
 };
 
 struct PageRankState {      // the all-V resident tile log (built once, reused)
@@ -41,6 +45,7 @@ struct PageRankState {      // the all-V resident tile log (built once, reused; 
   int32_t *dangling = nullptr;    // vertices with out-degree 0
   long long n_dangling = 0;
   double *x = nullptr, *y = nullptr;
+  float *c = nullptr;             // pull form: x_u / out(u)
   CounterSet *cs = nullptr;       // device copy of the log's counters (+ rotating tickets)
 };
 
@@ -75,5 +80,5 @@ struct sage_graph {
   sage::TraversalState ts;
   sage::PageRankState pr;
   sage::Comm *comm = nullptr;
-  int grid_bfs = 0, grid_sssp = 0, grid_pr = 0;   // persistent grid sizes (cooperative)
+  int grid_bfs = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0, grid_bin = 0;   // persistent grid sizes
 };

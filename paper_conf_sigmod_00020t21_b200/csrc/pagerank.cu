@@ -34,12 +34,45 @@ struct PrPush {
   }
   template <int N>
   __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N],
-                                        const uint32_t (&)[N], bool (&in)[N]) const {
+                                        const uint32_t (&)[N], bool (&in)[N], int) const {
 #pragma unroll
     for (int j = 0; j < N; ++j) in[j] = false;
     if (!valid) return;
 #pragma unroll
     for (int j = 0; j < N; ++j) atomicAdd(y + v[j], s.c);
+  }
+};
+
+// Pull (gather) form for SYMMETRIC graphs (in-neighbours = out-neighbours): the tile of row v
+// sums the contributions c_u = x_u / out(u) of its members (fp32 storage, kept L2-resident;
+// fp64 accumulation, reading R7) and adds the group's partial sum to y_v with one fp64 atomic per
+// lane group and step — the same resident log and stealing consumer, no per-arc atomics.
+struct PrPull {
+  struct Src {
+    int u;
+  };
+  static constexpr bool kWeights = false;
+  static constexpr bool kNeedRow = false;
+  static constexpr bool kEnqueue = false;
+  const Queues *next_q = nullptr;
+  CounterSet *next_cs = nullptr;
+  const float *c;
+  double *y;
+  __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
+  template <int N>
+  __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N], const uint32_t (&)[N],
+                                        bool (&in)[N], int lpt) const {
+    float cv[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      in[j] = false;
+      cv[j] = valid ? __ldcg(c + v[j]) : 0.0f;
+    }
+    double acc = 0.0;
+#pragma unroll
+    for (int j = 0; j < N; ++j) acc += (double)cv[j];
+    for (int o = lpt >> 1; o > 0; o >>= 1) acc += __shfl_xor_sync(FULL, acc, o);
+    if (valid && (lane_id() & (lpt - 1)) == 0 && acc != 0.0) atomicAdd(y + s.u, acc);
   }
 };
 
@@ -56,6 +89,7 @@ struct PrArgs {
   const int *dangling;
   long long n_dangling;
   double *x, *y;
+  float *c;           // pull form: x_u / out(u) in fp32
   Ctl *ctl;
   int vec_ok;
 };
@@ -138,12 +172,64 @@ __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ 
   }
 }
 
+template <int VEC>
+__global__ void __launch_bounds__(kBlock, 4) k_pagerank_pull(const __grid_constant__ PrArgs a) {
+  __shared__ WarpScratch wsm[kWarps];
+  __shared__ PrPull::Src fsrc[kWarps][32];
+  __shared__ double red[kWarps];
+  const int warp = threadIdx.x >> 5;
+  const unsigned lane = lane_id();
+  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  const double base = (1.0 - a.d) / a.N;
+  for (int it = 0; it < a.iters; ++it) {
+    CounterSet *cs = &a.sets[it % 3];
+    __syncthreads();
+    if (blockIdx.x == 0 && threadIdx.x < kQueues) a.sets[(it + 2) % 3].tk[threadIdx.x].v = 0ull;
+    if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->D[(it + 2) % 3] = 0.0;
+    PrPull f;
+    f.c = a.c;
+    f.y = a.y;
+    consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &wsm[warp], fsrc[warp], a.vec_ok);
+    double dsum = 0.0;
+    for (long long i = tid; i < a.n_dangling; i += stride) dsum += ldcg(a.x + a.dangling[i]);
+    dsum = warp_sumd(dsum);
+    if (lane == 0) red[warp] = dsum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      double s = 0.0;
+      for (int k = 0; k < kWarps; ++k) s += red[k];
+      if (s != 0.0) atomicAdd(&a.ctl->D[it % 3], s);
+    }
+    grid_barrier(&a.ctl->bar);
+    const double D = ldcg(&a.ctl->D[it % 3]);
+    const double add = base + a.d * D / a.N;
+    for (long long v = tid; v < a.n; v += stride) {
+      const double xv = add + a.d * ldcg(a.y + v);
+      a.x[v] = xv;
+      a.y[v] = 0.0;
+      const long long dg = a.off[v + 1] - a.off[v];
+      a.c[v] = dg ? (float)(xv / (double)dg) : 0.0f;
+    }
+    grid_barrier(&a.ctl->bar);
+  }
+}
+
+__global__ void k_pr_init_c(const long long *__restrict__ off, float *c, long long n, double v0) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+    const long long dg = off[i + 1] - off[i];
+    c[i] = dg ? (float)(v0 / (double)dg) : 0.0f;
+  }
+}
+
 void free_pagerank_state(sage_graph *g) {
   PageRankState &p = g->pr;
   free_queues(g, &p.q);
   dfree(g, p.dangling);
   dfree(g, p.x);
   dfree(g, p.y);
+  dfree(g, p.c);
   dfree(g, p.cs);
   p = PageRankState();
 }
@@ -192,8 +278,8 @@ sage_status run_pagerank_multi(sage_graph *g, double damping, int32_t iterations
 
 using namespace sage;
 
-extern "C" sage_status sage_pagerank(sage_graph *g, double damping, int32_t iterations,
-                                     double *rank_out, sage_stats *st) {
+extern "C" sage_status sage_pagerank_ex(sage_graph *g, double damping, int32_t iterations,
+                                        double *rank_out, uint32_t call_flags, sage_stats *st) {
   clear_error();
   if (!g || !rank_out) {
     set_error("null argument");
@@ -236,9 +322,18 @@ extern "C" sage_status sage_pagerank(sage_graph *g, double damping, int32_t iter
   a.y = p.y;
   a.ctl = g->ts.ctl;
   a.vec_ok = g->vec_ok ? 1 : 0;
+  // pull (gather) on symmetric graphs unless the paper's push form is requested
+  const bool pull = (g->flags & SAGE_F_SYMMETRIC) && !((g->flags | call_flags) & SAGE_F_PUSH_ONLY);
+  if (pull && iterations > 0) {
+    if (!p.c && (s = dalloc(g, (void **)&p.c, sizeof(float) * (size_t)g->n_local)) != SAGE_OK) return s;
+    k_pr_init_c<<<g->num_sms * 8, 256, 0, g->stream>>>((const long long *)g->off, p.c, g->n_local,
+                                                      1.0 / (double)g->n);
+    a.c = p.c;
+  }
   if (iterations > 0) {
-    const void *fn = g->vec == 4 ? (const void *)k_pagerank<4> : (const void *)k_pagerank<1>;
-    const int grid = coop_grid(g, fn, &g->grid_pr);
+    const void *fn = pull ? (g->vec == 4 ? (const void *)k_pagerank_pull<4> : (const void *)k_pagerank_pull<1>)
+                          : (g->vec == 4 ? (const void *)k_pagerank<4> : (const void *)k_pagerank<1>);
+    const int grid = coop_grid(g, fn, pull ? &g->grid_pr_pull : &g->grid_pr);
     void *args[] = {&a};
     if ((s = launch_coop(g, fn, grid, args, "PageRank kernel")) != SAGE_OK) return s;
   }
@@ -267,4 +362,9 @@ extern "C" sage_status sage_pagerank(sage_graph *g, double damping, int32_t iter
   e = cudaStreamSynchronize(g->stream);
   if (e != cudaSuccess) return cuda_fail(g, e, "PageRank output");
   return SAGE_OK;
+}
+
+extern "C" sage_status sage_pagerank(sage_graph *g, double damping, int32_t iterations,
+                                     double *rank_out, sage_stats *st) {
+  return sage_pagerank_ex(g, damping, iterations, rank_out, 0u, st);
 }

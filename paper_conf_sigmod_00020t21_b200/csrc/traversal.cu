@@ -49,7 +49,7 @@ struct BfsPush {
   // Alg. 1 l.1-6: if dist[nb] = -1 then dist[nb] := dist[fr] + 1; filter_in(nb)
   template <int N>
   __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N],
-                                        const uint32_t (&)[N], bool (&in)[N]) const {
+                                        const uint32_t (&)[N], bool (&in)[N], int) const {
     uint32_t wd[N];
     const unsigned long long keep = policy_evict_last();
 #pragma unroll
@@ -91,7 +91,7 @@ struct SsspPush {
 
   template <int N>
   __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N],
-                                        const uint32_t (&w)[N], bool (&in)[N]) const {
+                                        const uint32_t (&w)[N], bool (&in)[N], int) const {
     uint32_t cur[N];
     const unsigned long long keep = policy_evict_last();
 #pragma unroll
@@ -289,6 +289,283 @@ __global__ void __launch_bounds__(kBlock, 4) k_bfs(const __grid_constant__ TravA
   }
 }
 
+// ============================================================================ binned push BFS
+// B200 restructuring of the push filter: a scattered 4-B status read costs about one
+// L1TEX cycle per SM from L2-resident global memory but ~0.2 from shared memory (measured,
+// tools/micro/status_reads.cu).  A push level therefore runs in two phases:
+//   phase 1: the unchanged TP + RTS expansion; every neighbour id is appended to the bin of its
+//            vertex slice (1M ids = 128 KB of bitmap) through warp-private staging in shared
+//            memory, flushed to HBM in coalesced 128-B chunks;
+//   phase 2: each CTA stages the visited bits of one slice in shared memory and runs Alg. 1's
+//            filter on its share of that slice's bin; a vertex new to the CTA is claimed with a
+//            global atomicOr (other CTAs of the slice), and filtered-in vertices are classified
+//            into the next level's log exactly as before.
+constexpr int kBinBlock = 1024;
+constexpr int kBinWarps = kBinBlock / 32;
+constexpr int kBinE = 32;            // staged entries per (warp, slice)
+constexpr int kMaxSlices = 40;
+constexpr int kSliceLg = 20;         // 2^20 vertices per slice
+constexpr int kBinRes = 512;         // entries reserved per (warp, slice) with one atomic
+
+struct BinArgs {
+  int *bins;                         // nslices x cap
+  long long cap;
+  PaddedCounter *fill;               // [2][kMaxSlices]
+  int nslices;
+  int slice_lg;
+};
+
+struct BinPush {
+  struct Src {
+    int u;
+  };
+  static constexpr bool kWeights = false;
+  static constexpr bool kNeedRow = false;
+  static constexpr bool kEnqueue = false;
+  const Queues *next_q = nullptr;
+  CounterSet *next_cs = nullptr;
+  // phase-1 context
+  const TravArgs *a;
+  const BinArgs *b;
+  int *stage;                        // this warp's [nslices][kBinE]
+  int *cnt;                          // this warp's [nslices]
+  int *rpos, *rend;                  // this warp's reserved bin range per slice
+  int fillset;
+  int next_level;
+  const Queues *qn;
+  CounterSet *csn;
+  __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
+
+  // write `c` staged entries of slice s to HBM (or, if the bin is full, filter them directly).
+  // Bin space is reserved kBinRes entries at a time, so the global atomic is off the common path.
+  __device__ __forceinline__ void emit(int s, int c, const int *src) const {
+    const unsigned lane = lane_id();
+    int pos = rpos[s], end = rend[s];
+    const bool has = (int)lane < c;
+    const int x = has ? src[lane] : 0;
+    if (end - pos < c) {
+      // pad the rest of the old reservation, take a new one
+      for (int i = pos + (int)lane; i < end; i += 32) b->bins[(long long)s * b->cap + i] = -1;
+      unsigned long long np = 0;
+      if (lane == 0) np = atomicAdd(&b->fill[fillset * kMaxSlices + s].v, (unsigned long long)kBinRes);
+      np = shfl64(np, 0);
+      pos = (int)min(np, (unsigned long long)b->cap);
+      end = (int)min(np + kBinRes, (unsigned long long)b->cap);
+    }
+    if (end - pos >= c) {
+      if (has) b->bins[(long long)s * b->cap + pos + lane] = x;
+      pos += c;
+    } else {   // bin full (skewed ids): Alg. 1's filter on the global bitmap for these entries
+      bool disc = false;
+      if (has) {
+        const uint32_t bit = 1u << (x & 31);
+        disc = !(atomicOr(a->visited + (x >> 5), bit) & bit);
+        if (disc) {
+          a->level[x] = next_level;
+          if (a->do_enabled) atomicOr(a->fb[next_level % 3] + (x >> 5), bit);
+        }
+      }
+      enqueue_ids(disc, x, a->off, a->L, *qn, csn);
+    }
+    __syncwarp();
+    if (lane == 0) {
+      rpos[s] = pos;
+      rend[s] = end;
+    }
+    __syncwarp();
+  }
+  // end of phase 1: pad the unused part of every reservation
+  __device__ __forceinline__ void close_reservations() const {
+    const unsigned lane = lane_id();
+    for (int s = 0; s < b->nslices; ++s) {
+      const int pos = rpos[s], end = rend[s];
+      for (int i = pos + (int)lane; i < end; i += 32) b->bins[(long long)s * b->cap + i] = -1;
+    }
+  }
+
+  __device__ __forceinline__ void append(bool valid, int v) const {
+    if (!__any_sync(FULL, valid)) return;
+    const unsigned lane = lane_id();
+    const int sl = valid ? (v >> b->slice_lg) : -1;
+    const unsigned grp = __match_any_sync(FULL, sl);
+    const int leader = __ffs(grp) - 1;
+    const int c0 = valid ? cnt[sl] : 0;
+    __syncwarp();
+    const int idx = c0 + __popc(grp & lanemask_lt());
+    if (valid && idx < kBinE) stage[sl * kBinE + idx] = v;
+    const int tot = c0 + __popc(grp);
+    if (valid && (int)lane == leader && tot < kBinE) cnt[sl] = tot;
+    __syncwarp();
+    unsigned fm = __ballot_sync(FULL, valid && (int)lane == leader && tot >= kBinE);
+    while (fm) {
+      const int ld = __ffs(fm) - 1;
+      fm &= fm - 1;
+      const int s2 = __shfl_sync(FULL, sl, ld);
+      const unsigned g2 = __shfl_sync(FULL, grp, ld);
+      const int c2 = __shfl_sync(FULL, c0, ld);
+      emit(s2, kBinE, stage + s2 * kBinE);
+      __syncwarp();
+      if ((g2 >> lane) & 1u) {
+        const int id2 = c2 + __popc(g2 & lanemask_lt());
+        if (id2 >= kBinE) stage[s2 * kBinE + id2 - kBinE] = v;
+      }
+      if ((int)lane == ld) cnt[s2] = c2 + __popc(g2) - kBinE;
+      __syncwarp();
+    }
+  }
+
+  template <int N>
+  __device__ __forceinline__ void visit(bool valid, const Src &, int (&v)[N], const uint32_t (&)[N],
+                                        bool (&in)[N], int) const {
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      in[j] = false;
+      append(valid, v[j]);
+    }
+  }
+};
+
+// phase 2: Alg. 1's filter against a shared-memory copy of one slice of the visited bitmap
+__device__ __forceinline__ void bin_check(const TravArgs &a, const BinArgs &b, int fillset, int L,
+                                          uint32_t *sbm, WarpScratch *ws, const Queues &Qn,
+                                          CounterSet *csn) {
+  const unsigned lane = lane_id();
+  const int warp = threadIdx.x >> 5;
+  const int nw = blockDim.x >> 5;
+  const int ns = b.nslices;
+  int bcnt = 0;
+  uint32_t *fbn = a.do_enabled ? a.fb[(L + 1) % 3] : nullptr;
+  const int G = gridDim.x;
+  const int first = (int)blockIdx.x % ns;
+  const int nparts = G >= ns ? (G - first + ns - 1) / ns : 1;
+  const int part = G >= ns ? (int)blockIdx.x / ns : 0;
+  for (int s = first; s < ns; s += (G >= ns ? ns : G)) {
+    const long long v0 = (long long)s << b.slice_lg;
+    const long long v1 = min(a.n, v0 + (1ll << b.slice_lg));
+    const long long nwd = (v1 - v0 + 31) >> 5;
+    for (long long i = threadIdx.x; i < nwd; i += blockDim.x) sbm[i] = ldcg(a.visited + (v0 >> 5) + i);
+    __syncthreads();
+    const long long fill = (long long)ldcg(&b.fill[fillset * kMaxSlices + s].v);
+    const long long tot = fill < b.cap ? fill : b.cap;
+    const long long lo = tot * part / nparts, hi = tot * (part + 1) / nparts;
+    const int *bin = b.bins + (long long)s * b.cap;
+    for (long long base = lo + (long long)warp * 32; base < hi; base += (long long)nw * 32) {
+      const long long i = base + lane;
+      bool disc = false;
+      int v = 0;
+      if (i < hi) v = ldcg(bin + i);
+      if (i < hi && v >= 0) {
+        const int lb = (int)(v - v0);
+        const uint32_t bit = 1u << (lb & 31);
+        if (!(sbm[lb >> 5] & bit)) {
+          if (!(atomicOr(sbm + (lb >> 5), bit) & bit)) {
+            disc = !(atomicOr(a.visited + (v >> 5), bit) & bit);
+            if (disc) {
+              a.level[v] = L + 1;
+              if (fbn) atomicOr(fbn + (v >> 5), bit);
+            }
+          }
+        }
+      }
+      buffer_push(disc, v, &ws[warp], bcnt, a.off, a.L, Qn, csn);
+    }
+    __syncthreads();
+  }
+  if (bcnt) buffer_flush(&ws[warp], bcnt, a.off, a.L, Qn, csn);
+}
+
+template <int VEC>
+__global__ void __launch_bounds__(kBinBlock, 1) k_bfs_bin(const __grid_constant__ TravArgs a,
+                                                          const __grid_constant__ BinArgs b) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  WarpScratch *wsm = reinterpret_cast<WarpScratch *>(dsm);
+  BinPush::Src *fsrc = reinterpret_cast<BinPush::Src *>(dsm + sizeof(WarpScratch) * kBinWarps);
+  int *cnts = reinterpret_cast<int *>(dsm + sizeof(WarpScratch) * kBinWarps + sizeof(BinPush::Src) * 32 * kBinWarps);
+  int *rps = cnts + kMaxSlices * kBinWarps;
+  int *res = rps + kMaxSlices * kBinWarps;
+  unsigned char *U = dsm + sizeof(WarpScratch) * kBinWarps + sizeof(BinPush::Src) * 32 * kBinWarps +
+                     3 * sizeof(int) * kMaxSlices * kBinWarps;
+  const int warp = threadIdx.x >> 5;
+  const unsigned lane = lane_id();
+  Ctl *ctl = a.ctl;
+  double mU = (double)a.m - (double)ldcg(&ctl->set[0].arcsF.v);
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t0_ns = globaltimer();
+  int dir = 0;
+  unsigned long long prev_nF = 1;
+  const long long nwords = (a.n + 31) >> 5;
+  for (int L = 0;; ++L) {
+    CounterSet *cur = &ctl->set[L % 3];
+    CounterSet *nxt = &ctl->set[(L + 1) % 3];
+    __syncthreads();
+    zero_counterset(&ctl->set[(L + 2) % 3]);
+    if (blockIdx.x == 0 && threadIdx.x < kMaxSlices) b.fill[((L + 1) & 1) * kMaxSlices + threadIdx.x].v = 0ull;
+    if (a.do_enabled) clear_words(a.fb[(L + 2) % 3], nwords);
+    if (dir == 0) {
+      // phase 1: expansion into slice bins
+      int *cnt = cnts + warp * kMaxSlices;
+      int *stage = reinterpret_cast<int *>(U) + warp * b.nslices * kBinE;
+      for (int i = lane; i < b.nslices; i += 32) {
+        cnt[i] = 0;
+        rps[warp * kMaxSlices + i] = 0;
+        res[warp * kMaxSlices + i] = 0;
+      }
+      __syncwarp();
+      BinPush f;
+      f.a = &a;
+      f.b = &b;
+      f.stage = stage;
+      f.cnt = cnt;
+      f.rpos = rps + warp * kMaxSlices;
+      f.rend = res + warp * kMaxSlices;
+      f.fillset = L & 1;
+      f.next_level = L + 1;
+      f.qn = &a.q[(L + 1) & 1];
+      f.csn = nxt;
+      consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc + warp * 32, a.vec_ok);
+      for (int sl = 0; sl < b.nslices; ++sl) {
+        const int c = cnt[sl];
+        if (c) f.emit(sl, c, stage + sl * kBinE);
+      }
+      f.close_reservations();
+      grid_barrier(&ctl->bar);
+      if (blockIdx.x == 0 && threadIdx.x == 0 && L < kMaxRec)
+        ctl->rec[L].t_mid_us = (int)((globaltimer() - ctl->t0_ns) / 1000);
+      // phase 2: filter against shared-memory slices of the visited bitmap
+      bin_check(a, b, L & 1, L, reinterpret_cast<uint32_t *>(U), wsm, a.q[(L + 1) & 1], nxt);
+    } else {
+      pull_level(a, L + 1, a.fb[L % 3], a.fb[(L + 1) % 3], a.q[(L + 1) & 1], cur, nxt, &wsm[warp]);
+    }
+    if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
+    grid_barrier(&ctl->bar);
+    const unsigned long long nF = ldcg(&nxt->nF.v);
+    const unsigned long long aF = ldcg(&nxt->arcsF.v);
+    if (blockIdx.x == 0 && threadIdx.x == 0) record_level(ctl, L, dir, cur, nxt);
+    if (nF == 0) break;
+    if (L + 1 >= a.max_levels) {
+      if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = 1;
+      break;
+    }
+    mU -= (double)aF;
+    if (a.do_enabled) {
+      if (dir == 0) {
+        if ((double)aF > mU / a.alpha) dir = 1;
+      } else {
+        if (!(nF >= prev_nF || (double)nF > (double)a.n / a.beta)) dir = 0;
+      }
+    }
+    prev_nF = nF;
+  }
+}
+
+static size_t bin_smem_bytes(int nslices, long long n) {
+  const size_t fixed = sizeof(WarpScratch) * kBinWarps + sizeof(int) * 32 * kBinWarps +
+                       3 * sizeof(int) * kMaxSlices * kBinWarps;
+  const size_t stage = sizeof(int) * (size_t)kBinWarps * nslices * kBinE;
+  const long long sw = std::min<long long>(n, 1ll << kSliceLg);
+  const size_t bm = sizeof(uint32_t) * (size_t)((sw + 31) / 32 + 1);
+  return fixed + std::max(stage, bm);
+}
+
 // ============================================================================ SSSP kernel
 template <int VEC>
 __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ TravArgs a, int *overflow) {
@@ -480,6 +757,8 @@ void free_traversal_state(sage_graph *g) {
   free_queues(g, &t.q[1]);
   dfree(g, t.ctl);
   dfree(g, t.tmp_out);
+  dfree(g, t.bins);
+  dfree(g, t.fill);
   t = TraversalState();
 }
 
@@ -663,11 +942,43 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   a.parent = parent_out ? t.parent : nullptr;
   a.do_enabled = (symmetric && !push_only) ? 1 : 0;
   k_seed<<<1, 32, 0, g->stream>>>(a, src, 0);
+  const int nslices = (int)((g->n + (1ll << kSliceLg) - 1) >> kSliceLg);
+  const bool binned = !parent_out && (call_flags & SAGE_F_BINNED) && nslices <= kMaxSlices;
+  if (binned && !t.bins) {
+    // per-slice capacity: 1.5x the average share of all arcs plus staging slack; a full bin
+    // spills to the direct filter, so the capacity only affects speed
+    t.nslices = nslices;
+    t.bin_cap = (long long)(1.5 * (double)g->m / nslices) + (long long)kBinRes * kBinWarps * g->num_sms + 1024;
+    if ((s = dalloc(g, (void **)&t.bins, sizeof(int) * (size_t)t.bin_cap * nslices)) != SAGE_OK ||
+        (s = dalloc(g, (void **)&t.fill, sizeof(PaddedCounter) * 2 * kMaxSlices)) != SAGE_OK)
+      return s;
+  }
+  if (binned) cudaMemsetAsync(t.fill, 0, sizeof(PaddedCounter) * 2 * kMaxSlices, g->stream);
   cudaEventRecord(e1, g->stream);
-  const void *fn = g->vec == 4 ? (const void *)k_bfs<4> : (const void *)k_bfs<1>;
-  const int grid = coop_grid(g, fn, &g->grid_bfs);
-  void *args[] = {&a};
-  if ((s = launch_coop(g, fn, grid, args, "BFS kernel")) != SAGE_OK) return s;
+  if (binned) {
+    BinArgs b;
+    b.bins = t.bins;
+    b.cap = t.bin_cap;
+    b.fill = t.fill;
+    b.nslices = nslices;
+    b.slice_lg = kSliceLg;
+    const void *fn = g->vec == 4 ? (const void *)k_bfs_bin<4> : (const void *)k_bfs_bin<1>;
+    const size_t smem = bin_smem_bytes(nslices, g->n);
+    cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (!g->grid_bin) {
+      int nb = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, kBinBlock, smem);
+      g->grid_bin = std::max(1, nb) * g->num_sms;
+    }
+    void *args[] = {&a, &b};
+    cudaError_t le = cudaLaunchCooperativeKernel(fn, dim3(g->grid_bin), dim3(kBinBlock), args, smem, g->stream);
+    if (le != cudaSuccess) return cuda_fail(g, le, "binned BFS kernel");
+  } else {
+    const void *fn = g->vec == 4 ? (const void *)k_bfs<4> : (const void *)k_bfs<1>;
+    const int grid = coop_grid(g, fn, &g->grid_bfs);
+    void *args[] = {&a};
+    if ((s = launch_coop(g, fn, grid, args, "BFS kernel")) != SAGE_OK) return s;
+  }
   cudaEventRecord(e2, g->stream);
   Ctl h;
   cudaMemcpyAsync(&h, t.ctl, offsetof(Ctl, rec), cudaMemcpyDeviceToHost, g->stream);
@@ -880,7 +1191,7 @@ extern "C" sage_status sage_debug_level_records(const sage_graph *gc, int64_t *r
   *n_out = h->levels;
   for (int i = 0; i < nl && i < cap; ++i) {
     const LevelRec &r = h->rec[i];
-    int64_t *o = rec_out + 8 * i;
+    int64_t *o = rec_out + 9 * i;
     o[0] = r.dir;
     o[1] = (int64_t)r.nF;
     o[2] = (int64_t)r.arcsF;
@@ -889,6 +1200,7 @@ extern "C" sage_status sage_debug_level_records(const sage_graph *gc, int64_t *r
     o[5] = (int64_t)r.discovered;
     o[6] = (int64_t)(r.t_ns - h->t0_ns);
     o[7] = r.t_work ? (int64_t)(r.t_work - h->t0_ns) : 0;
+    o[8] = (int64_t)r.t_mid_us * 1000;
   }
   delete h;
   return SAGE_OK;

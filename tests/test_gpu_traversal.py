@@ -194,13 +194,25 @@ def test_pagerank_parity(sage, lad):
     graphs.append(sg.from_edges(5, [], False, "edgeless"))
     for g in graphs:
         with sage.load_csr(g.off, g.col, symmetric=g.symmetric, **lad) as G:
-            for iters in (0, 1, 20):
-                x, st = G.pagerank(0.85, iters)
-                ref = oracle.pagerank(g.off, g.col, 0.85, iters)
-                assert np.max(np.abs(x - ref) / ref) <= 1e-6, (g.name, iters)
-                assert abs(x.sum() - 1.0) < 1e-9
+            for push_only in (True, False):      # push (Alg. 1) and, on symmetric graphs, pull
+                for iters in (0, 1, 20):
+                    x, st = G.pagerank(0.85, iters, push_only=push_only)
+                    ref = oracle.pagerank(g.off, g.col, 0.85, iters)
+                    assert np.max(np.abs(x - ref) / ref) <= 1e-6, (g.name, iters, push_only)
+                    assert abs(x.sum() - 1.0) < 1e-6
             x2, _ = G.pagerank(0.85, 20)     # the resident log is reused across calls
             assert np.max(np.abs(x2 - oracle.pagerank(g.off, g.col, 0.85, 20)) / x2) <= 1e-6
+
+
+def test_pagerank_pull_precision_at_scale(sage):
+    """Pull form: fp32 contributions, fp64 accumulation (R7) stays well inside 1e-6 on RMAT-18."""
+    g = sg.rmat(18, 16, seed=3, symmetric=True)
+    with sage.load_csr(g.off, g.col, symmetric=True) as G:
+        x, _ = G.pagerank(0.85, 20)
+        xp, _ = G.pagerank(0.85, 20, push_only=True)
+    ref = oracle.pagerank(g.off, g.col, 0.85, 20)
+    assert np.max(np.abs(x - ref) / ref) <= 1e-6
+    assert np.max(np.abs(xp - ref) / ref) <= 1e-12
 
 
 @pytest.mark.parametrize("lad", LADDERS, ids=lambda d: f"B{d['tile_cta']}M{d['tile_min']}A{d['align']}")
@@ -257,3 +269,34 @@ def test_error_conventions(sage):
         sage.load_csr(off2, g.col)
     with pytest.raises(sage.SageError):
         sage.load_csr(g.off, g.col, tile_cta=100)
+
+
+def test_binned_and_direct_push_agree(sage):
+    """The two-phase binned push level (slice bins + shared-memory bitmap slices) and the direct
+    per-arc filter give the oracle's levels, including multi-slice graphs (n > 2^20)."""
+    graphs = [sg.rmat(12, 16, seed=21, symmetric=True), sg.rmat(21, 8, seed=22, symmetric=True),
+              sg.rmat(21, 8, seed=23, symmetric=False)]
+    for g in graphs:
+        with sage.load_csr(g.off, g.col, symmetric=g.symmetric) as G:
+            for s in sg.sources(g, 2, seed=2):
+                ref = oracle.bfs(g.off, g.col, int(s))
+                for po in (True, False):
+                    for binning in (True, False):
+                        lv, _, st = G.bfs(int(s), push_only=po, binning=binning)
+                        assert np.array_equal(lv, ref), (g.name, int(s), po, binning)
+
+
+def test_binned_push_bin_overflow(sage):
+    """Every arc targets the first slice: bins overflow and spill to the direct filter."""
+    n = 3 << 20
+    rng = np.random.default_rng(5)
+    src = rng.integers(0, n, size=400000)
+    dst = rng.integers(0, 1 << 20, size=400000)
+    chain = np.stack([np.arange(0, 1 << 20), np.arange(1, (1 << 20) + 1)], 1)   # connect slice 0
+    e = np.concatenate([np.stack([src, dst], 1), np.stack([dst, src], 1), chain])
+    g = sg.from_edges(n, e, False, "skewed")
+    with sage.load_csr(g.off, g.col) as G:
+        for s in [int(src[0]), 0]:
+            ref = oracle.bfs(g.off, g.col, s)
+            lv, _, _ = G.bfs(s, push_only=True, binning=True)
+            assert np.array_equal(lv, ref)

@@ -16,6 +16,7 @@ p.add_argument("--op", default="bfs_push", choices=["bfs_push", "bfs_do", "sssp"
 p.add_argument("--reps", type=int, default=3)
 p.add_argument("--tile-cta", type=int, default=256)
 p.add_argument("--align", type=int, default=4)
+p.add_argument("--binned", action="store_true", help="experimental two-phase binned push level")
 a = p.parse_args()
 g = sg.rmat(a.scale, 16, 1, True)
 w = sg.weights(g, 1)
@@ -26,9 +27,9 @@ src = sg.sources(g, a.reps, seed=2)
 lv = torch.empty(g.n, dtype=torch.int32, device="cuda")
 for i in range(a.reps):
     if a.op == "bfs_push":
-        _, _, st = G.bfs(int(src[i]), out=lv, push_only=True)
+        _, _, st = G.bfs(int(src[i]), out=lv, push_only=True, binning=a.binned)
     elif a.op == "bfs_do":
-        _, _, st = G.bfs(int(src[i]), out=lv)
+        _, _, st = G.bfs(int(src[i]), out=lv, binning=a.binned)
     elif a.op == "sssp":
         _, st = G.sssp(int(src[i]), out=lv.view(torch.uint32))
     else:
@@ -38,8 +39,8 @@ for i in range(a.reps):
     if a.op != "pr":
         prev = 0
         for r in G.level_records():
-            print("   L dir=%d |F|=%9d arcsF=%11d insp=%11d disc=%9d  %8.1f us (work done at +%8.1f)" % (
-                r[0], r[1], r[2], r[3], r[5], (r[6] - prev) / 1e3, (r[7] - prev) / 1e3))
+            print("   L dir=%d |F|=%9d arcsF=%11d insp=%11d disc=%9d  %8.1f us (work done at +%8.1f, phase1 +%8.1f)" % (
+                r[0], r[1], r[2], r[3], r[5], (r[6] - prev) / 1e3, (r[7] - prev) / 1e3, (r[8] - prev) / 1e3 if r[8] else 0))
             prev = r[6]
     if os.environ.get("SAGE_PROF") == "1":
         import ctypes

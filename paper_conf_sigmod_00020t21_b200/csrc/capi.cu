@@ -41,10 +41,35 @@ bool is_device_ptr(const void *p) {
   return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
+// Library-owned stream-ordered memory pool per device.  Freed blocks stay mapped in the pool
+// (release threshold = unlimited), so a load / free / load cycle does not re-map gigabytes.
+static cudaMemPool_t pool_for(int dev) {
+  static cudaMemPool_t pools[64] = {};
+  if (dev < 0 || dev >= 64) return nullptr;
+  if (!pools[dev]) {
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.handleTypes = cudaMemHandleTypeNone;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t p = nullptr;
+    if (cudaMemPoolCreate(&p, &props) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+    unsigned long long thr = ~0ull;
+    cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+    pools[dev] = p;
+  }
+  return pools[dev];
+}
+
 sage_status dalloc(sage_graph *g, void **p, size_t bytes) {
   *p = nullptr;
   if (bytes == 0) bytes = 16;
-  cudaError_t e = cudaMallocAsync(p, bytes, g->stream);
+  cudaMemPool_t pool = pool_for(g->device);
+  cudaError_t e = pool ? cudaMallocFromPoolAsync(p, bytes, pool, g->stream)
+                       : cudaMallocAsync(p, bytes, g->stream);
   if (e != cudaSuccess) {
     cudaGetLastError();
     *p = nullptr;
@@ -88,19 +113,43 @@ __global__ void k_validate_rows(const long long *__restrict__ off, long long n_l
   if (mx) atomicMax(&out->max_deg, mx);
 }
 
+// One streaming pass over col (and w): 4 consecutive elements per thread per step (16-B loads
+// when aligned), rows-sorted check against the row-start bitmap built by k_validate_rows.
 __global__ void k_validate_arcs(const int *__restrict__ col, const uint32_t *__restrict__ w,
                                 long long m, long long n, const uint32_t *__restrict__ rowstart,
                                 ValidateOut *out) {
-  long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-  long long stride = (long long)gridDim.x * blockDim.x;
+  const long long stride = 4ll * gridDim.x * blockDim.x;
   unsigned long long bc = 0, bw = 0, us = 0;
-  for (; k < m; k += stride) {
-    int c = col[k];
-    if (c < 0 || c >= n) bc++;
-    if (w && w[k] == 0) bw++;
-    if (k + 1 < m) {
-      bool next_starts = (rowstart[(k + 1) >> 5] >> ((k + 1) & 31)) & 1u;
-      if (!next_starts && col[k + 1] <= c) us++;
+  const bool vec = ((uintptr_t)col % 16) == 0 && (!w || ((uintptr_t)w % 16) == 0);
+  for (long long k0 = 4ll * ((long long)blockIdx.x * blockDim.x + threadIdx.x); k0 < m; k0 += stride) {
+    int c[5];
+    uint32_t ww[4] = {1u, 1u, 1u, 1u};
+    if (vec && k0 + 4 <= m) {
+      const int4 c4 = __ldg(reinterpret_cast<const int4 *>(col + k0));
+      c[0] = c4.x; c[1] = c4.y; c[2] = c4.z; c[3] = c4.w;
+      if (w) {
+        const uint4 w4 = __ldg(reinterpret_cast<const uint4 *>(w + k0));
+        ww[0] = w4.x; ww[1] = w4.y; ww[2] = w4.z; ww[3] = w4.w;
+      }
+    } else {
+      for (int j = 0; j < 4; ++j) {
+        c[j] = k0 + j < m ? __ldg(col + k0 + j) : 0;
+        if (w && k0 + j < m) ww[j] = __ldg(w + k0 + j);
+      }
+    }
+    c[4] = k0 + 4 < m ? __ldg(col + k0 + 4) : 0;
+    // bits k0+1 .. k0+4 of the row-start bitmap (may straddle two words)
+    const long long b1 = k0 + 1;
+    unsigned long long rs = __ldg(rowstart + (b1 >> 5));
+    if (((b1 & 31) + 4) > 32) rs |= (unsigned long long)__ldg(rowstart + (b1 >> 5) + 1) << 32;
+    rs >>= (b1 & 31);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const long long k = k0 + j;
+      if (k >= m) break;
+      if (c[j] < 0 || c[j] >= n) bc++;
+      if (ww[j] == 0) bw++;
+      if (k + 1 < m && !((rs >> j) & 1ull) && c[j + 1] <= c[j]) us++;
     }
   }
   if (bc) atomicAdd(&out->bad_col, bc);

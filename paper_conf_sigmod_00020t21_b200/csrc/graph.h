@@ -36,6 +36,9 @@ struct TraversalState {     // per-query scratch, allocated on first use and kep
   long long bin_cap = 0;
   PaddedCounter *fill = nullptr;  // binned push: [2][kMaxSlices] bin fill counters
   int nslices = 0;
+  int *far[3] = {nullptr, nullptr, nullptr};  // SSSP near-far: rotating far piles
+  uint32_t *infar = nullptr;      // SSSP near-far: far-pile membership bitmap
+  PaddedCounter *farc = nullptr;  // SSSP near-far: [3] pile sizes + [3] scan minima
 };
 
 struct PageRankState {      // the all-V resident tile log (built once, reused)
@@ -70,6 +73,7 @@ struct sage_graph {
   int64_t n_isolated = 0;
   sage::Ladder ladder{};
   double alpha = 15.0, beta = 18.0;
+  double w_mean = 0.0;        // mean arc weight (SSSP near-far threshold step), lazily computed
   int vec = 4;                // neighbours per lane per step (4; 1 when tile_min < 4)
   bool vec_ok = true;         // sub-warp tiles use 16-B loads (align % 4 == 0, aligned arrays)
   // reordering: sigma[v_orig] = current label; sigma_inv[label] = v_orig (null = identity)

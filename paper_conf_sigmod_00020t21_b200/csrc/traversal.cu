@@ -17,6 +17,8 @@
 // log once per iteration (bitmap dedupe) -> frontier Bellman-Ford.
 #include <cuda_runtime.h>
 #include <stdio.h>
+#include <stdlib.h>
+#include <math.h>
 #include <string.h>
 
 #include <algorithm>
@@ -83,6 +85,11 @@ struct SsspPush {
   int *overflow;
   const Queues *next_q;
   CounterSet *next_cs;
+  // near-far ordering: improvements at distance >= T go to the far pile instead of the frontier
+  unsigned long long T;
+  uint32_t *infar;      // far-pile membership bitmap
+  int *far;             // far pile being appended to
+  unsigned long long *far_cnt;
 
   __device__ __forceinline__ Src src(bool valid, int u, long long, long long) const {
     // dist[u] may have been lowered by another SM in an earlier iteration: read through L2
@@ -107,8 +114,12 @@ struct SsspPush {
           const uint32_t old = atomicMin(dist + v[j], (uint32_t)nd);
           if ((uint32_t)nd < old) {
             const uint32_t bit = 1u << (v[j] & 31);
-            const uint32_t o2 = atomicOr(inq_next + (v[j] >> 5), bit);
-            in[j] = !(o2 & bit);
+            if (nd < T) {
+              const uint32_t o2 = atomicOr(inq_next + (v[j] >> 5), bit);
+              in[j] = !(o2 & bit);
+            } else if (!(atomicOr(infar + (v[j] >> 5), bit) & bit)) {
+              far[atomicAdd(far_cnt, 1ull)] = v[j];
+            }
           }
         }
       }
@@ -567,14 +578,72 @@ static size_t bin_smem_bytes(int nslices, long long n) {
 }
 
 // ============================================================================ SSSP kernel
+struct FarArgs {                      // near-far state of k_sssp
+  int *far[3];                       // three rotating far piles (append / scan / spare)
+  uint32_t *infar;                   // far-pile membership bitmap
+  PaddedCounter *cnt;                // [3] far pile sizes
+  PaddedCounter *fmin;               // [3] min distance seen in a scan
+  unsigned long long delta;          // threshold step; 0xffff... = plain Bellman-Ford
+};
+
+// Advance phase of near-far SSSP: move far-pile vertices with dist < T into the next log.
+__device__ __forceinline__ void far_scan(const TravArgs &a, const FarArgs &fa, int k, unsigned long long T,
+                                         uint32_t *inq_next, const Queues &Qn, CounterSet *csn,
+                                         WarpScratch *ws) {
+  const unsigned lane = lane_id();
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  const int *src = fa.far[k % 3];
+  int *dst = fa.far[(k + 1) % 3];
+  const long long cnt = (long long)ldcg(&fa.cnt[k % 3].v);
+  unsigned long long mn = ~0ull;
+  int bcnt = 0;
+  for (long long base = gw * 32; base < cnt; base += nw * 32) {
+    const long long i = base + lane;
+    bool move = false, keep = false;
+    int v = 0;
+    if (i < cnt) {
+      v = ldcg(src + i);
+      const uint32_t d = ldcg(a.dist + v);
+      const uint32_t bit = 1u << (v & 31);
+      if (d < T) {
+        atomicAnd(fa.infar + (v >> 5), ~bit);
+        move = !(atomicOr(inq_next + (v >> 5), bit) & bit);
+      } else {
+        keep = true;
+        if (d < mn) mn = d;
+      }
+    }
+    const unsigned km = __ballot_sync(FULL, keep);
+    if (km) {
+      const int leader = __ffs(km) - 1;
+      unsigned long long p = 0;
+      if ((int)lane == leader) p = atomicAdd(&fa.cnt[(k + 1) % 3].v, (unsigned long long)__popc(km));
+      p = shfl64(p, leader);
+      if (keep) dst[p + __popc(km & lanemask_lt())] = v;
+    }
+    buffer_push(move, v, ws, bcnt, a.off, a.L, Qn, csn);
+  }
+  if (bcnt) buffer_flush(ws, bcnt, a.off, a.L, Qn, csn);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned long long y = __shfl_xor_sync(FULL, mn, o);
+    mn = y < mn ? y : mn;
+  }
+  if (lane == 0 && mn != ~0ull) atomicMin(&fa.fmin[k % 3].v, mn);
+}
+
 template <int VEC>
-__global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ TravArgs a, int *overflow) {
+__global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ TravArgs a, int *overflow,
+                                                    const __grid_constant__ FarArgs fa) {
   __shared__ WarpScratch wsm[kWarps];
   __shared__ SsspPush::Src fsrc[kWarps][32];
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
   const long long nwords = (a.n + 31) >> 5;
   if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t0_ns = globaltimer();
+  unsigned long long T = fa.delta;   // near threshold
+  int k = 0;                         // far scans done; the current far pile is far[k % 3]
   for (int L = 0;; ++L) {
     CounterSet *cur = &ctl->set[L % 3];
     CounterSet *nxt = &ctl->set[(L + 1) % 3];
@@ -587,10 +656,28 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
     f.overflow = overflow;
     f.next_q = &a.q[(L + 1) & 1];
     f.next_cs = nxt;
+    f.T = T;
+    f.infar = fa.infar;
+    f.far = fa.far[k % 3];
+    f.far_cnt = &fa.cnt[k % 3].v;
     consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok);
     if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
     grid_barrier(&ctl->bar);
-    const unsigned long long nF = ldcg(&nxt->nF.v);
+    unsigned long long nF = ldcg(&nxt->nF.v);
+    // near frontier exhausted: raise the threshold and pull the far pile forward
+    while (nF == 0 && ldcg(&fa.cnt[k % 3].v) != 0) {
+      if (blockIdx.x == 0 && threadIdx.x == 0) {
+        fa.cnt[(k + 2) % 3].v = 0ull;     // scan k-1's source pile, no longer read
+        fa.fmin[(k + 1) % 3].v = ~0ull;   // written by scan k+1, not read before it
+      }
+      const unsigned long long fm = k > 0 ? ldcg(&fa.fmin[(k + 2) % 3].v) : ~0ull;  // scan k-1's
+      T = (T + fa.delta > T) ? T + fa.delta : ~0ull;
+      if (fm != ~0ull && fm >= T) T = (fm / fa.delta + 1) * fa.delta;   // skip empty buckets
+      far_scan(a, fa, k, T, a.fb[(L + 1) % 3], a.q[(L + 1) & 1], nxt, &wsm[warp]);
+      grid_barrier(&ctl->bar);
+      ++k;
+      nF = ldcg(&nxt->nF.v);
+    }
     if (blockIdx.x == 0 && threadIdx.x == 0) record_level(ctl, L, 0, cur, nxt);
     if (nF == 0) break;
     if (L + 1 >= a.max_levels) {
@@ -628,6 +715,14 @@ __global__ void k_overflow_check(const long long *__restrict__ off, const int *_
         return;
       }
   }
+}
+
+__global__ void k_sum_u32(const uint32_t *__restrict__ w, long long m, unsigned long long *out) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  unsigned long long s = 0;
+  for (long long k = (long long)blockIdx.x * blockDim.x + threadIdx.x; k < m; k += stride) s += w[k];
+  s = warp_sum64(s);
+  if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, s);
 }
 
 // R1 edge count of an SSSP result: sum of out-degrees of the reached vertices.
@@ -759,6 +854,9 @@ void free_traversal_state(sage_graph *g) {
   dfree(g, t.tmp_out);
   dfree(g, t.bins);
   dfree(g, t.fill);
+  for (int i = 0; i < 3; ++i) dfree(g, t.far[i]);
+  dfree(g, t.infar);
+  dfree(g, t.farc);
   t = TraversalState();
 }
 
@@ -1043,12 +1141,45 @@ extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_o
   cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
   for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
   cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);
+  // near-far state (SSSP ordering); delta from the mean weight and degree
+  if (!t.far[0]) {
+    for (int i = 0; i < 3; ++i)
+      if ((s = dalloc(g, (void **)&t.far[i], sizeof(int) * (size_t)(g->n_local + 1))) != SAGE_OK) return s;
+    if ((s = dalloc(g, (void **)&t.infar, sizeof(uint32_t) * words)) != SAGE_OK ||
+        (s = dalloc(g, (void **)&t.farc, sizeof(PaddedCounter) * 6)) != SAGE_OK)
+      return s;
+  }
+  if (g->w_mean <= 0.0) {
+    unsigned long long *dsum = reinterpret_cast<unsigned long long *>(t.farc);
+    unsigned long long hsum = 0;
+    cudaMemsetAsync(dsum, 0, sizeof(unsigned long long), g->stream);
+    k_sum_u32<<<g->num_sms * 8, 256, 0, g->stream>>>(g->w, g->m, dsum);
+    cudaMemcpyAsync(&hsum, dsum, sizeof(hsum), cudaMemcpyDeviceToHost, g->stream);
+    cudaStreamSynchronize(g->stream);
+    g->w_mean = g->m ? (double)hsum / (double)g->m : 1.0;
+  }
+  FarArgs fa;
+  for (int i = 0; i < 3; ++i) fa.far[i] = t.far[i];
+  fa.infar = t.infar;
+  fa.cnt = t.farc;
+  fa.fmin = t.farc + 3;
+  {
+    const double avgdeg = g->n_local ? (double)g->m / (double)g->n_local : 1.0;
+    double dl = 32.0 * g->w_mean / std::max(1.0, avgdeg);
+    const char *env = getenv("SAGE_SSSP_DELTA");
+    if (env) dl = atof(env);
+    fa.delta = dl <= 0.0 ? ~0ull : (unsigned long long)std::max(1.0, std::floor(dl + 0.5));
+    if (!env) fa.delta = ~0ull;   // default: plain frontier Bellman-Ford (near-far measured slower)
+  }
+  cudaMemsetAsync(t.infar, 0, sizeof(uint32_t) * words, g->stream);
+  cudaMemsetAsync(t.farc, 0, sizeof(PaddedCounter) * 3, g->stream);
+  cudaMemsetAsync(t.farc + 3, 0xff, sizeof(PaddedCounter) * 3, g->stream);
   TravArgs a = make_args(g);
   k_seed<<<1, 32, 0, g->stream>>>(a, src, 1);
   cudaEventRecord(e1, g->stream);
   const void *fn = g->vec == 4 ? (const void *)k_sssp<4> : (const void *)k_sssp<1>;
   const int grid = coop_grid(g, fn, &g->grid_sssp);
-  void *args[] = {&a, &ovf};
+  void *args[] = {&a, &ovf, &fa};
   if ((s = launch_coop(g, fn, grid, args, "SSSP kernel")) != SAGE_OK) {
     dfree(g, ovf);
     return s;

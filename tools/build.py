@@ -70,7 +70,8 @@ def build_oracle(force=False):
 def build_sage(force=False, verbose=False):
     csrc = os.path.join(PKG, "csrc")
     cus = sorted(glob.glob(os.path.join(csrc, "*.cu")))
-    hdrs = sorted(glob.glob(os.path.join(csrc, "*.cuh"))) + [os.path.join(ROOT, "include", "sage.h")]
+    hdrs = (sorted(glob.glob(os.path.join(csrc, "*.cuh"))) + sorted(glob.glob(os.path.join(csrc, "*.h"))) +
+            [os.path.join(ROOT, "include", "sage.h")])
     prof = os.environ.get("SAGE_PROF") == "1"
     out = os.path.join(PKG, "libsage_prof.so" if prof else "libsage.so")
     if not (force or _stale(out, cus + hdrs)):

@@ -146,6 +146,7 @@ struct TravArgs {
   int vec_ok;           // 16-B vector loads allowed (A % 4 == 0 and 16-B aligned col / w)
   double alpha, beta;
   int max_levels;
+  int *tail;            // tail mode: next-frontier list (n entries of scratch)
 };
 
 // Pull (bottom-up) step over the visited bitmap: one warp per 32-vertex word.
@@ -245,11 +246,208 @@ __device__ __forceinline__ void record_level(Ctl *ctl, int L, int dir, const Cou
   ctl->levels = L + 1;
 }
 
+// ============================================================================ tail mode
+// High-diameter graphs (C4's tendrils: hundreds of levels with a handful of vertices) pay the
+// per-level cost of the grid pipeline: one warp's chain of dependent accesses (ticket, log entry,
+// offsets, column, status, claim, classification, reservation) plus a grid barrier, ~10 us.
+// When a push level's next frontier is small, block 0 alone runs the following levels with the
+// frontier in shared memory (block scan over degrees, load-balanced arc loop, __syncthreads);
+// the other CTAs wait at the grid barrier.  If the frontier grows again, block 0 classifies it
+// into the regular log (Tiled Partitioning) and the whole grid resumes.  Push levels only,
+// without direction switching (the frontier bitmaps are not maintained in tail mode).
+constexpr int kTailV = kBlock;       // max frontier vertices handled by one CTA (one per thread)
+constexpr int kTailE = 16384;        // max frontier arcs handled by one CTA
+constexpr int kTailCollect = 512;    // max log entries gathered when entering tail mode
+
+struct TailSmem {
+  int f[2][kTailV];                  // frontier (ping-pong)
+  long long b[2][kTailV];            // row start of each frontier vertex
+  int d[2][kTailV];                  // its out-degree
+  int pre[kTailV + 1];
+  int buf[kTailCollect];
+  int wsum[kWarps];
+  int nnext;
+  unsigned long long anext;
+};
+
+// exclusive block scan of x (one value per thread, 256 threads); returns the total
+__device__ __forceinline__ int block_scan_excl(int x, int *out_excl, int *wsum) {
+  const int lane = (int)lane_id(), warp = threadIdx.x >> 5;
+  int inc = x;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(FULL, inc, o);
+    if (lane >= o) inc += y;
+  }
+  if (lane == 31) wsum[warp] = inc;
+  __syncthreads();
+  int base = 0, total = 0;
+  for (int w = 0; w < kWarps; ++w) {
+    if (w < warp) base += wsum[w];
+    total += wsum[w];
+  }
+  *out_excl = base + inc - x;
+  __syncthreads();
+  return total;
+}
+
+// Block 0 only.  Runs levels Lstart, Lstart+1, ... while the frontier is small.
+__device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
+  Ctl *ctl = a.ctl;
+  const int tid = threadIdx.x, lane = (int)lane_id(), warp = tid >> 5;
+  int nf = 0;
+  // ---- gather the frontier of level Lstart from its log and deduplicate
+  {
+    const CounterSet *cs = &ctl->set[Lstart % 3];
+    const Queues &Q = a.q[Lstart & 1];
+    int E = 0;
+    for (int c = 0; c <= a.L.ncls; ++c) {
+      const int cnt = (int)ldcg(&cs->cnt[c].v);
+      for (int i = tid; i < cnt; i += blockDim.x)
+        ts.buf[E + i] = c == 0 ? ldcg_tile(Q.cta + i).u : (c == a.L.ncls ? ldcg(Q.frag + i) : ldcg(Q.cls[c] + i));
+      E += cnt;
+    }
+    int P = 1;
+    while (P < E) P <<= 1;
+    for (int i = E + tid; i < P; i += blockDim.x) ts.buf[i] = 0x7fffffff;
+    __syncthreads();
+    for (int k = 2; k <= P; k <<= 1)
+      for (int j = k >> 1; j > 0; j >>= 1) {
+        for (int i = tid; i < P; i += blockDim.x) {
+          const int l = i ^ j;
+          if (l > i) {
+            const int x = ts.buf[i], y = ts.buf[l];
+            if ((x > y) == ((i & k) == 0)) {
+              ts.buf[i] = y;
+              ts.buf[l] = x;
+            }
+          }
+        }
+        __syncthreads();
+      }
+    for (int base = 0; base < E; base += blockDim.x) {
+      const int i = base + tid;
+      const bool keep = i < E && (i == 0 || ts.buf[i] != ts.buf[i - 1]);
+      int pos;
+      const int tot = block_scan_excl(keep ? 1 : 0, &pos, ts.wsum);
+      if (keep) {
+        const int u = ts.buf[i];
+        const long long rb = a.off[u];
+        ts.f[0][nf + pos] = u;
+        ts.b[0][nf + pos] = rb;
+        ts.d[0][nf + pos] = (int)(a.off[u + 1] - rb);
+      }
+      nf += tot;
+    }
+    __syncthreads();
+  }
+  // statistics kept in registers of thread 0, written once
+  unsigned long long s_exp = 0, s_arcs = 0, s_disc = 0, s_reach = 0;
+  int cur = 0;
+  int L = Lstart;
+  for (;; ++L) {
+    // exclusive scan of the frontier's degrees (nf <= kTailV = blockDim: one row per thread)
+    int p1;
+    const int A = block_scan_excl(tid < nf ? ts.d[cur][tid] : 0, &p1, ts.wsum);
+    if (tid < nf) ts.pre[tid] = p1;
+    if (tid == 0) {
+      ts.pre[nf] = A;
+      ts.nnext = 0;
+      ts.anext = 0;
+    }
+    __syncthreads();
+    const int nx = cur ^ 1;
+    for (int k = tid; k < A; k += blockDim.x) {
+      int lo = 0, hi = nf - 1;      // largest o with pre[o] <= k
+      while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (ts.pre[mid] <= k) lo = mid; else hi = mid - 1;
+      }
+      const int v = a.col[ts.b[cur][lo] + (k - ts.pre[lo])];
+      const uint32_t bit = 1u << (v & 31);
+      if (!(atomicOr(a.visited + (v >> 5), bit) & bit)) {
+        a.level[v] = L + 1;
+        if (a.parent) a.parent[v] = ts.f[cur][lo];
+        const int idx = atomicAdd(&ts.nnext, 1);
+        a.tail[idx] = v;
+        const long long rb = a.off[v];
+        const int dg = (int)(a.off[v + 1] - rb);
+        if (idx < kTailV) {
+          ts.f[nx][idx] = v;
+          ts.b[nx][idx] = rb;
+          ts.d[nx][idx] = dg;
+        }
+        atomicAdd(&ts.anext, (unsigned long long)dg);
+      }
+    }
+    __syncthreads();
+    const int nn = ts.nnext;
+    const unsigned long long an = ts.anext;
+    if (tid == 0) {
+      s_exp += nf;
+      s_arcs += A;
+      s_disc += nn;
+      s_reach += an;
+      if (L < kMaxRec) {
+        LevelRec &r = ctl->rec[L];
+        r.dir = 0;
+        r.nF = nf;
+        r.arcsF = A;
+        r.inspected = A;
+        r.scanned = 0;
+        r.discovered = nn;
+        r.t_ns = r.t_work = globaltimer();
+      }
+    }
+    const bool fits = nn <= kTailV && an <= (unsigned long long)kTailE;
+    if (nn == 0 || L + 1 >= a.max_levels || !fits) break;
+    nf = nn;
+    cur = nx;
+    __syncthreads();
+  }
+  const int nn = ts.nnext;
+  if (tid == 0) {
+    ctl->tot_push_expanded += s_exp;
+    ctl->tot_push_arcs += s_arcs;
+    ctl->tot_push_disc += s_disc;
+    ctl->tot_arcs_reached += s_reach;
+    ctl->tot_improved += s_disc;
+    ctl->push_levels += L - Lstart + 1;
+    ctl->levels = L + 1;
+    ctl->tail_levels += L - Lstart + 1;
+    if (nn == 0) {
+      ctl->tail_state = 1;
+    } else if (L + 1 >= a.max_levels) {
+      ctl->status = 1;
+      ctl->tail_state = 1;
+    }
+  }
+  if (nn == 0 || L + 1 >= a.max_levels) return;
+  // the frontier grew: classify it into level L+1's log and hand back to the grid
+  constexpr int nctr = sizeof(CounterSet) / sizeof(PaddedCounter);
+  if (tid < nctr) {
+    reinterpret_cast<PaddedCounter *>(&ctl->set[(L + 1) % 3])[tid].v = 0ull;
+    reinterpret_cast<PaddedCounter *>(&ctl->set[(L + 2) % 3])[tid].v = 0ull;
+  }
+  __threadfence_block();
+  __syncthreads();
+  for (int base = warp * 32; base < nn; base += blockDim.x) {
+    const int i = base + lane;
+    const bool act = i < nn;
+    enqueue_ids(act, act ? ldcg(a.tail + i) : 0, a.off, a.L, a.q[(L + 1) & 1], &ctl->set[(L + 1) % 3]);
+  }
+  if (tid == 0) {
+    ctl->tail_state = 2;
+    ctl->tail_resume = L + 1;
+  }
+}
+
 // ============================================================================ BFS kernel
 template <int VEC>
 __global__ void __launch_bounds__(kBlock, 4) k_bfs(const __grid_constant__ TravArgs a) {
   __shared__ WarpScratch wsm[kWarps];
   __shared__ BfsPush::Src fsrc[kWarps][32];
+  __shared__ TailSmem tsm;
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
   double mU = (double)a.m - (double)ldcg(&ctl->set[0].arcsF.v);
@@ -287,6 +485,23 @@ __global__ void __launch_bounds__(kBlock, 4) k_bfs(const __grid_constant__ TravA
     if (L + 1 >= a.max_levels) {
       if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = 1;
       break;
+    }
+    // small frontier on a push-only traversal: block 0 runs the next levels alone
+    if (!a.do_enabled && nF <= kTailV && aF <= (unsigned long long)kTailE) {
+      unsigned long long ents = 0;
+      for (int c = 0; c <= a.L.ncls; ++c) ents += ldcg(&nxt->cnt[c].v);
+      if (ents <= (unsigned long long)kTailCollect) {
+        if (blockIdx.x == 0) {
+          __syncthreads();
+          if (threadIdx.x == 0) ctl->tail_state = 0;
+          __syncthreads();
+          tail_run(a, L + 1, tsm);
+        }
+        grid_barrier(&ctl->bar);
+        if (ldcg(&ctl->tail_state) == 1) break;
+        L = ldcg(&ctl->tail_resume) - 1;   // ++L resumes the grid at the returned level
+        continue;
+      }
     }
     mU -= (double)aF;
     if (a.do_enabled) {
@@ -950,6 +1165,7 @@ static TravArgs make_args(sage_graph *g) {
   a.alpha = g->alpha;
   a.beta = g->beta;
   a.max_levels = (int)std::min<long long>(g->n + 1, 0x7fffffffll);
+  a.tail = (int *)g->ts.tmp_out;
   a.vec_ok = g->vec_ok ? 1 : 0;
   return a;
 }

@@ -12,17 +12,24 @@ import sagegen as sg  # noqa: E402
 
 p = argparse.ArgumentParser()
 p.add_argument("--scale", type=int, default=24)
+p.add_argument("--graph", default="rmat", choices=["rmat", "uk", "twitter"])
+p.add_argument("--n", type=int, default=0, help="vertices for uk / twitter shapes")
 p.add_argument("--op", default="bfs_push", choices=["bfs_push", "bfs_do", "sssp", "pr"])
 p.add_argument("--reps", type=int, default=3)
 p.add_argument("--tile-cta", type=int, default=256)
 p.add_argument("--align", type=int, default=4)
 p.add_argument("--binned", action="store_true", help="experimental two-phase binned push level")
 a = p.parse_args()
-g = sg.rmat(a.scale, 16, 1, True)
+if a.graph == "rmat":
+    g = sg.rmat(a.scale, 16, 1, True)
+elif a.graph == "uk":
+    g = sg.uk_like(n=a.n or 10_000_000, seed=1, n_tendrils=200)
+else:
+    g = sg.twitter_like(n=a.n or 4_000_000, tuples=(a.n or 4_000_000) * 36, seed=1)
 w = sg.weights(g, 1)
 s = stream = torch.cuda.current_stream()
 G = sage.load_csr(torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda(), torch.from_numpy(w).cuda(),
-                  symmetric=True, borrow=True, stream=stream.cuda_stream, tile_cta=a.tile_cta, align=a.align)
+                  symmetric=g.symmetric, borrow=True, stream=stream.cuda_stream, tile_cta=a.tile_cta, align=a.align)
 src = sg.sources(g, a.reps, seed=2)
 lv = torch.empty(g.n, dtype=torch.int32, device="cuda")
 for i in range(a.reps):
@@ -36,7 +43,12 @@ for i in range(a.reps):
         x = torch.empty(g.n, dtype=torch.float64, device="cuda")
         _, st = G.pagerank(0.85, 5, out=x)
     print(a.op, i, {k: st[k] for k in ("levels", "kernel_ms", "ms", "edges_traversed", "model_bytes")}, flush=True)
-    if a.op != "pr":
+    if a.op != "pr" and os.environ.get("LEVELS", "1") == "0":
+        rec = G.level_records()
+        dt = np.diff(np.concatenate([[0], rec[:, 6]])) / 1e3
+        small = dt[rec[:, 2] < 10000]
+        print("   levels=%d  median small-level us=%.1f  total small-level ms=%.2f" % (len(rec), np.median(small) if len(small) else 0, small.sum() / 1e3))
+    if a.op != "pr" and os.environ.get("LEVELS", "1") == "1":
         prev = 0
         for r in G.level_records():
             print("   L dir=%d |F|=%9d arcsF=%11d insp=%11d disc=%9d  %8.1f us (work done at +%8.1f, phase1 +%8.1f)" % (

@@ -54,10 +54,12 @@ enum {
   SAGE_F_NO_VALIDATE = 8u, /* skip the validation pass of sage_load_csr                              */
   SAGE_F_PUSH_ONLY = 16u,  /* disable direction switching: every level is the paper's push
                               expansion (Alg. 2/3).  Can also be set per call (sage_bfs_ex).     */
-  SAGE_F_BINNED = 32u      /* per call (sage_bfs_ex), experimental: two-phase push levels (neighbour
+  SAGE_F_BINNED = 32u,     /* per call (sage_bfs_ex), experimental: two-phase push levels (neighbour
                               ids binned by vertex slice, then filtered against shared-memory
                               slices of the visited bitmap).  Results identical;
                               slower than the default direct filter on B200 as measured.        */
+  SAGE_F_NO_STEALING = 64u /* per call (sage_bfs_ex), ablation (Fig. 10): tiles are dealt to
+                              warps statically instead of through Resident Tile Stealing        */
 };
 
 /* Multi-GPU description (1D vertex partition).  NULL in sage_csr = single GPU.

@@ -19,7 +19,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, os.environ.get("SAGE_LIB", "libsage.so"))
 
 OK, E_INVALID, E_NOMEM, E_CUDA, E_NCCL, E_OVERFLOW, E_UNSUPPORTED = range(7)
-F_SYMMETRIC, F_DEVICE_PTRS, F_BORROW, F_NO_VALIDATE, F_PUSH_ONLY, F_BINNED = 1, 2, 4, 8, 16, 32
+F_SYMMETRIC, F_DEVICE_PTRS, F_BORROW, F_NO_VALIDATE, F_PUSH_ONLY, F_BINNED, F_NO_STEALING = 1, 2, 4, 8, 16, 32, 64
 STATUS_NAMES = {0: "SAGE_OK", 1: "SAGE_E_INVALID", 2: "SAGE_E_NOMEM", 3: "SAGE_E_CUDA",
                 4: "SAGE_E_NCCL", 5: "SAGE_E_OVERFLOW", 6: "SAGE_E_UNSUPPORTED"}
 
@@ -192,14 +192,14 @@ class Graph:
 
     # ------------------------------------------------------------------ queries
     def bfs(self, source: int, out=None, parent_out=None, parents: bool = False, push_only: bool = False,
-            binning: bool = False):
+            binning: bool = False, stealing: bool = True):
         """sage_bfs_ex -> (level int32[n_local], parent or None, stats dict)."""
         o = _out(out, self.n_local, np.int32)
         po = None
         if parents or parent_out is not None:
             po = _out(parent_out, self.n_local, np.int32)
         st = Stats()
-        fl = (F_PUSH_ONLY if push_only else 0) | (F_BINNED if binning else 0)
+        fl = (F_PUSH_ONLY if push_only else 0) | (F_BINNED if binning else 0) | (0 if stealing else F_NO_STEALING)
         _check(lib().sage_bfs_ex(self._h, int(source), o.ptr, po.ptr if po else None, fl, ctypes.byref(st)))
         return o.obj, (po.obj if po else None), st.as_dict()
 

@@ -428,12 +428,14 @@ __device__ __forceinline__ void buffer_flush(WarpScratch *ws, int &cnt,
 //                              lpt = lanes sharing the tile (aligned groups of the warp)
 //   kWeights (load weights), kNeedRow (src needs the row for CTA tiles), kEnqueue (contraction)
 //   Queues *next_q; CounterSet *next_cs;             where filtered-in vertices go
+// steal = false (ablation of Resident Tile Stealing, Fig. 10): tiles are dealt to warps
+// statically, round robin in batch units, instead of through the device-wide tickets.
 template <int VEC, class F>
 __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Queues &Q,
                                             CounterSet *cs, const long long *__restrict__ off,
                                             const int *__restrict__ col,
                                             const uint32_t *__restrict__ w, WarpScratch *ws,
-                                            typename F::Src *fsrc, bool vec_ok) {
+                                            typename F::Src *fsrc, bool vec_ok, bool steal = true) {
   const unsigned lane = lane_id();
   const unsigned long long pol = policy_evict_first();
   const long long gwarp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -458,11 +460,15 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
     if ((unsigned long long)gwarp >= grabs) continue;
     const int sub = lane / lpt, sl = lane % lpt;
     const bool contiguous = lpt < 32 && vec_ok && VEC == 4;
-    for (;;) {
+    for (unsigned long long rr = 0;; ++rr) {
       PROF_T(tt0);
       unsigned long long base = 0;
-      if (lane == 0) base = atomicAdd(&cs->tk[c].v, batch);
-      base = shfl64(base, 0);
+      if (steal) {
+        if (lane == 0) base = atomicAdd(&cs->tk[c].v, batch);
+        base = shfl64(base, 0);
+      } else {
+        base = ((unsigned long long)gwarp + rr * (unsigned long long)nwarps) * batch;
+      }
       PROF_T(tt1);
       PROF_ADD(5, tt1 - tt0);
       PROF_ADD(6, 1);
@@ -543,11 +549,16 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
   // ---- fragments: warp scan-based gather
   const unsigned long long fcount = shfl64(my_cnt, L.ncls);
   const unsigned long long fgrabs = (fcount + 31) / 32;
+  unsigned long long frr = 0;
   for (;;) {
     if (fcount == 0 || (unsigned long long)gwarp >= fgrabs) break;
     unsigned long long base = 0;
-    if (lane == 0) base = atomicAdd(&cs->tk[L.ncls].v, 32ull);
-    base = shfl64(base, 0);
+    if (steal) {
+      if (lane == 0) base = atomicAdd(&cs->tk[L.ncls].v, 32ull);
+      base = shfl64(base, 0);
+    } else {
+      base = ((unsigned long long)gwarp + frr++ * (unsigned long long)nwarps) * 32ull;
+    }
     if (base >= fcount) break;
     const bool valid = base + lane < fcount;
     int u = 0, hl = 0, tl = 0;

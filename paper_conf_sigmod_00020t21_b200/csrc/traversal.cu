@@ -147,6 +147,7 @@ struct TravArgs {
   double alpha, beta;
   int max_levels;
   int *tail;            // tail mode: next-frontier list (n entries of scratch)
+  int steal;            // 0 = ablation: static tile assignment instead of stealing
 };
 
 // Pull (bottom-up) step over the visited bitmap: one warp per 32-vertex word.
@@ -444,7 +445,10 @@ __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
 
 // ============================================================================ BFS kernel
 template <int VEC>
-__global__ void __launch_bounds__(kBlock, 4) k_bfs(const __grid_constant__ TravArgs a) {
+#ifndef SAGE_BFS_MINB
+#define SAGE_BFS_MINB 4
+#endif
+__global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_constant__ TravArgs a) {
   __shared__ WarpScratch wsm[kWarps];
   __shared__ BfsPush::Src fsrc[kWarps][32];
   __shared__ TailSmem tsm;
@@ -472,7 +476,8 @@ __global__ void __launch_bounds__(kBlock, 4) k_bfs(const __grid_constant__ TravA
       f.v_base = 0;
       f.next_q = &a.q[(L + 1) & 1];
       f.next_cs = nxt;
-      consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok);
+      consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok,
+                       a.steal != 0);
     } else {
       pull_level(a, L + 1, fbc, fbn, a.q[(L + 1) & 1], cur, nxt, &wsm[warp]);
     }
@@ -558,6 +563,7 @@ struct BinPush {
   int *rpos, *rend;                  // this warp's reserved bin range per slice
   int fillset;
   int next_level;
+  int nbits;                         // bits of a slice id
   const Queues *qn;
   CounterSet *csn;
   __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
@@ -609,33 +615,40 @@ struct BinPush {
     }
   }
 
+  // Warp multi-split of 32 ids into their slices: lanes of one slice are found with one ballot per
+  // slice-id bit (no match.any), ranked with popc, staged in this warp's smem rows (stride
+  // kBinE + 1 against bank conflicts); a full row is flushed to HBM in one coalesced store.
   __device__ __forceinline__ void append(bool valid, int v) const {
-    if (!__any_sync(FULL, valid)) return;
     const unsigned lane = lane_id();
-    const int sl = valid ? (v >> b->slice_lg) : -1;
-    const unsigned grp = __match_any_sync(FULL, sl);
-    const int leader = __ffs(grp) - 1;
+    const int sl = valid ? (v >> b->slice_lg) : 0;
+    unsigned grp = __ballot_sync(FULL, valid);
+    if (!grp) return;
+    for (int bit = 0; bit < nbits; ++bit) {
+      const bool on = (sl >> bit) & 1;
+      const unsigned bb = __ballot_sync(FULL, on);
+      grp &= on ? bb : ~bb;
+    }
     const int c0 = valid ? cnt[sl] : 0;
-    __syncwarp();
     const int idx = c0 + __popc(grp & lanemask_lt());
-    if (valid && idx < kBinE) stage[sl * kBinE + idx] = v;
     const int tot = c0 + __popc(grp);
-    if (valid && (int)lane == leader && tot < kBinE) cnt[sl] = tot;
+    const bool leader = valid && (grp & lanemask_lt()) == 0;
+    if (valid && idx < kBinE) stage[sl * (kBinE + 1) + idx] = v;
     __syncwarp();
-    unsigned fm = __ballot_sync(FULL, valid && (int)lane == leader && tot >= kBinE);
+    if (leader) cnt[sl] = tot < kBinE ? tot : tot - kBinE;
+    unsigned fm = __ballot_sync(FULL, leader && tot >= kBinE);
     while (fm) {
       const int ld = __ffs(fm) - 1;
       fm &= fm - 1;
       const int s2 = __shfl_sync(FULL, sl, ld);
       const unsigned g2 = __shfl_sync(FULL, grp, ld);
       const int c2 = __shfl_sync(FULL, c0, ld);
-      emit(s2, kBinE, stage + s2 * kBinE);
       __syncwarp();
+      emit(s2, kBinE, stage + s2 * (kBinE + 1));
+      // the group's overflow (positions >= kBinE) restarts the row
       if ((g2 >> lane) & 1u) {
         const int id2 = c2 + __popc(g2 & lanemask_lt());
-        if (id2 >= kBinE) stage[s2 * kBinE + id2 - kBinE] = v;
+        if (id2 >= kBinE) stage[s2 * (kBinE + 1) + id2 - kBinE] = v;
       }
-      if ((int)lane == ld) cnt[s2] = c2 + __popc(g2) - kBinE;
       __syncwarp();
     }
   }
@@ -675,25 +688,32 @@ __device__ __forceinline__ void bin_check(const TravArgs &a, const BinArgs &b, i
     const long long tot = fill < b.cap ? fill : b.cap;
     const long long lo = tot * part / nparts, hi = tot * (part + 1) / nparts;
     const int *bin = b.bins + (long long)s * b.cap;
-    for (long long base = lo + (long long)warp * 32; base < hi; base += (long long)nw * 32) {
-      const long long i = base + lane;
-      bool disc = false;
-      int v = 0;
-      if (i < hi) v = ldcg(bin + i);
-      if (i < hi && v >= 0) {
-        const int lb = (int)(v - v0);
-        const uint32_t bit = 1u << (lb & 31);
-        if (!(sbm[lb >> 5] & bit)) {
-          if (!(atomicOr(sbm + (lb >> 5), bit) & bit)) {
-            disc = !(atomicOr(a.visited + (v >> 5), bit) & bit);
-            if (disc) {
-              a.level[v] = L + 1;
-              if (fbn) atomicOr(fbn + (v >> 5), bit);
+    for (long long base = lo + (long long)warp * 128; base < hi; base += (long long)nw * 128) {
+      int vv[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const long long i = base + j * 32 + lane;
+        vv[j] = i < hi ? ldcg(bin + i) : -1;
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int v = vv[j];
+        bool disc = false;
+        if (v >= 0) {
+          const int lb = (int)(v - v0);
+          const uint32_t bit = 1u << (lb & 31);
+          if (!(sbm[lb >> 5] & bit)) {
+            if (!(atomicOr(sbm + (lb >> 5), bit) & bit)) {
+              disc = !(atomicOr(a.visited + (v >> 5), bit) & bit);
+              if (disc) {
+                a.level[v] = L + 1;
+                if (fbn) atomicOr(fbn + (v >> 5), bit);
+              }
             }
           }
         }
+        buffer_push(disc, v, &ws[warp], bcnt, a.off, a.L, Qn, csn);
       }
-      buffer_push(disc, v, &ws[warp], bcnt, a.off, a.L, Qn, csn);
     }
     __syncthreads();
   }
@@ -729,7 +749,7 @@ __global__ void __launch_bounds__(kBinBlock, 1) k_bfs_bin(const __grid_constant_
     if (dir == 0) {
       // phase 1: expansion into slice bins
       int *cnt = cnts + warp * kMaxSlices;
-      int *stage = reinterpret_cast<int *>(U) + warp * b.nslices * kBinE;
+      int *stage = reinterpret_cast<int *>(U) + warp * b.nslices * (kBinE + 1);
       for (int i = lane; i < b.nslices; i += 32) {
         cnt[i] = 0;
         rps[warp * kMaxSlices + i] = 0;
@@ -745,12 +765,14 @@ __global__ void __launch_bounds__(kBinBlock, 1) k_bfs_bin(const __grid_constant_
       f.rend = res + warp * kMaxSlices;
       f.fillset = L & 1;
       f.next_level = L + 1;
+      f.nbits = 0;
+      while ((1 << f.nbits) < b.nslices) ++f.nbits;
       f.qn = &a.q[(L + 1) & 1];
       f.csn = nxt;
       consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc + warp * 32, a.vec_ok);
       for (int sl = 0; sl < b.nslices; ++sl) {
         const int c = cnt[sl];
-        if (c) f.emit(sl, c, stage + sl * kBinE);
+        if (c) f.emit(sl, c, stage + sl * (kBinE + 1));
       }
       f.close_reservations();
       grid_barrier(&ctl->bar);
@@ -786,7 +808,7 @@ __global__ void __launch_bounds__(kBinBlock, 1) k_bfs_bin(const __grid_constant_
 static size_t bin_smem_bytes(int nslices, long long n) {
   const size_t fixed = sizeof(WarpScratch) * kBinWarps + sizeof(int) * 32 * kBinWarps +
                        3 * sizeof(int) * kMaxSlices * kBinWarps;
-  const size_t stage = sizeof(int) * (size_t)kBinWarps * nslices * kBinE;
+  const size_t stage = sizeof(int) * (size_t)kBinWarps * nslices * (kBinE + 1);
   const long long sw = std::min<long long>(n, 1ll << kSliceLg);
   const size_t bm = sizeof(uint32_t) * (size_t)((sw + 31) / 32 + 1);
   return fixed + std::max(stage, bm);
@@ -1166,6 +1188,7 @@ static TravArgs make_args(sage_graph *g) {
   a.beta = g->beta;
   a.max_levels = (int)std::min<long long>(g->n + 1, 0x7fffffffll);
   a.tail = (int *)g->ts.tmp_out;
+  a.steal = 1;
   a.vec_ok = g->vec_ok ? 1 : 0;
   return a;
 }
@@ -1255,6 +1278,7 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   TravArgs a = make_args(g);
   a.parent = parent_out ? t.parent : nullptr;
   a.do_enabled = (symmetric && !push_only) ? 1 : 0;
+  a.steal = (call_flags & SAGE_F_NO_STEALING) ? 0 : 1;
   k_seed<<<1, 32, 0, g->stream>>>(a, src, 0);
   const int nslices = (int)((g->n + (1ll << kSliceLg) - 1) >> kSliceLg);
   const bool binned = !parent_out && (call_flags & SAGE_F_BINNED) && nslices <= kMaxSlices;

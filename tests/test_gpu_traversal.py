@@ -300,3 +300,17 @@ def test_binned_push_bin_overflow(sage):
             ref = oracle.bfs(g.off, g.col, s)
             lv, _, _ = G.bfs(s, push_only=True, binning=True)
             assert np.array_equal(lv, ref)
+
+
+def test_no_stealing_ablation_parity(sage):
+    """SAGE_F_NO_STEALING (static tile assignment, the Fig. 10 ablation) gives the same levels."""
+    for g in [sg.rmat(14, 16, seed=31, symmetric=True), sg.rmat(13, 16, seed=32, symmetric=False)]:
+        with sage.load_csr(g.off, g.col, symmetric=g.symmetric) as G:
+            for s in sg.sources(g, 3, seed=2):
+                ref = oracle.bfs(g.off, g.col, int(s))
+                lv, _, _ = G.bfs(int(s), push_only=True, stealing=False)
+                assert np.array_equal(lv, ref)
+    g = sg.rmat(13, 16, seed=33, symmetric=True)
+    with sage.load_csr(g.off, g.col, symmetric=True, tile_cta=4096, tile_min=4096, align=0) as G:
+        s = int(sg.sources(g, 1, seed=2)[0])
+        assert np.array_equal(G.bfs(s, push_only=True)[0], oracle.bfs(g.off, g.col, s))

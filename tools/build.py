@@ -81,7 +81,9 @@ def build_sage(force=False, verbose=False):
     os.makedirs(objdir, exist_ok=True)
     common = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC",
               "-I", os.path.join(ROOT, "include"), "-I", csrc, "-I", nccl_inc,
-              "--expt-relaxed-constexpr", "-Xptxas", "-v" if verbose else "-O3"] + (["-DSAGE_PROF=1"] if prof else [])
+              "--expt-relaxed-constexpr", "-Xptxas", "-v" if verbose else "-O3"] + (["-DSAGE_PROF=1"] if prof else []) + \
+             [f"-D{k}={v}" for k, v in os.environ.items() if k.startswith("SAGE_DEF_")
+              for k in [k[len("SAGE_DEF_"):]]]
     objs = []
     for cu in cus:
         obj = os.path.join(objdir, os.path.basename(cu)[:-3] + ".o")

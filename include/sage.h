@@ -166,6 +166,15 @@ sage_status sage_pagerank(sage_graph *g, double damping, int32_t iterations, dou
 sage_status sage_pagerank_ex(sage_graph *g, double damping, int32_t iterations, double *rank_out,
                              uint32_t call_flags, sage_stats *st);
 
+/* Betweenness Centrality contributions (Alg. 1 l.8-24): for
+ * every source s in `sources` (host array, original ids) a forward push BFS counting shortest
+ * paths (sigma, fp64) and a backward dependency accumulation by decreasing level (delta, fp64);
+ * bc_out[v] = sum over the sources of delta_s(v), v != s (Brandes; no normalisation — an
+ * undirected graph counts every pair in both directions).  At most 4096 levels per source.
+ * Single GPU.                                                                                  */
+sage_status sage_bc(sage_graph *g, const int32_t *sources, int64_t n_sources, double *bc_out,
+                    sage_stats *st);
+
 /* `rounds` rounds of Sampling-based Reordering (§6; readings R17-R25): relabels the
  * vertices in place (the CSR is rewritten, rows sorted, weights moved with their arcs) and
  * composes the permutation; later queries still speak original ids.  Single GPU only.         */

@@ -35,6 +35,7 @@ def _lib():
         lib.ora_check_sssp.argtypes = [i64, p, p, p, i32, p]
         lib.ora_pagerank.argtypes = [i64, p, p, dbl, i32, p]
         lib.ora_pagerank_step.argtypes = [i64, p, p, dbl, p, p]
+        lib.ora_bc.argtypes = [i64, p, p, p, i64, p]
         lib.ora_tiles_row.argtypes = [i64, i64, i32, i32, i32, p]
         lib.ora_tiles_row.restype = i64
         lib.ora_tile_log.argtypes = [p, p, i64, i32, i32, i32, p]
@@ -118,6 +119,19 @@ def pagerank_step(off, col, x, damping: float = 0.85) -> np.ndarray:
     out = np.empty(n, dtype=np.float64)
     if _lib().ora_pagerank_step(n, po, pc, float(damping), px, out.ctypes.data) != 0:
         raise ValueError("empty graph")
+    return out
+
+
+# ---------------------------------------------------------------- BC (Alg. 1 l.8-24, NEXT #1)
+def bc(off, col, sources) -> np.ndarray:
+    """sum over s in ``sources`` of the Brandes dependencies delta_s(v) (v != s), fp64."""
+    off, po = _c(off, np.int64)
+    col, pc = _c(col, np.int32)
+    src, ps = _c(np.atleast_1d(sources), np.int32)
+    n = len(off) - 1
+    out = np.empty(n, dtype=np.float64)
+    if _lib().ora_bc(n, po, pc, ps, len(src), out.ctypes.data) != 0:
+        raise ValueError("bad source")
     return out
 
 

@@ -219,6 +219,51 @@ int ora_pagerank_step(int64_t n, const int64_t *off, const int32_t *col, double 
 }
 
 /* ===================================================================================== */
+/* BC — Alg. 1 l.8-24: forward BFS that counts shortest paths
+ * (l.8-17: dist[nb] := dist[fr]+1 on first visit; sigma[nb] += sigma[fr] when dist[nb] =
+ * dist[fr]+1) and backward dependency accumulation by decreasing level (l.19-24: delta[fr] +=
+ * sigma[fr]/sigma[nb] * (delta[nb] + 1) for every arc fr->nb with dist[nb] = dist[fr]+1).
+ * This is Brandes' algorithm; the oracle writes it out plainly (FIFO BFS, then the BFS order
+ * reversed).  sigma and delta are fp64.  For every source s in `sources`, bc[v] += delta_s(v)
+ * for v != s (delta_s(s) is not added).  Unreachable vertices get 0.                          */
+int ora_bc(int64_t n, const int64_t *off, const int32_t *col, const int32_t *sources, int64_t ns,
+           double *bc) {
+  int32_t *dist = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+  int32_t *order = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+  double *sigma = (double *)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
+  double *delta = (double *)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
+  if (!dist || !order || !sigma || !delta) { free(dist); free(order); free(sigma); free(delta); return 2; }
+  for (int64_t v = 0; v < n; ++v) bc[v] = 0.0;
+  for (int64_t k = 0; k < ns; ++k) {
+    const int32_t s = sources[k];
+    if (s < 0 || s >= n) { free(dist); free(order); free(sigma); free(delta); return 1; }
+    for (int64_t v = 0; v < n; ++v) { dist[v] = -1; sigma[v] = 0.0; delta[v] = 0.0; }
+    int64_t head = 0, tail = 0;
+    dist[s] = 0;
+    sigma[s] = 1.0;
+    order[tail++] = s;
+    while (head < tail) {                         /* forward: Alg. 1 l.8-17 */
+      const int32_t u = order[head++];
+      for (int64_t e = off[u]; e < off[u + 1]; ++e) {
+        const int32_t v = col[e];
+        if (dist[v] == -1) { dist[v] = dist[u] + 1; order[tail++] = v; }
+        if (dist[v] == dist[u] + 1) sigma[v] += sigma[u];
+      }
+    }
+    for (int64_t i = tail - 1; i >= 0; --i) {     /* backward: Alg. 1 l.19-24 */
+      const int32_t u = order[i];
+      for (int64_t e = off[u]; e < off[u + 1]; ++e) {
+        const int32_t v = col[e];
+        if (dist[v] == dist[u] + 1) delta[u] += sigma[u] / sigma[v] * (delta[v] + 1.0);
+      }
+      if (u != s) bc[u] += delta[u];
+    }
+  }
+  free(dist); free(order); free(sigma); free(delta);
+  return 0;
+}
+
+/* ===================================================================================== */
 /* c4. Tiled Partitioning of one row [b, e) — Alg. 2 as the resident tile log of
  * Alg. 3 l.2-7.  The block-sized tile consumes full tile-size chunks of the row
  * (Alg. 2 l.9-25; the leader keeps neighbor_size mod tile.size() at the row END, l.14-16),

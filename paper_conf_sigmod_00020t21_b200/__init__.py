@@ -24,7 +24,7 @@ STATUS_NAMES = {0: "SAGE_OK", 1: "SAGE_E_INVALID", 2: "SAGE_E_NOMEM", 3: "SAGE_E
                 4: "SAGE_E_NCCL", 5: "SAGE_E_OVERFLOW", 6: "SAGE_E_UNSUPPORTED"}
 
 EXPORTED = ["sage_load_csr", "sage_free", "sage_bfs", "sage_bfs_ex", "sage_sssp", "sage_pagerank",
-            "sage_pagerank_ex",
+            "sage_pagerank_ex", "sage_bc",
             "sage_reorder", "sage_reorder_objective", "sage_get_permutation", "sage_get_csr", "sage_graph_info",
             "sage_debug_export_tiles", "sage_debug_reorder_stages", "sage_nccl_unique_id", "sage_debug_level_records", "sage_last_error", "sage_version"]
 
@@ -86,6 +86,7 @@ def lib():
         L.sage_sssp.argtypes = [p, i32, p, ctypes.POINTER(Stats)]
         L.sage_pagerank.argtypes = [p, dbl, i32, p, ctypes.POINTER(Stats)]
         L.sage_pagerank_ex.argtypes = [p, dbl, i32, p, u32, ctypes.POINTER(Stats)]
+        L.sage_bc.argtypes = [p, p, i64, p, ctypes.POINTER(Stats)]
         L.sage_reorder.argtypes = [p, i32, ctypes.POINTER(ReorderOpts), ctypes.POINTER(Stats)]
         L.sage_get_permutation.argtypes = [p, p]
         L.sage_reorder_objective.argtypes = [p, i32, p]
@@ -215,6 +216,14 @@ class Graph:
         st = Stats()
         _check(lib().sage_pagerank_ex(self._h, float(damping), int(iterations), o.ptr,
                                       F_PUSH_ONLY if push_only else 0, ctypes.byref(st)))
+        return o.obj, st.as_dict()
+
+    def bc(self, sources, out=None):
+        """sage_bc: sum over ``sources`` of the Brandes dependencies (fp64)."""
+        src = np.ascontiguousarray(np.atleast_1d(sources), dtype=np.int32)
+        o = _out(out, self.n_local, np.float64)
+        st = Stats()
+        _check(lib().sage_bc(self._h, src.ctypes.data, len(src), o.ptr, ctypes.byref(st)))
         return o.obj, st.as_dict()
 
     def reorder(self, rounds: int = 1, sector_width: int = 8, candidates=None):

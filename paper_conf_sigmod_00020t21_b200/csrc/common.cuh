@@ -46,6 +46,8 @@ struct Queues {        // one resident tile log (one level's, or the all-V log o
   CtaTile *cta;        // class 0
   int *cls[kMaxCls];   // cls[c], 1 <= c < ncls
   int *frag;           // fragment queue (vertex ids)
+  int *order;          // optional: every enqueued vertex is also appended here (BC's BFS order)
+  unsigned long long *order_cnt;
 };
 
 // One counter per 128-B line: every warp of the grid hits these with atomics, and counters that
@@ -308,10 +310,16 @@ __device__ __forceinline__ void enqueue_warp(bool active, int v, long long b, lo
     if (totq) mybase = atomicAdd(&cs->cnt[0].v, totq);
   } else if ((int)lane <= L.ncls) {
     if (mine_mask) mybase = atomicAdd(&cs->cnt[lane].v, (unsigned long long)__popc(mine_mask));
+  } else if (lane == 29) {
+    if (Q.order) mybase = atomicAdd(Q.order_cnt, (unsigned long long)__popc(am));
   } else if (lane == 30) {
     atomicAdd(&cs->nF.v, (unsigned long long)__popc(am));
   } else if (lane == 31) {
     if (deg) atomicAdd(&cs->arcsF.v, deg);
+  }
+  if (Q.order) {
+    const unsigned long long ob = shfl64(mybase, 29);
+    if (active) Q.order[ob + __popc(am & lt)] = v;
   }
   // sub-CTA classes and fragments
 #pragma unroll

@@ -365,6 +365,13 @@ def _extras(a, G, g, srcs, level, flush, stream, sage):
                   "ms": float(np.mean([t for t, _ in r])), "iterations": r[-1][1]["levels"],
                   "arcs_relaxed_per_edge": r[-1][1]["arcs_inspected"] / g.m,
                   "model_GBps": float(np.mean([st["model_bytes"] / (st["kernel_ms"] * 1e-3) / 1e9 for _, st in r]))}
+    # Betweenness Centrality (NEXT #1): one source = forward sigma BFS + backward delta sweep
+    bcv = torch.empty(g.n, dtype=torch.float64, device="cuda")
+    G.bc([int(srcs[0])], out=bcv)
+    r = _time_calls(lambda i: G.bc([int(srcs[i])], out=bcv)[1], k, flush, stream)
+    ex["bc"] = {"ms_per_source": float(np.mean([t for t, _ in r])),
+                "gteps": len(r) / sum(t * 1e-3 * 1e9 / st["edges_traversed"] for t, st in r),
+                "note": "edges = reached undirected edges of the source; both passes inside the time"}
     # PageRank 20 iterations: pull (default on symmetric graphs) and the paper's push form
     x = torch.empty(g.n, dtype=torch.float64, device="cuda")
     ex["pagerank"] = {}

@@ -77,3 +77,12 @@ def test_c2_reorder_keeps_bfs(c2):
         assert np.array_equal(lv, ref)
         perm = H.permutation()
         assert np.array_equal(np.sort(perm), np.arange(c2.n, dtype=np.int32))
+
+
+def test_c2_bc_one_source(c2, G):
+    """NEXT #1 at full size: one source's Brandes dependencies vs the serial oracle."""
+    s = sg.sources(c2, 1, seed=6)
+    got, st = G.bc(s)
+    ref = oracle.bc(c2.off, c2.col, s)
+    tol = 1e-9 * np.max(np.abs(ref)) + 1e-6 * np.abs(ref)
+    assert np.all(np.abs(got - ref) <= tol)

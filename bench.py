@@ -432,12 +432,13 @@ def _extras(a, G, g, srcs, level, flush, stream, sage):
     # one Sampling-based Reordering round on a copy of the graph (C3-style reorder on/off)
     with sage.load_csr(torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda(), symmetric=True,
                        stream=stream.cuda_stream) as H:
+        H.reorder(1)                 # warm-up round (first call builds the resident log, grows the pool)
         ob0 = H.objective(8)
         _, _, b0 = H.bfs(int(srcs[1]), out=level, push_only=True)
         st = H.reorder(1)
         ob1 = H.objective(8)
         _, _, b1 = H.bfs(int(srcs[1]), out=level, push_only=True)
-        ex["reorder"] = {"round_ms": st["ms"], "swaps": st["vertices_discovered"], "movers": st["vertices_expanded"],
+        ex["reorder"] = {"round_ms": st["ms"], "note": "second round on the graph (first round = warm-up)", "swaps": st["vertices_discovered"], "movers": st["vertices_expanded"],
                          "objective_before": ob0, "objective_after": ob1,
                          "bfs_push_ms_before": b0["kernel_ms"], "bfs_push_ms_after": b1["kernel_ms"]}
     return ex

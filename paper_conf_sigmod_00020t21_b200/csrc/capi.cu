@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 #include <stdarg.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <string>
@@ -67,7 +68,8 @@ static cudaMemPool_t pool_for(int dev) {
 sage_status dalloc(sage_graph *g, void **p, size_t bytes) {
   *p = nullptr;
   if (bytes == 0) bytes = 16;
-  cudaMemPool_t pool = pool_for(g->device);
+  static const bool use_pool = getenv("SAGE_NO_POOL") == nullptr;
+  cudaMemPool_t pool = use_pool ? pool_for(g->device) : nullptr;
   cudaError_t e = pool ? cudaMallocFromPoolAsync(p, bytes, pool, g->stream)
                        : cudaMallocAsync(p, bytes, g->stream);
   if (e != cudaSuccess) {

@@ -39,6 +39,7 @@ struct TraversalState {     // per-query scratch, allocated on first use and kep
   int *far[3] = {nullptr, nullptr, nullptr};  // SSSP near-far: rotating far piles
   uint32_t *infar = nullptr;      // SSSP near-far: far-pile membership bitmap
   PaddedCounter *farc = nullptr;  // SSSP near-far: [3] pile sizes + [3] scan minima
+  void *tailmem = nullptr;        // BFS tail mode state (global scratch)
 };
 
 struct PageRankState {      // the all-V resident tile log (built once, reused)

@@ -127,6 +127,7 @@ struct SsspPush {
   }
 };
 
+struct TailSmem;
 // ============================================================================ kernel args
 struct TravArgs {
   const long long *off;
@@ -147,6 +148,7 @@ struct TravArgs {
   double alpha, beta;
   int max_levels;
   int *tail;            // tail mode: next-frontier list (n entries of scratch)
+  struct TailSmem *tailmem;   // tail mode state (global scratch: only block 0 uses it)
   int steal;            // 0 = ablation: static tile assignment instead of stealing
 };
 
@@ -292,7 +294,10 @@ __device__ __forceinline__ int block_scan_excl(int x, int *out_excl, int *wsum) 
   return total;
 }
 
-// Block 0 only.  Runs levels Lstart, Lstart+1, ... while the frontier is small.
+// Block 0 only.  Runs levels Lstart, Lstart+1, ... while the frontier is small.  The state `ts`
+// lives in a small global scratch block (L1-cached for this CTA) rather than in shared memory, so
+// the persistent kernel's static shared memory — and with it the L1 left for the status words of
+// the main path — is unchanged.
 __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
   Ctl *ctl = a.ctl;
   const int tid = threadIdx.x, lane = (int)lane_id(), warp = tid >> 5;
@@ -451,7 +456,6 @@ template <int VEC>
 __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_constant__ TravArgs a) {
   __shared__ WarpScratch wsm[kWarps];
   __shared__ BfsPush::Src fsrc[kWarps][32];
-  __shared__ TailSmem tsm;
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
   double mU = (double)a.m - (double)ldcg(&ctl->set[0].arcsF.v);
@@ -500,7 +504,7 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
           __syncthreads();
           if (threadIdx.x == 0) ctl->tail_state = 0;
           __syncthreads();
-          tail_run(a, L + 1, tsm);
+          tail_run(a, L + 1, *a.tailmem);
         }
         grid_barrier(&ctl->bar);
         if (ldcg(&ctl->tail_state) == 1) break;
@@ -1092,6 +1096,7 @@ void free_traversal_state(sage_graph *g) {
   dfree(g, t.bins);
   dfree(g, t.fill);
   for (int i = 0; i < 3; ++i) dfree(g, t.far[i]);
+  dfree(g, t.tailmem);
   dfree(g, t.infar);
   dfree(g, t.farc);
   t = TraversalState();
@@ -1115,6 +1120,10 @@ sage_status ensure_traversal_state(sage_graph *g) {
       free_traversal_state(g);
       return st;
     }
+  if ((st = dalloc(g, &t.tailmem, sizeof(TailSmem))) != SAGE_OK) {
+    free_traversal_state(g);
+    return st;
+  }
   for (int i = 0; i < 2; ++i)
     if ((st = alloc_queues(g, &t.q[i], n, g->m)) != SAGE_OK) {
       free_traversal_state(g);
@@ -1188,6 +1197,7 @@ static TravArgs make_args(sage_graph *g) {
   a.beta = g->beta;
   a.max_levels = (int)std::min<long long>(g->n + 1, 0x7fffffffll);
   a.tail = (int *)g->ts.tmp_out;
+  a.tailmem = reinterpret_cast<TailSmem *>(g->ts.tailmem);
   a.steal = 1;
   a.vec_ok = g->vec_ok ? 1 : 0;
   return a;

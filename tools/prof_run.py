@@ -14,7 +14,7 @@ p = argparse.ArgumentParser()
 p.add_argument("--scale", type=int, default=24)
 p.add_argument("--graph", default="rmat", choices=["rmat", "uk", "twitter"])
 p.add_argument("--n", type=int, default=0, help="vertices for uk / twitter shapes")
-p.add_argument("--op", default="bfs_push", choices=["bfs_push", "bfs_do", "sssp", "pr"])
+p.add_argument("--op", default="bfs_push", choices=["bfs_push", "bfs_do", "sssp", "pr", "reorder", "bc"])
 p.add_argument("--reps", type=int, default=3)
 p.add_argument("--tile-cta", type=int, default=256)
 p.add_argument("--align", type=int, default=4)
@@ -39,16 +39,20 @@ for i in range(a.reps):
         _, _, st = G.bfs(int(src[i]), out=lv, binning=a.binned)
     elif a.op == "sssp":
         _, st = G.sssp(int(src[i]), out=lv.view(torch.uint32))
+    elif a.op == "reorder":
+        st = G.reorder(1)
+    elif a.op == "bc":
+        _, st = G.bc([int(src[i])])
     else:
         x = torch.empty(g.n, dtype=torch.float64, device="cuda")
         _, st = G.pagerank(0.85, 5, out=x)
     print(a.op, i, {k: st[k] for k in ("levels", "kernel_ms", "ms", "edges_traversed", "model_bytes")}, flush=True)
-    if a.op != "pr" and os.environ.get("LEVELS", "1") == "0":
+    if a.op not in ("pr", "reorder", "bc") and os.environ.get("LEVELS", "1") == "0":
         rec = G.level_records()
         dt = np.diff(np.concatenate([[0], rec[:, 6]])) / 1e3
         small = dt[rec[:, 2] < 10000]
         print("   levels=%d  median small-level us=%.1f  total small-level ms=%.2f" % (len(rec), np.median(small) if len(small) else 0, small.sum() / 1e3))
-    if a.op != "pr" and os.environ.get("LEVELS", "1") == "1":
+    if a.op not in ("pr", "reorder", "bc") and os.environ.get("LEVELS", "1") == "1":
         prev = 0
         for r in G.level_records():
             print("   L dir=%d |F|=%9d arcsF=%11d insp=%11d disc=%9d  %8.1f us (work done at +%8.1f, phase1 +%8.1f)" % (

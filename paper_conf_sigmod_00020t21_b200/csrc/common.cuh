@@ -161,10 +161,15 @@ __device__ __forceinline__ uint32_t ld_colu(const uint32_t *p, unsigned long lon
                : "=r"(r) : "l"(p), "l"(pol));
   return r;
 }
-// status word load (coherent, L1-cacheable, kept in L2)
+// status word load (kept in L2).  SAGE_STATUS_NC selects the non-coherent path: a stale read
+// is harmless for the visited bitmap (bits only go 0 -> 1 within a kernel, atomicOr decides).
 __device__ __forceinline__ uint32_t ld_status(const uint32_t *p, unsigned long long pol) {
   uint32_t r;
+#if defined(SAGE_STATUS_NC) && SAGE_STATUS_NC
+  asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+#else
   asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+#endif
   return r;
 }
 template <class T> __device__ __forceinline__ T ldcg(const T *p) { return __ldcg(p); }

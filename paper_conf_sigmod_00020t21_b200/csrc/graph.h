@@ -40,6 +40,7 @@ struct TraversalState {     // per-query scratch, allocated on first use and kep
   uint32_t *infar = nullptr;      // SSSP near-far: far-pile membership bitmap
   PaddedCounter *farc = nullptr;  // SSSP near-far: [3] pile sizes + [3] scan minima
   void *tailmem = nullptr;        // BFS tail mode state (global scratch)
+  uint32_t *expd = nullptr;       // SSSP near-far: last expanded distance per vertex
 };
 
 struct PageRankState {      // the all-V resident tile log (built once, reused)

@@ -90,10 +90,13 @@ struct SsspPush {
   uint32_t *infar;      // far-pile membership bitmap
   int *far;             // far pile being appended to
   unsigned long long *far_cnt;
+  uint32_t *expd;       // distance at which each vertex was last expanded (near-far only)
 
   __device__ __forceinline__ Src src(bool valid, int u, long long, long long) const {
     // dist[u] may have been lowered by another SM in an earlier iteration: read through L2
-    return Src{valid ? ldcg(dist + u) : 0xffffffffu};
+    const uint32_t du = valid ? ldcg(dist + u) : 0xffffffffu;
+    if (valid && expd) expd[u] = du;
+    return Src{du};
   }
 
   template <int N>
@@ -822,6 +825,7 @@ static size_t bin_smem_bytes(int nslices, long long n) {
 struct FarArgs {                      // near-far state of k_sssp
   int *far[3];                       // three rotating far piles (append / scan / spare)
   uint32_t *infar;                   // far-pile membership bitmap
+  uint32_t *expd;                    // last expanded distance per vertex (stale far entries)
   PaddedCounter *cnt;                // [3] far pile sizes
   PaddedCounter *fmin;               // [3] min distance seen in a scan
   unsigned long long delta;          // threshold step; 0xffff... = plain Bellman-Ford
@@ -849,7 +853,8 @@ __device__ __forceinline__ void far_scan(const TravArgs &a, const FarArgs &fa, i
       const uint32_t bit = 1u << (v & 31);
       if (d < T) {
         atomicAnd(fa.infar + (v >> 5), ~bit);
-        move = !(atomicOr(inq_next + (v >> 5), bit) & bit);
+        // skip entries whose vertex was already expanded at its current distance
+        move = ldcg(fa.expd + v) != d && !(atomicOr(inq_next + (v >> 5), bit) & bit);
       } else {
         keep = true;
         if (d < mn) mn = d;
@@ -901,6 +906,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
     f.infar = fa.infar;
     f.far = fa.far[k % 3];
     f.far_cnt = &fa.cnt[k % 3].v;
+    f.expd = fa.delta == ~0ull ? nullptr : fa.expd;
     consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok);
     if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
     grid_barrier(&ctl->bar);
@@ -1097,6 +1103,7 @@ void free_traversal_state(sage_graph *g) {
   dfree(g, t.fill);
   for (int i = 0; i < 3; ++i) dfree(g, t.far[i]);
   dfree(g, t.tailmem);
+  dfree(g, t.expd);
   dfree(g, t.infar);
   dfree(g, t.farc);
   t = TraversalState();
@@ -1411,6 +1418,7 @@ extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_o
   FarArgs fa;
   for (int i = 0; i < 3; ++i) fa.far[i] = t.far[i];
   fa.infar = t.infar;
+  fa.expd = reinterpret_cast<uint32_t *>(t.far[2]) + 0;   // placeholder, set below
   fa.cnt = t.farc;
   fa.fmin = t.farc + 3;
   {
@@ -1421,6 +1429,12 @@ extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_o
     fa.delta = dl <= 0.0 ? ~0ull : (unsigned long long)std::max(1.0, std::floor(dl + 0.5));
     if (!env) fa.delta = ~0ull;   // default: plain frontier Bellman-Ford (near-far measured slower)
   }
+  if (fa.delta != ~0ull) {
+    if (!t.expd && (s = dalloc(g, (void **)&t.expd, sizeof(uint32_t) * (size_t)g->n_local)) != SAGE_OK)
+      return s;
+    cudaMemsetAsync(t.expd, 0xff, sizeof(uint32_t) * (size_t)g->n_local, g->stream);
+  }
+  fa.expd = t.expd;
   cudaMemsetAsync(t.infar, 0, sizeof(uint32_t) * words, g->stream);
   cudaMemsetAsync(t.farc, 0, sizeof(PaddedCounter) * 3, g->stream);
   cudaMemsetAsync(t.farc + 3, 0xff, sizeof(PaddedCounter) * 3, g->stream);

@@ -531,16 +531,14 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
 // B200 restructuring of the push filter: a scattered 4-B status read costs about one
 // L1TEX cycle per SM from L2-resident global memory but ~0.2 from shared memory (measured,
 // tools/micro/status_reads.cu).  A push level therefore runs in two phases:
-//   phase 1: the unchanged TP + RTS expansion; every neighbour id is appended to the bin of its
-//            vertex slice (1M ids = 128 KB of bitmap) through warp-private staging in shared
-//            memory, flushed to HBM in coalesced 128-B chunks;
+//   phase 1: the unchanged TP + RTS expansion; every neighbour id is stored into the bin of its
+//            vertex slice (1M ids = 128 KB of bitmap), in a chunk reserved per (warp, slice);
 //   phase 2: each CTA stages the visited bits of one slice in shared memory and runs Alg. 1's
 //            filter on its share of that slice's bin; a vertex new to the CTA is claimed with a
 //            global atomicOr (other CTAs of the slice), and filtered-in vertices are classified
 //            into the next level's log exactly as before.
 constexpr int kBinBlock = 1024;
 constexpr int kBinWarps = kBinBlock / 32;
-constexpr int kBinE = 32;            // staged entries per (warp, slice)
 constexpr int kMaxSlices = 40;
 constexpr int kSliceLg = 20;         // 2^20 vertices per slice
 constexpr int kBinRes = 512;         // entries reserved per (warp, slice) with one atomic
@@ -565,8 +563,6 @@ struct BinPush {
   // phase-1 context
   const TravArgs *a;
   const BinArgs *b;
-  int *stage;                        // this warp's [nslices][kBinE]
-  int *cnt;                          // this warp's [nslices]
   int *rpos, *rend;                  // this warp's reserved bin range per slice
   int fillset;
   int next_level;
@@ -575,44 +571,6 @@ struct BinPush {
   CounterSet *csn;
   __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
 
-  // write `c` staged entries of slice s to HBM (or, if the bin is full, filter them directly).
-  // Bin space is reserved kBinRes entries at a time, so the global atomic is off the common path.
-  __device__ __forceinline__ void emit(int s, int c, const int *src) const {
-    const unsigned lane = lane_id();
-    int pos = rpos[s], end = rend[s];
-    const bool has = (int)lane < c;
-    const int x = has ? src[lane] : 0;
-    if (end - pos < c) {
-      // pad the rest of the old reservation, take a new one
-      for (int i = pos + (int)lane; i < end; i += 32) b->bins[(long long)s * b->cap + i] = -1;
-      unsigned long long np = 0;
-      if (lane == 0) np = atomicAdd(&b->fill[fillset * kMaxSlices + s].v, (unsigned long long)kBinRes);
-      np = shfl64(np, 0);
-      pos = (int)min(np, (unsigned long long)b->cap);
-      end = (int)min(np + kBinRes, (unsigned long long)b->cap);
-    }
-    if (end - pos >= c) {
-      if (has) b->bins[(long long)s * b->cap + pos + lane] = x;
-      pos += c;
-    } else {   // bin full (skewed ids): Alg. 1's filter on the global bitmap for these entries
-      bool disc = false;
-      if (has) {
-        const uint32_t bit = 1u << (x & 31);
-        disc = !(atomicOr(a->visited + (x >> 5), bit) & bit);
-        if (disc) {
-          a->level[x] = next_level;
-          if (a->do_enabled) atomicOr(a->fb[next_level % 3] + (x >> 5), bit);
-        }
-      }
-      enqueue_ids(disc, x, a->off, a->L, *qn, csn);
-    }
-    __syncwarp();
-    if (lane == 0) {
-      rpos[s] = pos;
-      rend[s] = end;
-    }
-    __syncwarp();
-  }
   // end of phase 1: pad the unused part of every reservation
   __device__ __forceinline__ void close_reservations() const {
     const unsigned lane = lane_id();
@@ -622,41 +580,63 @@ struct BinPush {
     }
   }
 
-  // Warp multi-split of 32 ids into their slices: lanes of one slice are found with one ballot per
-  // slice-id bit (no match.any), ranked with popc, staged in this warp's smem rows (stride
-  // kBinE + 1 against bank conflicts); a full row is flushed to HBM in one coalesced store.
+  // Warp multi-split of 32 ids into their slices without staging: lanes of one slice are found
+  // with one ballot per slice-id bit, ranked with popc, and stored straight into this warp's
+  // reserved chunk of the slice's bin (one global atomic per kBinRes ids and slice).
   __device__ __forceinline__ void append(bool valid, int v) const {
     const unsigned lane = lane_id();
     const int sl = valid ? (v >> b->slice_lg) : 0;
     unsigned grp = __ballot_sync(FULL, valid);
     if (!grp) return;
-    for (int bit = 0; bit < nbits; ++bit) {
-      const bool on = (sl >> bit) & 1;
-      const unsigned bb = __ballot_sync(FULL, on);
-      grp &= on ? bb : ~bb;
+#pragma unroll
+    for (int bit = 0; bit < 6; ++bit) {
+      if (bit < nbits) {
+        const bool on = (sl >> bit) & 1;
+        const unsigned bb = __ballot_sync(FULL, on);
+        grp &= on ? bb : ~bb;
+      }
     }
-    const int c0 = valid ? cnt[sl] : 0;
-    const int idx = c0 + __popc(grp & lanemask_lt());
-    const int tot = c0 + __popc(grp);
-    const bool leader = valid && (grp & lanemask_lt()) == 0;
-    if (valid && idx < kBinE) stage[sl * (kBinE + 1) + idx] = v;
-    __syncwarp();
-    if (leader) cnt[sl] = tot < kBinE ? tot : tot - kBinE;
-    unsigned fm = __ballot_sync(FULL, leader && tot >= kBinE);
-    while (fm) {
-      const int ld = __ffs(fm) - 1;
-      fm &= fm - 1;
+    const unsigned lt = lanemask_lt();
+    const int rank = __popc(grp & lt), c = __popc(grp);
+    const bool leader = valid && rank == 0;
+    int pos = valid ? rpos[sl] : 0;
+    const int end = valid ? rend[sl] : 0;
+    unsigned nm = __ballot_sync(FULL, leader && end - pos < c);
+    while (nm) {   // new reservation for the slices whose chunk is too small (rare)
+      const int ld = __ffs(nm) - 1;
+      nm &= nm - 1;
       const int s2 = __shfl_sync(FULL, sl, ld);
-      const unsigned g2 = __shfl_sync(FULL, grp, ld);
-      const int c2 = __shfl_sync(FULL, c0, ld);
+      const int p2 = rpos[s2], e2 = rend[s2];
+      for (int i = p2 + (int)lane; i < e2; i += 32) b->bins[(long long)s2 * b->cap + i] = -1;
+      unsigned long long np = 0;
+      if (lane == 0) np = atomicAdd(&b->fill[fillset * kMaxSlices + s2].v, (unsigned long long)kBinRes);
+      np = shfl64(np, 0);
       __syncwarp();
-      emit(s2, kBinE, stage + s2 * (kBinE + 1));
-      // the group's overflow (positions >= kBinE) restarts the row
-      if ((g2 >> lane) & 1u) {
-        const int id2 = c2 + __popc(g2 & lanemask_lt());
-        if (id2 >= kBinE) stage[s2 * (kBinE + 1) + id2 - kBinE] = v;
+      if (lane == 0) {
+        rpos[s2] = (int)min(np, (unsigned long long)b->cap);
+        rend[s2] = (int)min(np + kBinRes, (unsigned long long)b->cap);
       }
       __syncwarp();
+    }
+    pos = valid ? rpos[sl] : 0;
+    const bool fits = valid && pos + c <= rend[sl];
+    if (fits) b->bins[(long long)sl * b->cap + pos + rank] = v;
+    __syncwarp();
+    if (leader && fits) rpos[sl] = pos + c;
+    __syncwarp();
+    // bin capacity exhausted (skewed ids): Alg. 1's filter on the global bitmap directly
+    const bool direct = valid && !fits;
+    if (__any_sync(FULL, direct)) {
+      bool disc = false;
+      if (direct) {
+        const uint32_t bit = 1u << (v & 31);
+        disc = !(atomicOr(a->visited + (v >> 5), bit) & bit);
+        if (disc) {
+          a->level[v] = next_level;
+          if (a->do_enabled) atomicOr(a->fb[next_level % 3] + (v >> 5), bit);
+        }
+      }
+      enqueue_ids(disc, v, a->off, a->L, *qn, csn);
     }
   }
 
@@ -733,11 +713,10 @@ __global__ void __launch_bounds__(kBinBlock, 1) k_bfs_bin(const __grid_constant_
   extern __shared__ __align__(16) unsigned char dsm[];
   WarpScratch *wsm = reinterpret_cast<WarpScratch *>(dsm);
   BinPush::Src *fsrc = reinterpret_cast<BinPush::Src *>(dsm + sizeof(WarpScratch) * kBinWarps);
-  int *cnts = reinterpret_cast<int *>(dsm + sizeof(WarpScratch) * kBinWarps + sizeof(BinPush::Src) * 32 * kBinWarps);
-  int *rps = cnts + kMaxSlices * kBinWarps;
+  int *rps = reinterpret_cast<int *>(dsm + sizeof(WarpScratch) * kBinWarps + sizeof(BinPush::Src) * 32 * kBinWarps);
   int *res = rps + kMaxSlices * kBinWarps;
   unsigned char *U = dsm + sizeof(WarpScratch) * kBinWarps + sizeof(BinPush::Src) * 32 * kBinWarps +
-                     3 * sizeof(int) * kMaxSlices * kBinWarps;
+                     2 * sizeof(int) * kMaxSlices * kBinWarps;
   const int warp = threadIdx.x >> 5;
   const unsigned lane = lane_id();
   Ctl *ctl = a.ctl;
@@ -755,10 +734,7 @@ __global__ void __launch_bounds__(kBinBlock, 1) k_bfs_bin(const __grid_constant_
     if (a.do_enabled) clear_words(a.fb[(L + 2) % 3], nwords);
     if (dir == 0) {
       // phase 1: expansion into slice bins
-      int *cnt = cnts + warp * kMaxSlices;
-      int *stage = reinterpret_cast<int *>(U) + warp * b.nslices * (kBinE + 1);
       for (int i = lane; i < b.nslices; i += 32) {
-        cnt[i] = 0;
         rps[warp * kMaxSlices + i] = 0;
         res[warp * kMaxSlices + i] = 0;
       }
@@ -766,8 +742,6 @@ __global__ void __launch_bounds__(kBinBlock, 1) k_bfs_bin(const __grid_constant_
       BinPush f;
       f.a = &a;
       f.b = &b;
-      f.stage = stage;
-      f.cnt = cnt;
       f.rpos = rps + warp * kMaxSlices;
       f.rend = res + warp * kMaxSlices;
       f.fillset = L & 1;
@@ -777,10 +751,6 @@ __global__ void __launch_bounds__(kBinBlock, 1) k_bfs_bin(const __grid_constant_
       f.qn = &a.q[(L + 1) & 1];
       f.csn = nxt;
       consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc + warp * 32, a.vec_ok);
-      for (int sl = 0; sl < b.nslices; ++sl) {
-        const int c = cnt[sl];
-        if (c) f.emit(sl, c, stage + sl * (kBinE + 1));
-      }
       f.close_reservations();
       grid_barrier(&ctl->bar);
       if (blockIdx.x == 0 && threadIdx.x == 0 && L < kMaxRec)
@@ -814,11 +784,11 @@ __global__ void __launch_bounds__(kBinBlock, 1) k_bfs_bin(const __grid_constant_
 
 static size_t bin_smem_bytes(int nslices, long long n) {
   const size_t fixed = sizeof(WarpScratch) * kBinWarps + sizeof(int) * 32 * kBinWarps +
-                       3 * sizeof(int) * kMaxSlices * kBinWarps;
-  const size_t stage = sizeof(int) * (size_t)kBinWarps * nslices * (kBinE + 1);
+                       2 * sizeof(int) * kMaxSlices * kBinWarps;
   const long long sw = std::min<long long>(n, 1ll << kSliceLg);
   const size_t bm = sizeof(uint32_t) * (size_t)((sw + 31) / 32 + 1);
-  return fixed + std::max(stage, bm);
+  (void)nslices;
+  return fixed + bm;
 }
 
 // ============================================================================ SSSP kernel

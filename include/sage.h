@@ -52,6 +52,12 @@ enum {
   SAGE_F_BORROW = 4u,      /* with DEVICE_PTRS: use the caller arrays in place (no copy); the caller
                               keeps them alive and unmodified until sage_free                      */
   SAGE_F_NO_VALIDATE = 8u, /* skip the validation pass of sage_load_csr                              */
+  SAGE_F_HOST_COLUMNS = 128u, /* out-of-core: col_indices /
+                              weights (host arrays) stay in pinned, mapped host memory and the
+                              kernels read them zero-copy over the host link; with SAGE_F_BORROW
+                              the caller's pages are registered in place, otherwise copied into
+                              library-owned pinned memory.  A tile alignment of 32 (128 B) keeps
+                              every tile request line-aligned.  sage_reorder is unsupported.     */
   SAGE_F_PUSH_ONLY = 16u,  /* disable direction switching: every level is the paper's push
                               expansion (Alg. 2/3).  Can also be set per call (sage_bfs_ex).     */
   SAGE_F_BINNED = 32u,     /* per call (sage_bfs_ex), experimental: two-phase push levels (neighbour

@@ -20,6 +20,7 @@ LIB_PATH = os.path.join(_HERE, os.environ.get("SAGE_LIB", "libsage.so"))
 
 OK, E_INVALID, E_NOMEM, E_CUDA, E_NCCL, E_OVERFLOW, E_UNSUPPORTED = range(7)
 F_SYMMETRIC, F_DEVICE_PTRS, F_BORROW, F_NO_VALIDATE, F_PUSH_ONLY, F_BINNED, F_NO_STEALING = 1, 2, 4, 8, 16, 32, 64
+F_HOST_COLUMNS = 128
 STATUS_NAMES = {0: "SAGE_OK", 1: "SAGE_E_INVALID", 2: "SAGE_E_NOMEM", 3: "SAGE_E_CUDA",
                 4: "SAGE_E_NCCL", 5: "SAGE_E_OVERFLOW", 6: "SAGE_E_UNSUPPORTED"}
 
@@ -299,7 +300,7 @@ def load_csr(off, col, w=None, n: int | None = None, symmetric: bool = False, pu
              borrow: bool = False, validate: bool = True, tile_cta: int = 256, tile_min: int = 8,
              align: int = 4, alpha: float = 15.0, beta: float = 18.0, stream=None,
              rank: int = 0, world: int = 1, nccl_unique_id: bytes | None = None,
-             v_begin: int = 0, v_end: int | None = None) -> Graph:
+             v_begin: int = 0, v_end: int | None = None, host_columns: bool = False) -> Graph:
     """sage_load_csr.  ``off``/``col``/``w`` are host arrays or tensors, or CUDA tensors."""
     po, ko, dev_o = _ptr(off, np.int64)
     pc, kc, dev_c = _ptr(col, np.int32)
@@ -314,6 +315,8 @@ def load_csr(off, col, w=None, n: int | None = None, symmetric: bool = False, pu
         flags |= F_DEVICE_PTRS | (F_BORROW if borrow else 0)
     if not validate:
         flags |= F_NO_VALIDATE
+    if host_columns:
+        flags |= F_HOST_COLUMNS | (F_BORROW if borrow else 0)
     csr = Csr()
     csr.n = int(n if n is not None else n_rows)
     csr.m = int(len(col))

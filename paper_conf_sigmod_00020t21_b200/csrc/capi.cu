@@ -213,6 +213,11 @@ static void destroy(sage_graph *g) {
   if (g->own_off) dfree(g, g->off);
   if (g->own_col) dfree(g, g->col);
   if (g->own_w) dfree(g, g->w);
+  cudaStreamSynchronize(g->stream);
+  for (int i = 0; i < 2; ++i) {
+    if (g->host_registered[i]) cudaHostUnregister(g->host_registered[i]);
+    if (g->host_owned[i]) cudaFreeHost(g->host_owned[i]);
+  }
   dfree(g, g->sigma);
   dfree(g, g->sigma_inv);
   cudaStreamSynchronize(g->stream);
@@ -300,7 +305,48 @@ sage_status sage_load_csr(const sage_csr *in, sage_graph **out) {
   // copy or borrow
   const size_t offb = sizeof(int64_t) * (size_t)(n_local + 1);
   const size_t colb = sizeof(int32_t) * (size_t)in->m;
-  if (borrow) {
+  if (flags & SAGE_F_HOST_COLUMNS) {
+    // out-of-core (NEXT #4): columns / weights stay in pinned host memory and the
+    // kernels read them zero-copy over PCIe / C2C; offsets and all per-vertex state are on the GPU
+    if (devptrs) {
+      set_error("SAGE_F_HOST_COLUMNS needs host input arrays");
+      destroy(g);
+      return SAGE_E_INVALID;
+    }
+    if ((st = dalloc(g, (void **)&g->off, offb)) != SAGE_OK) {
+      destroy(g);
+      return st;
+    }
+    g->own_off = true;
+    cudaMemcpyAsync(g->off, in->row_offsets, offb, cudaMemcpyHostToDevice, g->stream);
+    const void *hsrc[2] = {in->col_indices, in->weights};
+    for (int i = 0; i < 2; ++i) {
+      if (!hsrc[i] || !colb) continue;
+      void *h = nullptr;
+      cudaError_t e;
+      if (flags & SAGE_F_BORROW) {   // register the caller's pages in place
+        h = const_cast<void *>(hsrc[i]);
+        e = cudaHostRegister(h, colb, cudaHostRegisterMapped | cudaHostRegisterReadOnly);
+        if (e == cudaSuccess) g->host_registered[i] = h;
+      } else {                       // library-owned pinned copy
+        e = cudaHostAlloc(&h, colb + 16, cudaHostAllocMapped);
+        if (e == cudaSuccess) {
+          g->host_owned[i] = h;
+          memcpy(h, hsrc[i], colb);
+        }
+      }
+      void *d = nullptr;
+      if (e == cudaSuccess) e = cudaHostGetDevicePointer(&d, h, 0);
+      if (e != cudaSuccess) {
+        cuda_fail(nullptr, e, "host-resident columns");
+        destroy(g);
+        return SAGE_E_CUDA;
+      }
+      if (i == 0) g->col = (int32_t *)d;
+      else g->w = (uint32_t *)d;
+    }
+    g->host_columns = true;
+  } else if (borrow) {
     g->off = const_cast<int64_t *>(in->row_offsets);
     g->col = const_cast<int32_t *>(in->col_indices);
     g->w = const_cast<uint32_t *>(in->weights);

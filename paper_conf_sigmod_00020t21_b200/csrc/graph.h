@@ -70,6 +70,9 @@ struct sage_graph {
   int32_t *col = nullptr;     // device, m
   uint32_t *w = nullptr;      // device, m or null
   bool own_off = false, own_col = false, own_w = false;
+  bool host_columns = false;          // SAGE_F_HOST_COLUMNS: col / w are mapped pinned host memory
+  void *host_registered[2] = {nullptr, nullptr};   // caller pages registered in place (col, w)
+  void *host_owned[2] = {nullptr, nullptr};        // library-owned pinned copies (col, w)
   bool rows_sorted = false;
   int64_t max_degree = 0;
   int64_t n_isolated = 0;

@@ -534,6 +534,10 @@ extern "C" sage_status sage_reorder(sage_graph *g, int32_t rounds, const sage_re
     set_error("sage_reorder is single-GPU only");
     return SAGE_E_UNSUPPORTED;
   }
+  if (g->host_columns) {
+    set_error("sage_reorder needs device-resident columns (not SAGE_F_HOST_COLUMNS)");
+    return SAGE_E_UNSUPPORTED;
+  }
   int S = 8;
   if (opt && opt->sector_width) S = opt->sector_width;
   if (S < 1 || S > 64 || (S & (S - 1))) {

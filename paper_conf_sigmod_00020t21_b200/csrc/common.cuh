@@ -172,6 +172,14 @@ __device__ __forceinline__ uint32_t ld_status(const uint32_t *p, unsigned long l
 #endif
   return r;
 }
+// Predicated atomicOr: issues the atomic only when `pred`; otherwise returns `dflt`.  Written as
+// one predicated instruction (no branch) so a lane's several claims are in flight together.
+__device__ __forceinline__ uint32_t atom_or_if(bool pred, uint32_t *p, uint32_t bits, uint32_t dflt) {
+  uint32_t r = dflt;
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q atom.global.or.b32 %0, [%1], %2;\n\t}"
+               : "+r"(r) : "l"(p), "r"(bits), "r"((uint32_t)pred));
+  return r;
+}
 template <class T> __device__ __forceinline__ T ldcg(const T *p) { return __ldcg(p); }
 __device__ __forceinline__ CtaTile ldcg_tile(const CtaTile *p) {
   longlong2 v = __ldcg(reinterpret_cast<const longlong2 *>(p));
@@ -473,8 +481,8 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
     if ((unsigned long long)gwarp >= grabs) continue;
     const int sub = lane / lpt, sl = lane % lpt;
     const bool contiguous = lpt < 32 && vec_ok && VEC == 4;
+    const int lg_spt = __ffs(spt) - 1;
     for (unsigned long long rr = 0;; ++rr) {
-      PROF_T(tt0);
       unsigned long long base = 0;
       if (steal) {
         if (lane == 0) base = atomicAdd(&cs->tk[c].v, batch);
@@ -482,80 +490,96 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
       } else {
         base = ((unsigned long long)gwarp + rr * (unsigned long long)nwarps) * batch;
       }
-      PROF_T(tt1);
-      PROF_ADD(5, tt1 - tt0);
-      PROF_ADD(6, 1);
       if (base >= count) break;
       const unsigned long long end = (base + batch < count) ? base + batch : count;
-      for (unsigned long long i = base; i < end; i += tps) {
-        const unsigned long long ti = i + sub;
-        const bool valid = ti < end;
-        long long start = 0, rb = 0, re = 0;
-        int u = 0;
-        if (valid) {
-          if (c == 0) {
-            CtaTile T = ldcg_tile(Q.cta + ti);
-            start = T.start;
-            u = T.u;
-            if (F::kNeedRow) {
+      for (unsigned long long r0 = base; r0 < end; r0 += 32) {
+        // ---- metadata round: lane k resolves tile r0 + k (log entry -> row -> tile start and
+        //      the filter's per-source context) in ONE round of loads for up to 32 tiles; the
+        //      steps below read them from shared memory.
+        const int nt = (end - r0) < 32ull ? (int)(end - r0) : 32;
+        {
+          const bool mv = (int)lane < nt;
+          long long start = 0, rb = 0, re = 0;
+          int u = 0;
+          if (mv) {
+            const unsigned long long ti = r0 + lane;
+            if (c == 0) {
+              CtaTile T = ldcg_tile(Q.cta + ti);
+              start = T.start;
+              u = T.u;
+              if (F::kNeedRow) {
+                rb = ld_off(off + u);
+                re = ld_off(off + u + 1);
+              }
+            } else {
+              u = ldcg(Q.cls[c] + ti);
               rb = ld_off(off + u);
               re = ld_off(off + u + 1);
+              RowSplit s = split_row(rb, re, L);
+              start = class_tile_start(re, s.r, t);
             }
-          } else {
-            u = ldcg(Q.cls[c] + ti);
-            rb = ld_off(off + u);
-            re = ld_off(off + u + 1);
-            RowSplit s = split_row(rb, re, L);
-            start = class_tile_start(re, s.r, t);
           }
+          const typename F::Src sc = f.src(mv, u, rb, re);
+          __syncwarp();
+          ws->hb[lane] = start;
+          fsrc[lane] = sc;
+          __syncwarp();
         }
-        const typename F::Src sc = f.src(valid, u, rb, re);
-        PROF_T(tv0);
-        if (contiguous) {
-          // sub-warp tiles: each lane reads VEC consecutive elements (one 16-B load)
-          const long long p0 = start + (long long)sl * VEC;
-          int v[VEC];
-          uint32_t ww[VEC];
-          int4 c4 = make_int4(0, 0, 0, 0);
-          uint4 w4 = make_uint4(0, 0, 0, 0);
-          if (valid) {
-            c4 = ld_col4(col + p0, pol);
-            if (F::kWeights) w4 = ld_col4u(w + p0, pol);
-          }
-          v[0] = c4.x; v[1 % VEC] = c4.y; v[2 % VEC] = c4.z; v[3 % VEC] = c4.w;
-          ww[0] = w4.x; ww[1 % VEC] = w4.y; ww[2 % VEC] = w4.z; ww[3 % VEC] = w4.w;
-          bool in[VEC];
-          f.template visit<VEC>(valid, sc, v, ww, in, lpt);
-          PROF_T(tv1);
-          PROF_ADD(2, tv1 - tv0);
-          if constexpr (F::kEnqueue) {
-#pragma unroll
-            for (int j = 0; j < VEC; ++j)
-              buffer_push(in[j], v[j], ws, bcnt, off, L, *f.next_q, f.next_cs);
-          }
-        } else {
-          // strided: lane sl reads elements sl, sl+lpt, ... (coalesced, consecutive per load)
-          for (int s = 0; s < spt; ++s) {
-            const long long p0 = start + (long long)s * (lpt * VEC) + sl;
-            int v[VEC];
-            uint32_t ww[VEC];
+        // ---- steps: step st covers tile k = (st / spt) * tps + sub, sub-step st % spt.  The
+        //      column loads of step st + 1 are issued before the filter of step st runs, so
+        //      the column stream's latency hides behind the status reads.
+        const int nst = ((nt + tps - 1) / tps) << lg_spt;
+        int vn[VEC];
+        uint32_t wn[VEC];
+        auto load_step = [&](int st, int (&v)[VEC], uint32_t (&ww)[VEC]) {
+          const int k = ((st >> lg_spt) * tps) + sub;
+          const bool valid = k < nt;
+          const long long start = ws->hb[valid ? k : 0];
+          if (contiguous) {
+            int4 c4 = make_int4(0, 0, 0, 0);
+            uint4 w4 = make_uint4(0, 0, 0, 0);
+            const long long p0 = start + (long long)sl * VEC;
+            if (valid) {
+              c4 = ld_col4(col + p0, pol);
+              if (F::kWeights) w4 = ld_col4u(w + p0, pol);
+            }
+            v[0] = c4.x; v[1 % VEC] = c4.y; v[2 % VEC] = c4.z; v[3 % VEC] = c4.w;
+            ww[0] = w4.x; ww[1 % VEC] = w4.y; ww[2 % VEC] = w4.z; ww[3 % VEC] = w4.w;
+          } else {
+            const long long p0 = start + (long long)(st & (spt - 1)) * (lpt * VEC) + sl;
 #pragma unroll
             for (int j = 0; j < VEC; ++j) {
               v[j] = valid ? ld_col(col + p0 + j * lpt, pol) : 0;
               ww[j] = (valid && F::kWeights) ? ld_colu(w + p0 + j * lpt, pol) : 0u;
             }
-            bool in[VEC];
-            f.template visit<VEC>(valid, sc, v, ww, in, lpt);
-            PROF_T(tv2);
-            PROF_ADD(3, tv2 - tv0);
-            PROF_ADD(4, 1);
-            if constexpr (F::kEnqueue) {
+          }
+        };
+        load_step(0, vn, wn);
+        for (int st = 0; st < nst; ++st) {
+          PROF_T(tv0);
+          int v[VEC];
+          uint32_t ww[VEC];
 #pragma unroll
-              for (int j = 0; j < VEC; ++j)
-                buffer_push(in[j], v[j], ws, bcnt, off, L, *f.next_q, f.next_cs);
-            }
+          for (int j = 0; j < VEC; ++j) {
+            v[j] = vn[j];
+            ww[j] = wn[j];
+          }
+          if (st + 1 < nst) load_step(st + 1, vn, wn);
+          const int k = ((st >> lg_spt) * tps) + sub;
+          const bool valid = k < nt;
+          const typename F::Src sc = fsrc[valid ? k : 0];
+          bool in[VEC];
+          f.template visit<VEC>(valid, sc, v, ww, in, lpt);
+          PROF_T(tv1);
+          PROF_ADD(2, tv1 - tv0);
+          PROF_ADD(4, 1);
+          if constexpr (F::kEnqueue) {
+#pragma unroll
+            for (int j = 0; j < VEC; ++j)
+              buffer_push(in[j], v[j], ws, bcnt, off, L, *f.next_q, f.next_cs);
           }
         }
+        __syncwarp();
       }
     }
   }

@@ -56,14 +56,17 @@ struct BfsPush {
     const unsigned long long keep = policy_evict_last();
 #pragma unroll
     for (int j = 0; j < N; ++j) wd[j] = valid ? ld_status(visited + (v[j] >> 5), keep) : 0xffffffffu;
+    // claims of all N neighbours in flight together (predicated, no branch between them)
+    uint32_t old[N];
 #pragma unroll
     for (int j = 0; j < N; ++j) {
       const uint32_t bit = 1u << (v[j] & 31);
-      in[j] = false;
-      if (!(wd[j] & bit)) {
-        const uint32_t old = atomicOr(visited + (v[j] >> 5), bit);
-        in[j] = !(old & bit);
-      }
+      old[j] = atom_or_if(!(wd[j] & bit), visited + (v[j] >> 5), bit, bit);
+    }
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const uint32_t bit = 1u << (v[j] & 31);
+      in[j] = !(old[j] & bit);
       if (in[j]) {
         level[v[j]] = next_level;
         if (parent) parent[v[j]] = s.u + v_base;

@@ -193,9 +193,12 @@ def main():
         n, m = int(hdr[0]), int(hdr[1])
         off_full = torch.from_numpy(g.off).cuda() if rank == 0 else torch.empty(n + 1, dtype=torch.int64, device="cuda")
         col_full = torch.from_numpy(g.col).cuda() if rank == 0 else torch.empty(m, dtype=torch.int32, device="cuda")
+        w_full = (torch.from_numpy(g.w.view(np.int32)).cuda() if rank == 0 else
+                  torch.empty(m, dtype=torch.int32, device="cuda"))
         if world > 1:
             torch.distributed.broadcast(off_full, 0)
             torch.distributed.broadcast(col_full, 0)
+            torch.distributed.broadcast(w_full, 0)
             obj = [gname, sage.nccl_unique_id() if rank == 0 else None]
             torch.distributed.broadcast_object_list(obj, 0)
             gname, uid = obj
@@ -205,7 +208,8 @@ def main():
         b0 = int(off_full[vb])
         off_d = (off_full[vb:ve + 1] - b0).contiguous()
         col_d = col_full[b0:int(off_full[ve])].contiguous()
-        G = sage.load_csr(off_d, col_d, n=n, symmetric=True, borrow=True, stream=stream.cuda_stream,
+        w_d = w_full[b0:int(off_full[ve])].contiguous().view(torch.uint32)
+        G = sage.load_csr(off_d, col_d, w_d, n=n, symmetric=True, borrow=True, stream=stream.cuda_stream,
                           rank=rank, world=world, nccl_unique_id=uid, v_begin=vb, v_end=ve)
         n_rows = ve - vb
         if rank != 0:
@@ -216,7 +220,7 @@ def main():
             g.off = off_full.cpu().numpy()
             g.m = m
             g.w = None
-        del off_full, col_full
+        del off_full, col_full, w_full
     srcs = sg.sources(g, a.warmup + a.steps, seed=2)
     level = torch.empty(n_rows, dtype=torch.int32, device="cuda")
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
@@ -286,12 +290,39 @@ def main():
     if rank == 0 and not a.no_extras and not multi:
         line.update(_extras(a, G, g, srcs, level, flush, stream, sage))
     if multi:
+        line["sssp"] = _sssp_multi(a, G, srcs, n_rows, world, flush, stream)
         line["e2e"] = _e2e_multi(a, G, g, srcs, sage, rank, world, off_d, col_d, n, uid if world == 1 else None)
     if rank == 0:
         print(json.dumps(line), flush=True)
     G.free()
     if world > 1:
         torch.distributed.destroy_process_group()
+
+
+def _sssp_multi(a, G, srcs, n_rows, world, flush, stream):
+    """Multi-GPU SSSP (min reduce-scatter per Bellman-Ford iteration): GTEPS over up to 4 sources,
+    each step's time = max over ranks."""
+    import torch
+    dist = torch.empty(n_rows, dtype=torch.uint32, device="cuda")
+    G.sssp(int(srcs[0]), out=dist)
+    times, edges, iters = [], [], []
+    for i in range(min(4, a.steps)):
+        flush.fill_(float(i))
+        torch.cuda.synchronize()
+        if world > 1:
+            torch.distributed.barrier()
+        _, st = G.sssp(int(srcs[a.warmup + i]), out=dist)
+        times.append(st["ms"])
+        edges.append(st["edges_traversed"])
+        iters.append(st["levels"])
+    if world > 1:
+        tt = torch.tensor(times, device="cuda")
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        times = tt.cpu().tolist()
+    g = [e / (t * 1e-3) / 1e9 for e, t in zip(edges, times)]
+    return {"gteps": len(g) / sum(1 / x for x in g), "ms": float(np.median(times)),
+            "iterations": int(np.median(iters)), "sources": len(g),
+            "exchange": "ncclReduceScatter(min) of candidate distances per iteration"}
 
 
 def _e2e_multi(a, G, g, srcs, sage, rank, world, off_d, col_d, n, uid):

@@ -70,8 +70,10 @@ enum {
 
 /* Multi-GPU description (1D vertex partition).  NULL in sage_csr = single GPU.
  * Non-NULL selects the NCCL path (also with world == 1: a 1-rank communicator).  On that path
- * sage_bfs (no parents) and sage_pagerank are collective; sage_sssp / sage_reorder return
- * SAGE_E_UNSUPPORTED.                                                    */
+ * sage_bfs (no parents), sage_sssp and sage_pagerank are collective (every rank calls them with
+ * the same arguments; outputs hold the rank's own rows); sage_reorder / sage_bc return
+ * SAGE_E_UNSUPPORTED.  Multi-GPU SSSP exchanges candidate distances of
+ * remote targets with one ncclReduceScatter(min) per Bellman-Ford iteration.                   */
 typedef struct {
   int32_t rank, world;         /* this process's rank and the number of ranks                    */
   const void *nccl_unique_id;  /* 128-byte ncclUniqueId created by rank 0 and broadcast by the

@@ -59,6 +59,7 @@ struct Comm {
   uint32_t *fb[3] = {nullptr, nullptr, nullptr};
   unsigned long long *stats = nullptr;  // 8 u64
   double *y = nullptr, *yown = nullptr, *dsum = nullptr;
+  uint32_t *cand = nullptr, *cown = nullptr;   // SSSP min-exchange buffers (p*P and P)
   PartMap pm;
 };
 
@@ -90,6 +91,13 @@ struct MultiArgs {
   int vec_ok;
   int lvl;                         // current level L
   PartMap pm;
+  // SSSP (frontier Bellman-Ford across ranks)
+  const uint32_t *w;
+  uint32_t *dist;                  // own rows' distances
+  uint32_t *cand;                  // p*P candidate distances for remote targets (UINT32_MAX = none)
+  const uint32_t *cown;            // own slice after the min reduce-scatter
+  uint32_t *inq_next;              // own rows: next-frontier dedupe bitmap
+  int *overflow;
 };
 
 struct BfsPushMulti {
@@ -243,6 +251,149 @@ __global__ void __launch_bounds__(kBlock) k_mpull(const __grid_constant__ MultiA
     if (insp) atomicAdd(&cur->inspected.v, insp);
     if (scanned) atomicAdd(&cur->scanned.v, scanned);
   }
+}
+
+// ---- multi-GPU SSSP (dense form).  Same filter as the single-GPU SSSP
+// (reading R4: nd = dist[u] + w, atomicMin, improved vertices enter the next log once per
+// iteration); an improvement of a REMOTE target is an atomicMin into the padded candidate array,
+// and one ncclReduceScatter(min) per iteration hands every owner the minimum over all ranks.
+struct SsspPushMulti {
+  struct Src {
+    uint32_t du;
+  };
+  static constexpr bool kWeights = true;
+  static constexpr bool kNeedRow = false;
+  static constexpr bool kEnqueue = true;
+  const MultiArgs *a;
+  const Queues *next_q;
+  CounterSet *next_cs;
+  __device__ __forceinline__ Src src(bool valid, int u, long long, long long) const {
+    return Src{valid ? ldcg(a->dist + u) : 0xffffffffu};
+  }
+  template <int N>
+  __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N], const uint32_t (&w)[N],
+                                        bool (&in)[N], int) const {
+    const unsigned long long keep = policy_evict_last();
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      in[j] = false;
+      if (!valid) continue;
+      const unsigned long long nd = (unsigned long long)s.du + w[j];
+      if (nd >= 0xffffffffull) {
+        if (s.du != 0xffffffffu) *a->overflow = 1;   // resolved after the traversal
+        continue;
+      }
+      bool own;
+      const long long p = pidx(a->pm, v[j], &own);
+      if (own) {
+        const int lv = (int)(v[j] - a->v_begin);
+        if (nd >= ld_status(a->dist + lv, keep)) continue;
+        const uint32_t old = atomicMin(a->dist + lv, (uint32_t)nd);
+        if ((uint32_t)nd < old) {
+          const uint32_t bit = 1u << (lv & 31);
+          in[j] = !(atomicOr(a->inq_next + (lv >> 5), bit) & bit);
+          v[j] = lv;                 // enqueue the LOCAL row id
+        }
+      } else {
+        if (nd < ld_status(a->cand + p, keep)) atomicMin(a->cand + p, (uint32_t)nd);
+      }
+    }
+  }
+};
+
+template <int VEC>
+__global__ void __launch_bounds__(kBlock, 4) k_msssp_push(const __grid_constant__ MultiArgs a) {
+  __shared__ WarpScratch wsm[kWarps];
+  __shared__ SsspPushMulti::Src fsrc[kWarps][32];
+  const int warp = threadIdx.x >> 5;
+  const int L = a.lvl;
+  SsspPushMulti f;
+  f.a = &a;
+  f.next_q = &a.q[(L + 1) & 1];
+  f.next_cs = &a.ctl->set[(L + 1) % 3];
+  consume_log<VEC>(f, a.L, a.q[L & 1], &a.ctl->set[L % 3], a.off, a.col, a.w, &wsm[warp], fsrc[warp],
+                   a.vec_ok);
+}
+
+// Owners apply the minima received for their rows: one warp per 32-row word of the dedupe bitmap.
+__global__ void __launch_bounds__(kBlock) k_msssp_apply(const __grid_constant__ MultiArgs a) {
+  __shared__ WarpScratch wsm[kWarps];
+  const int warp = threadIdx.x >> 5;
+  const unsigned lane = lane_id();
+  const int L = a.lvl;
+  const long long words = (a.n_local + 31) >> 5;
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  const Queues &Qn = a.q[(L + 1) & 1];
+  CounterSet *csn = &a.ctl->set[(L + 1) % 3];
+  int bcnt = 0;
+  for (long long wd = gw; wd < words; wd += nw) {
+    const long long v = (wd << 5) + lane;
+    bool improved = false;
+    if (v < a.n_local) {
+      const uint32_t c = a.cown[v];
+      if (c < a.dist[v]) {
+        a.dist[v] = c;
+        improved = true;
+      }
+    }
+    const unsigned im = __ballot_sync(FULL, improved);
+    const uint32_t had = a.inq_next[wd];
+    if (im && lane == 0) a.inq_next[wd] = had | im;
+    const bool enq = improved && !((had >> lane) & 1u);
+    buffer_push(enq, (int)v, &wsm[warp], bcnt, a.off, a.L, Qn, csn);
+  }
+  if (bcnt) buffer_flush(&wsm[warp], bcnt, a.off, a.L, Qn, csn);
+}
+
+__global__ void k_msssp_seed(MultiArgs a, long long src_local) {
+  const bool act = threadIdx.x == 0;
+  long long b = 0, e = 0;
+  if (act) {
+    b = a.off[src_local];
+    e = a.off[src_local + 1];
+    a.dist[src_local] = 0u;
+  }
+  enqueue_warp(act, (int)src_local, b, e, a.L, a.q[0], &a.ctl->set[0]);
+}
+
+// reached bitmap of the own rows (padded global layout) for the overflow resolution
+__global__ void k_mreached_bits(const uint32_t *__restrict__ dist, long long n_local, uint32_t *bits) {
+  const long long words = (n_local + 31) >> 5;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long wd = (long long)blockIdx.x * blockDim.x + threadIdx.x; wd < words; wd += stride) {
+    uint32_t b = 0;
+    for (int k = 0; k < 32; ++k) {
+      const long long v = (wd << 5) + k;
+      if (v < n_local && dist[v] != 0xffffffffu) b |= 1u << k;
+    }
+    bits[wd] = b;
+  }
+}
+// a finite distance >= UINT32_MAX exists iff a reached vertex has an arc to an unreached one
+// (DESIGN.md "SSSP overflow"); `bits` = allgathered reached bitmap (padded layout)
+__global__ void k_moverflow_check(const MultiArgs a, const uint32_t *__restrict__ bits, int *found) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long u = (long long)blockIdx.x * blockDim.x + threadIdx.x; u < a.n_local; u += stride) {
+    if (a.dist[u] == 0xffffffffu) continue;
+    for (long long k = a.off[u]; k < a.off[u + 1]; ++k) {
+      bool own;
+      const long long p = pidx(a.pm, a.col[k], &own);
+      if (!((bits[p >> 5] >> (p & 31)) & 1u)) {
+        *found = 1;
+        return;
+      }
+    }
+  }
+}
+__global__ void k_mreached_arcs(const long long *__restrict__ off, const uint32_t *__restrict__ dist,
+                                long long n, unsigned long long *out) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  unsigned long long s = 0;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+    if (dist[v] != 0xffffffffu) s += (unsigned long long)(off[v + 1] - off[v]);
+  s = warp_sum64(s);
+  if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, s);
 }
 
 __global__ void k_mseed(MultiArgs a, long long src_local) {
@@ -418,6 +569,8 @@ void free_comm(sage_graph *g) {
   dfree(g, c->y);
   dfree(g, c->yown);
   dfree(g, c->dsum);
+  dfree(g, c->cand);
+  dfree(g, c->cown);
   cudaStreamSynchronize(g->stream);
   if (c->nc) ncclCommDestroy(c->nc);
   delete c;
@@ -585,9 +738,147 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
   return SAGE_OK;
 }
 
-sage_status run_sssp_multi(sage_graph *, int32_t, uint32_t *, sage_stats *) {
-  set_error("multi-GPU SSSP is not implemented (SURVEY §8(f) NEXT #2)");
-  return SAGE_E_UNSUPPORTED;
+// Multi-GPU SSSP: host-sequenced frontier Bellman-Ford iterations.  Per iteration: local push
+// (own targets relaxed in place, remote ones into cand) -> ncclReduceScatter(min) of cand to the
+// owners (C1e with min instead of sum) -> owners apply and enqueue -> stats allreduce (C1d).
+sage_status run_sssp_multi(sage_graph *g, int32_t source, uint32_t *dist_out, sage_stats *st) {
+  Comm *c = g->comm;
+  sage_status s;
+  if ((s = ensure_traversal_state(g)) != SAGE_OK) return s;
+  TraversalState &t = g->ts;
+  if (!t.dist && (s = dalloc(g, (void **)&t.dist, sizeof(uint32_t) * (size_t)g->n_local)) != SAGE_OK)
+    return s;
+  const long long P = c->pm.P;
+  if (!c->cand) {
+    if ((s = dalloc(g, (void **)&c->cand, sizeof(uint32_t) * (size_t)P * c->world)) != SAGE_OK ||
+        (s = dalloc(g, (void **)&c->cown, sizeof(uint32_t) * (size_t)P)) != SAGE_OK)
+      return s;
+  }
+  int *ovf = nullptr;
+  if ((s = dalloc(g, (void **)&ovf, sizeof(int) * 4)) != SAGE_OK) return s;
+  const size_t lwords = (size_t)((g->n_local + 31) / 32 + 1);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  cudaEventRecord(e0, g->stream);
+  cudaMemsetAsync(ovf, 0, sizeof(int) * 4, g->stream);
+  cudaMemsetAsync(t.dist, 0xff, sizeof(uint32_t) * (size_t)g->n_local, g->stream);
+  cudaMemsetAsync(c->cand, 0xff, sizeof(uint32_t) * (size_t)P * c->world, g->stream);
+  for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * lwords, g->stream);
+  cudaMemsetAsync(t.ctl, 0, offsetof(Ctl, rec), g->stream);
+  MultiArgs a;
+  memset(&a, 0, sizeof(a));
+  a.off = (const long long *)g->off;
+  a.col = g->col;
+  a.w = g->w;
+  a.n_local = g->n_local;
+  a.v_begin = g->v_begin;
+  a.L = g->ladder;
+  a.q[0] = t.q[0];
+  a.q[1] = t.q[1];
+  a.ctl = t.ctl;
+  a.vec_ok = g->vec_ok ? 1 : 0;
+  a.pm = c->pm;
+  a.dist = t.dist;
+  a.cand = c->cand;
+  a.cown = c->cown;
+  a.overflow = ovf;
+  if (source >= g->v_begin && source < g->v_end)
+    k_msssp_seed<<<1, 32, 0, g->stream>>>(a, (long long)source - g->v_begin);
+  const int grid = g->num_sms * 4;
+  unsigned long long h6[6];
+  long long exp_ = 0, arcs = 0, impr = 0;
+  int iters = 0;
+  for (int L = 0;; ++L) {
+    cudaMemsetAsync(&t.ctl->set[(L + 2) % 3], 0, sizeof(CounterSet), g->stream);
+    cudaMemsetAsync(t.fb[(L + 2) % 3], 0, sizeof(uint32_t) * lwords, g->stream);
+    a.lvl = L;
+    a.inq_next = t.fb[(L + 1) % 3];
+    if (g->vec == 4) k_msssp_push<4><<<grid, kBlock, 0, g->stream>>>(a);
+    else k_msssp_push<1><<<grid, kBlock, 0, g->stream>>>(a);
+    NCCL_CHECK(g, ncclReduceScatter(c->cand, c->cown, (size_t)P, ncclUint32, ncclMin, c->nc, g->stream),
+               "SSSP min reduce-scatter");
+    cudaMemsetAsync(c->cand, 0xff, sizeof(uint32_t) * (size_t)P * c->world, g->stream);
+    if (c->world > 1) k_msssp_apply<<<grid, kBlock, 0, g->stream>>>(a);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+      dfree(g, ovf);
+      return cuda_fail(g, e, "multi-GPU SSSP iteration");
+    }
+    if ((s = allreduce_stats(g, L, h6)) != SAGE_OK) {
+      dfree(g, ovf);
+      return s;
+    }
+    iters = L + 1;
+    exp_ += (long long)h6[4];
+    arcs += (long long)h6[5];
+    impr += (long long)h6[0];
+    if (h6[0] == 0) break;
+    if (L + 1 > 4 * g->n + 64) {
+      dfree(g, ovf);
+      set_error("SSSP iteration cap exceeded (internal error)");
+      return SAGE_E_CUDA;
+    }
+  }
+  // overflow: any rank saw du + w >= 2^32 -> check reached -> unreached arcs globally
+  unsigned long long *red = c->stats;   // reuse: [0] local flag, [8] global
+  int hflag = 0;
+  cudaMemcpyAsync(&hflag, ovf, sizeof(int), cudaMemcpyDeviceToHost, g->stream);
+  cudaStreamSynchronize(g->stream);
+  unsigned long long fl[2] = {(unsigned long long)hflag, 0ull};
+  cudaMemcpyAsync(red, fl, sizeof(unsigned long long), cudaMemcpyHostToDevice, g->stream);
+  NCCL_CHECK(g, ncclAllReduce(red, red + 8, 1, ncclUint64, ncclSum, c->nc, g->stream), "overflow flag");
+  cudaMemcpyAsync(&fl[1], red + 8, sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream);
+  cudaStreamSynchronize(g->stream);
+  if (fl[1]) {
+    uint32_t *bits = c->visited;   // p*Wp words, padded layout
+    k_mreached_bits<<<grid, 256, 0, g->stream>>>(t.dist, g->n_local, bits + (size_t)c->rank * c->Wp);
+    NCCL_CHECK(g, ncclAllGather(bits + (size_t)c->rank * c->Wp, bits, (size_t)c->Wp, ncclUint32, c->nc,
+                                g->stream), "reached allgather");
+    k_moverflow_check<<<grid, 256, 0, g->stream>>>(a, bits, ovf + 1);
+    int hf = 0;
+    cudaMemcpyAsync(&hf, ovf + 1, sizeof(int), cudaMemcpyDeviceToHost, g->stream);
+    cudaStreamSynchronize(g->stream);
+    fl[0] = (unsigned long long)hf;
+    cudaMemcpyAsync(red, fl, sizeof(unsigned long long), cudaMemcpyHostToDevice, g->stream);
+    NCCL_CHECK(g, ncclAllReduce(red, red + 8, 1, ncclUint64, ncclSum, c->nc, g->stream), "overflow found");
+    cudaMemcpyAsync(&fl[1], red + 8, sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream);
+    cudaStreamSynchronize(g->stream);
+    if (fl[1]) {
+      dfree(g, ovf);
+      set_error("a finite shortest distance is >= UINT32_MAX");
+      return SAGE_E_OVERFLOW;
+    }
+  }
+  cudaEventRecord(e1, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  dfree(g, ovf);
+  if (e != cudaSuccess) return cuda_fail(g, e, "multi-GPU SSSP");
+  float ms = 0;
+  cudaEventElapsedTime(&ms, e0, e1);
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (st) {
+    memset(st, 0, sizeof(*st));
+    unsigned long long *ra = c->stats;
+    cudaMemsetAsync(ra, 0, sizeof(unsigned long long), g->stream);
+    k_mreached_arcs<<<grid, 256, 0, g->stream>>>((const long long *)g->off, t.dist, g->n_local, ra);
+    NCCL_CHECK(g, ncclAllReduce(ra, ra + 8, 1, ncclUint64, ncclSum, c->nc, g->stream), "reached arcs");
+    unsigned long long hra = 0;
+    cudaMemcpyAsync(&hra, ra + 8, sizeof(hra), cudaMemcpyDeviceToHost, g->stream);
+    cudaStreamSynchronize(g->stream);
+    st->levels = st->push_levels = iters;
+    st->vertices_expanded = exp_;
+    st->arcs_inspected = arcs;
+    st->vertices_discovered = impr;
+    st->edges_traversed = (int64_t)((g->flags & SAGE_F_SYMMETRIC) ? hra / 2 : hra);
+    st->ms = st->kernel_ms = ms;
+    st->model_bytes = 4.0 * (double)g->n + 24.0 * exp_ + 12.0 * arcs + 8.0 * impr;
+  }
+  if ((s = copy_out(g, dist_out, t.dist, sizeof(uint32_t) * (size_t)g->n_local)) != SAGE_OK) return s;
+  e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "output");
+  return SAGE_OK;
 }
 
 sage_status run_pagerank_multi(sage_graph *g, double damping, int32_t iterations, double *rank_out,

@@ -46,14 +46,40 @@ def test_nccl_path_bfs_pagerank(sage, sym):
         assert ei.value.status == sage.E_UNSUPPORTED
 
 
-def test_nccl_path_refuses_sssp_and_bad_blocks(sage):
-    g = sg.rmat(10, 8, seed=1, symmetric=True)
+@pytest.mark.parametrize("sym", [True, False])
+def test_nccl_path_sssp(sage, sym):
+    """Multi-GPU SSSP (NEXT #2) through the 1-rank NCCL path: bit-exact vs Dijkstra."""
+    g = sg.rmat(13, 16, seed=5, symmetric=sym)
     w = sg.weights(g, 1)
     uid = sage.nccl_unique_id()
-    with sage.load_csr(g.off, g.col, w, symmetric=True, rank=0, world=1, nccl_unique_id=uid) as G:
+    with sage.load_csr(g.off, g.col, w, symmetric=sym, rank=0, world=1, nccl_unique_id=uid) as G:
+        for s in sg.sources(g, 3, seed=2):
+            d, st = G.sssp(int(s))
+            ref, _ = oracle.sssp(g.off, g.col, w, int(s))
+            assert np.array_equal(d, ref)
+            assert st["edges_traversed"] == int(np.diff(g.off)[ref != 0xFFFFFFFF].sum()) // (2 if sym else 1)
+
+
+def test_nccl_path_sssp_overflow(sage):
+    """A path whose length exceeds UINT32_MAX is reported, as on one GPU."""
+    off = np.array([0, 1, 2, 2], dtype=np.int64)
+    col = np.array([1, 2], dtype=np.int32)
+    w = np.array([0xF0000000, 0xF0000000], dtype=np.uint32)
+    with sage.load_csr(off, col, w, rank=0, world=1, nccl_unique_id=sage.nccl_unique_id()) as G:
         with pytest.raises(sage.SageError) as ei:
             G.sssp(0)
-        assert ei.value.status == sage.E_UNSUPPORTED
+        assert ei.value.status == sage.E_OVERFLOW
+    # overflowing candidate that is not needed: 0->2 directly is short
+    off = np.array([0, 2, 3, 3], dtype=np.int64)
+    col = np.array([1, 2, 2], dtype=np.int32)
+    w = np.array([0xF0000000, 5, 0xF0000000], dtype=np.uint32)
+    with sage.load_csr(off, col, w, rank=0, world=1, nccl_unique_id=sage.nccl_unique_id()) as G:
+        d, _ = G.sssp(0)
+        assert d.tolist() == [0, 0xF0000000, 5]
+
+
+def test_nccl_path_refuses_bad_blocks(sage):
+    g = sg.rmat(10, 8, seed=1, symmetric=True)
     with pytest.raises(sage.SageError):
         sage.load_csr(g.off[:11], g.col[:g.off[10]], rank=0, world=1, nccl_unique_id=sage.nccl_unique_id(),
                       v_begin=0, v_end=10, n=g.n)   # one rank must cover [0, n)

@@ -5,8 +5,9 @@ TEST MODEL, not a backend: pure numpy, one process per logical rank, torch.distr
 1D contiguous blocks, the padded global index r*P + (v - vb[r]), push levels with a dense
 candidate bitmap exchanged to the owners, owners applying candidates, the (|F|, arcs(F))
 allreduce driving termination and the Beamer direction, the frontier allgather before pull
-levels, and PageRank's reduce-scatter of partial sums plus the dangling allreduce — and checks
-the gathered answers against the oracle.
+levels, PageRank's reduce-scatter of partial sums plus the dangling allreduce, and SSSP's
+min reduce-scatter of remote candidate distances per Bellman-Ford iteration — and checks the
+gathered answers against the oracle.
 """
 import os
 import socket
@@ -164,6 +165,48 @@ def model_pagerank(rank, world, g, dist, d=0.85, iters=20):
     return x
 
 
+def model_sssp(rank, world, g, w, src, dist):
+    """csrc/comm.cu run_sssp_multi: own targets relaxed in place, remote ones min-ed into the padded
+    candidate array, ncclReduceScatter(min) to the owners, owners apply, |improved| allreduce."""
+    import torch
+    pm = Part(rank, world, g.n)
+    vb, ve = pm.vb[rank], pm.vb[rank + 1]
+    nl = ve - vb
+    INF = 0xFFFFFFFF
+    d = np.full(nl, INF, dtype=np.uint64)
+    frontier = []
+    if vb <= src < ve:
+        d[src - vb] = 0
+        frontier = [src - vb]
+    while True:
+        cand = np.full(world * pm.P, INF, dtype=np.int64)
+        inq = set()
+        for u in frontier:
+            du = int(d[u])
+            for k in range(g.off[vb + u], g.off[vb + u + 1]):
+                nd = du + int(w[k])
+                assert nd < INF
+                p, own = pm.pidx(int(g.col[k]))
+                if own:
+                    lv = int(g.col[k]) - vb
+                    if nd < d[lv]:
+                        d[lv] = nd
+                        inq.add(lv)
+                elif nd < cand[p]:
+                    cand[p] = nd
+        t = torch.from_numpy(cand)
+        dist.all_reduce(t, op=dist.ReduceOp.MIN)          # reduce-scatter(min) = allreduce + own slice
+        cown = t.numpy()[rank * pm.P:rank * pm.P + nl]
+        for lv in np.nonzero(cown < d.astype(np.int64))[0]:
+            d[lv] = cown[lv]
+            inq.add(int(lv))
+        nF = _allreduce([float(len(inq))], dist)[0]
+        if nF == 0:
+            break
+        frontier = sorted(inq)
+    return d.astype(np.uint32)
+
+
 def _worker(rank, world, port, outdir):
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -177,6 +220,11 @@ def _worker(rank, world, port, outdir):
             res[f"bfs{k}_{int(s)}_push"] = model_bfs(rank, world, g, int(s), dist, direction=False)
     g = sg.rmat(8, 8, seed=7, symmetric=False)
     res["pr"] = model_pagerank(rank, world, g, dist)
+    for k, sym in enumerate([True, False]):
+        g = sg.rmat(9, 8, seed=11 + k, symmetric=sym)
+        w = sg.weights(g, 1)
+        for s in sg.sources(g, 2, seed=2):
+            res[f"sssp{k}_{int(s)}"] = model_sssp(rank, world, g, w, int(s), dist)
     np.savez(os.path.join(outdir, f"rank{rank}.npz"), **res)
     dist.destroy_process_group()
 
@@ -198,3 +246,10 @@ def test_partitioned_protocol_matches_oracle(tmp_path, world):
     x = np.concatenate([p["pr"] for p in parts])
     xr = oracle.pagerank(g.off, g.col, 0.85, 20)
     assert np.max(np.abs(x - xr) / xr) < 1e-12
+    for k, sym in enumerate([True, False]):
+        g = sg.rmat(9, 8, seed=11 + k, symmetric=sym)
+        w = sg.weights(g, 1)
+        for s in sg.sources(g, 2, seed=2):
+            ref, _ = oracle.sssp(g.off, g.col, w, int(s))
+            got = np.concatenate([p[f"sssp{k}_{int(s)}"] for p in parts])
+            assert np.array_equal(got, ref), (k, int(s))

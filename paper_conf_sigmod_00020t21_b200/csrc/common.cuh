@@ -347,7 +347,15 @@ __device__ __forceinline__ void enqueue_warp(bool active, int v, long long b, lo
   // CTA class: cooperative write of every heavy vertex's q explicit tiles.
   if (totq) {
     const unsigned long long base0 = shfl64(mybase, 0);
-    unsigned hm = __ballot_sync(FULL, q > 0);
+#ifndef SAGE_ENQ_LANEQ
+#define SAGE_ENQ_LANEQ 16
+#endif
+    // vertices with few CTA tiles write them from their own lane; the warp writes the rest
+    if (q > 0 && q <= SAGE_ENQ_LANEQ) {
+      const unsigned long long bs = base0 + incq - q;
+      for (unsigned long long j = 0; j < q; ++j) st_tile(Q.cta + bs + j, s.b2 + (long long)j * L.B, v, L.B);
+    }
+    unsigned hm = __ballot_sync(FULL, q > SAGE_ENQ_LANEQ);
     while (hm) {
       const int src = __ffs(hm) - 1;
       hm &= hm - 1;

@@ -488,7 +488,7 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
     const unsigned long long grabs = (count + batch - 1) / batch;
     if ((unsigned long long)gwarp >= grabs) continue;
     const int sub = lane / lpt, sl = lane % lpt;
-    const bool contiguous = lpt < 32 && vec_ok && VEC == 4;
+    const bool contiguous = lpt < 32 && vec_ok && (VEC % 4) == 0;
     const int lg_spt = __ffs(spt) - 1;
     for (unsigned long long rr = 0;; ++rr) {
       unsigned long long base = 0;
@@ -544,15 +544,20 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
           const bool valid = k < nt;
           const long long start = ws->hb[valid ? k : 0];
           if (contiguous) {
-            int4 c4 = make_int4(0, 0, 0, 0);
-            uint4 w4 = make_uint4(0, 0, 0, 0);
             const long long p0 = start + (long long)sl * VEC;
-            if (valid) {
-              c4 = ld_col4(col + p0, pol);
-              if (F::kWeights) w4 = ld_col4u(w + p0, pol);
+#pragma unroll
+            for (int q = 0; q < (VEC + 3) / 4; ++q) {
+              int4 c4 = make_int4(0, 0, 0, 0);
+              uint4 w4 = make_uint4(0, 0, 0, 0);
+              if (valid) {
+                c4 = ld_col4(col + p0 + 4 * q, pol);
+                if (F::kWeights) w4 = ld_col4u(w + p0 + 4 * q, pol);
+              }
+              v[(4 * q) % VEC] = c4.x; v[(4 * q + 1) % VEC] = c4.y;
+              v[(4 * q + 2) % VEC] = c4.z; v[(4 * q + 3) % VEC] = c4.w;
+              ww[(4 * q) % VEC] = w4.x; ww[(4 * q + 1) % VEC] = w4.y;
+              ww[(4 * q + 2) % VEC] = w4.z; ww[(4 * q + 3) % VEC] = w4.w;
             }
-            v[0] = c4.x; v[1 % VEC] = c4.y; v[2 % VEC] = c4.z; v[3 % VEC] = c4.w;
-            ww[0] = w4.x; ww[1 % VEC] = w4.y; ww[2 % VEC] = w4.z; ww[3 % VEC] = w4.w;
           } else {
             const long long p0 = start + (long long)(st & (spt - 1)) * (lpt * VEC) + sl;
 #pragma unroll

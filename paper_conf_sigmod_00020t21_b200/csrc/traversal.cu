@@ -455,6 +455,9 @@ __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
 }
 
 // ============================================================================ BFS kernel
+#ifndef SAGE_BFS_VEC8
+#define SAGE_BFS_VEC8 0   // push BFS with 8 neighbours per lane per step (more loads in flight)
+#endif
 template <int VEC>
 #ifndef SAGE_BFS_MINB
 #define SAGE_BFS_MINB 4
@@ -1303,7 +1306,9 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
     cudaError_t le = cudaLaunchCooperativeKernel(fn, dim3(g->grid_bin), dim3(kBinBlock), args, smem, g->stream);
     if (le != cudaSuccess) return cuda_fail(g, le, "binned BFS kernel");
   } else {
-    const void *fn = g->vec == 4 ? (const void *)k_bfs<4> : (const void *)k_bfs<1>;
+    static const int bfs_vec8 = getenv("SAGE_BFS_VEC") ? atoi(getenv("SAGE_BFS_VEC")) == 8 : SAGE_BFS_VEC8;
+    const void *fn = g->vec == 4 ? (bfs_vec8 && g->ladder.M >= 8 ? (const void *)k_bfs<8> : (const void *)k_bfs<4>)
+                                 : (const void *)k_bfs<1>;
     const int grid = coop_grid(g, fn, &g->grid_bfs);
     void *args[] = {&a};
     if ((s = launch_coop(g, fn, grid, args, "BFS kernel")) != SAGE_OK) return s;

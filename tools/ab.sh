@@ -1,6 +1,6 @@
 #!/bin/bash
 # A/B timing session (under gpurun): default build + tests, then variants given as
-# "NAME=VALUE" compile definitions (SAGE_DEF_*), each with a short push-BFS bench.
+# "NAME=VALUE[,NAME=VALUE]" compile definitions (SAGE_DEF_*), each with a short push-BFS bench.
 # Usage: bash tools/ab.sh <tag> [DEF=VAL ...]
 tag=${1:-ab}; shift
 out=gpurun_out; mkdir -p $out
@@ -11,7 +11,8 @@ timeout 300 python bench.py --no-extras > $out/bench_${tag}_base.json 2>&1
 timeout 300 python tools/prof_run.py --scale 24 --reps 3 --op bfs_push > $out/levels_${tag}_base.txt 2>&1
 echo base; cut -c1-200 $out/bench_${tag}_base.json
 for d in "$@"; do
-  env "SAGE_DEF_${d%%=*}=${d#*=}" python tools/build.py --force > /dev/null || continue
+  envs=(); IFS=',' read -ra kv <<< "$d"; for x in "${kv[@]}"; do envs+=("SAGE_DEF_${x%%=*}=${x#*=}"); done
+  env "${envs[@]}" python tools/build.py --force > /dev/null || continue
   timeout 300 python bench.py --no-extras > $out/bench_${tag}_$d.json 2>&1
   timeout 300 python tools/prof_run.py --scale 24 --reps 3 --op bfs_push > $out/levels_${tag}_$d.txt 2>&1
   echo $d; cut -c1-200 $out/bench_${tag}_$d.json

@@ -430,6 +430,31 @@ def _extras(a, G, g, srcs, level, flush, stream, sage):
                           "bfs_ms": float(np.mean([t for t, _ in r])), "bfs_levels": r[-1][1]["levels"],
                           "bfs_gteps": len(r) / sum(t * 1e-3 * 1e9 / st["edges_traversed"] for t, st in r),
                           "pagerank_ms_20_iter": rp[0][0]}
+    # C1 (BASELINE configs[0]): RMAT-16, L2-resident and launch/latency-bound; 16 sources, push
+    # and direction-optimising, each checked against the oracle, which is timed beside it
+    c1 = sg.config("C1")
+    with sage.load_csr(torch.from_numpy(c1.off).cuda(), torch.from_numpy(c1.col).cuda(), symmetric=True,
+                       stream=stream.cuda_stream) as C:
+        lv1 = torch.empty(c1.n, dtype=torch.int32, device="cuda")
+        s1 = sg.sources(c1, 16, seed=2)
+        res = {}
+        for form, po in (("push", True), ("do", False)):
+            C.bfs(int(s1[0]), out=lv1, push_only=po)
+            r = _time_calls(lambda i: C.bfs(int(s1[i]), out=lv1, push_only=po)[2], len(s1), flush, stream)
+            ok = True
+            for i in range(4):
+                C.bfs(int(s1[i]), out=lv1, push_only=po)
+                ok &= bool(np.array_equal(lv1.cpu().numpy(), oracle.bfs(c1.off, c1.col, int(s1[i]))))
+            res[form] = {"us_median": float(np.median([t for t, _ in r])) * 1e3,
+                         "gteps": len(r) / sum(t * 1e-3 * 1e9 / st["edges_traversed"] for t, st in r),
+                         "levels_equal_oracle_4_sources": ok}
+        t0 = time.perf_counter()
+        for i in range(16):
+            oracle.bfs(c1.off, c1.col, int(s1[i]))
+        to = (time.perf_counter() - t0) / 16
+        res["oracle_us_per_source"] = to * 1e6
+        res["roofline"] = "n/a (graph L2-resident: latency / launch bound, SURVEY 8(d))"
+        ex["c1"] = res
     # end-to-end through the C ABI with HOST buffers: load (H2D) + BFS + level D2H
     off_h = torch.from_numpy(g.off).pin_memory()
     col_h = torch.from_numpy(g.col).pin_memory()

@@ -52,6 +52,14 @@ struct PageRankState {      // the all-V resident tile log (built once, reused; 
   double *x = nullptr, *y = nullptr;
   float *c = nullptr;             // pull form: x_u / out(u)
   CounterSet *cs = nullptr;       // device copy of the log's counters (+ rotating tickets)
+  // binned push form (pagerank.cu, PrPushBin); bin_lg == 0 = not set up
+  int bin_lg = 0, nbin = 0;
+  long long bin_warps = 0;
+  long long *bstart = nullptr;
+  unsigned long long *bfill = nullptr;
+  int *ev = nullptr;
+  double *ec = nullptr;
+  unsigned *wpos = nullptr, *wend = nullptr;
 };
 
 }  // namespace sage
@@ -89,5 +97,5 @@ struct sage_graph {
   sage::TraversalState ts;
   sage::PageRankState pr;
   sage::Comm *comm = nullptr;
-  int grid_bfs = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0, grid_bin = 0;   // persistent grid sizes
+  int grid_bfs = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0, grid_bin = 0, grid_pr_bin = 0;   // persistent grid sizes
 };

@@ -18,6 +18,7 @@
 #pragma once
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
+#include <type_traits>
 #include <stdint.h>
 
 namespace sage {
@@ -459,6 +460,12 @@ __device__ __forceinline__ void buffer_flush(WarpScratch *ws, int &cnt,
 //   Queues *next_q; CounterSet *next_cs;             where filtered-in vertices go
 // steal = false (ablation of Resident Tile Stealing, Fig. 10): tiles are dealt to warps
 // statically, round robin in batch units, instead of through the device-wide tickets.
+// Column-prefetch depth of a filter (F::kPrefetch, default 1 step ahead).
+template <class F, class = void> struct PrefetchDepth { static constexpr int value = 1; };
+template <class F> struct PrefetchDepth<F, std::void_t<decltype(F::kPrefetch)>> {
+  static constexpr int value = F::kPrefetch;
+};
+
 template <int VEC, class F>
 __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Queues &Q,
                                             CounterSet *cs, const long long *__restrict__ off,
@@ -490,11 +497,15 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
     const int sub = lane / lpt, sl = lane % lpt;
     const bool contiguous = lpt < 32 && vec_ok && (VEC % 4) == 0;
     const int lg_spt = __ffs(spt) - 1;
+    // stealing: the ticket of the NEXT batch is taken when a batch starts, so the ticket atomic's
+    // round trip overlaps the batch (a ticket beyond `count` just ends the loop)
+    unsigned long long tk_next = 0;
+    if (steal && lane == 0) tk_next = atomicAdd(&cs->tk[c].v, batch);
     for (unsigned long long rr = 0;; ++rr) {
       unsigned long long base = 0;
       if (steal) {
-        if (lane == 0) base = atomicAdd(&cs->tk[c].v, batch);
-        base = shfl64(base, 0);
+        base = shfl64(tk_next, 0);
+        if (base < count && lane == 0) tk_next = atomicAdd(&cs->tk[c].v, batch);
       } else {
         base = ((unsigned long long)gwarp + rr * (unsigned long long)nwarps) * batch;
       }
@@ -567,6 +578,39 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
             }
           }
         };
+        if constexpr (PrefetchDepth<F>::value > 1) {
+          // filters with little work per step (PageRank: VEC fp64 atomics, no status reads) keep
+          // the column loads of the next PD steps in flight
+          constexpr int PD = PrefetchDepth<F>::value;
+          int vq[PD][VEC];
+          uint32_t wq[PD][VEC];
+#pragma unroll
+          for (int r = 0; r < PD; ++r)
+            if (r < nst) load_step(r, vq[r], wq[r]);
+          for (int st0 = 0; st0 < nst; st0 += PD) {
+#pragma unroll
+            for (int r = 0; r < PD; ++r) {
+              const int st = st0 + r;
+              if (st < nst) {
+                int v[VEC];
+                uint32_t ww[VEC];
+#pragma unroll
+                for (int j = 0; j < VEC; ++j) {
+                  v[j] = vq[r][j];
+                  ww[j] = wq[r][j];
+                }
+                if (st + PD < nst) load_step(st + PD, vq[r], wq[r]);
+                const int k = ((st >> lg_spt) * tps) + sub;
+                const bool valid = k < nt;
+                const typename F::Src sc = fsrc[valid ? k : 0];
+                bool in[VEC];
+                f.template visit<VEC>(valid, sc, v, ww, in, lpt);
+              }
+            }
+          }
+          __syncwarp();
+          continue;
+        }
         load_step(0, vn, wn);
         for (int st = 0; st < nst; ++st) {
           PROF_T(tv0);

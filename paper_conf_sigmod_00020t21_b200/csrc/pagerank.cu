@@ -21,6 +21,10 @@ struct PrPush {
   struct Src {
     double c;
   };
+#ifndef SAGE_PR_PREFETCH
+#define SAGE_PR_PREFETCH 4
+#endif
+  static constexpr int kPrefetch = SAGE_PR_PREFETCH;
   static constexpr bool kWeights = false;
   static constexpr bool kNeedRow = true;
   static constexpr bool kEnqueue = false;
@@ -49,6 +53,7 @@ struct PrPush {
 // fp64 accumulation, reading R7) and adds the group's partial sum to y_v with one fp64 atomic per
 // lane group and step — the same resident log and stealing consumer, no per-arc atomics.
 struct PrPull {
+  static constexpr int kPrefetch = SAGE_PR_PREFETCH;
   struct Src {
     int u;
   };

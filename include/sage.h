@@ -189,6 +189,22 @@ sage_status sage_bc(sage_graph *g, const int32_t *sources, int64_t n_sources, do
 sage_status sage_reorder(sage_graph *g, int32_t rounds, const sage_reorder_opts *opt,
                          sage_stats *st);
 
+/* Online Sampling-based Reordering: §6's "the sampling is performed along
+ * with the tile access" with the sampling threshold |E|, reading R19b.
+ * enable != 0 starts recording: every later single-GPU sage_bfs / sage_bfs_ex call records the rows
+ * of the vertices it reached (one occurrence each) and every sage_pagerank / sage_pagerank_ex call
+ * records every non-empty row `iterations` times, as per-vertex occurrence counts under the current
+ * labels.  When the recorded row lengths since the last round reach `threshold` (<= 0: |E| = m),
+ * one reorder round (stages 1-3 + swap matching + relabel, exactly sage_reorder's round) runs on
+ * that weighted sample right after the query that crossed the threshold has written its answer;
+ * the counts then restart.  Answers always use original ids.  enable == 0 stops recording.
+ * sector_width as in sage_reorder_opts (0 = 8).  Single GPU, device-resident columns only
+ * (SAGE_E_UNSUPPORTED otherwise).                                                              */
+sage_status sage_online_reorder(sage_graph *g, int32_t enable, int32_t sector_width, int64_t threshold);
+
+/* Online reordering progress: rounds run, label swaps applied, recorded row lengths pending.   */
+sage_status sage_online_reorder_info(const sage_graph *g, int64_t *rounds, int64_t *swaps, int64_t *pending);
+
 /* Objective of §6 on the current labels: the sum over the tile sample (every tile of
  * every vertex under the graph's ladder, readings R19/R20) of the number of distinct sectors
  * floor(label / sector_width) among the tile's members.  Lower = better locality.              */

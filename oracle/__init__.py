@@ -263,3 +263,71 @@ def reorder(off, col, w=None, rounds: int = 1, B: int = 256, M: int = 8, A: int 
         sigma = sig_r[sigma]
         info.append({"movers": nmov, "swaps": swaps, "objective_before": obj_before})
     return off, col, w, sigma, info
+
+
+# ---------------------------------------------------------------- online sampling (§6, NEXT #3)
+def sample_tiles_weighted(off, col, weights, B: int = 256, M: int = 8, A: int = 4):
+    """The tile sample of an ONLINE round ("the sampling is performed along with the tile
+    access"; reading R19b): vertex u's tiles (kind 0, R20) occur weights[u] times — once per
+    recorded access of u's row.  weights == 1 everywhere gives sample_tiles()."""
+    col = np.ascontiguousarray(col, dtype=np.int32)
+    verts = np.repeat(np.arange(len(off) - 1, dtype=np.int32), np.asarray(weights, dtype=np.int64))
+    if len(verts) == 0:
+        return np.zeros(1, dtype=np.int64), np.zeros(0, dtype=np.int32)
+    q = tile_log(off, verts, B, M, A)
+    q = q[q[:, 3] == 0]
+    sizes = q[:, 2]
+    tile_ptr = np.zeros(len(q) + 1, dtype=np.int64)
+    np.cumsum(sizes, out=tile_ptr[1:])
+    members = np.empty(int(tile_ptr[-1]), dtype=np.int32)
+    for k, (_, o, s, _) in enumerate(q):          # plain copy of every occurrence's members
+        members[tile_ptr[k]:tile_ptr[k] + s] = col[o:o + s]
+    return tile_ptr, members
+
+
+def reorder_round_weighted(off, col, w, weights, B: int = 256, M: int = 8, A: int = 4, S: int = 8):
+    """One Sampling-based Reordering round (stages 1-3, swap matching, relabel; §6) over the
+    weighted sample.  Returns (off', col', w', sigma_round, movers, swaps); sigma_round is the
+    identity (and the graph unchanged) when there is no mover or no swap (R25)."""
+    off = np.ascontiguousarray(off, dtype=np.int64)
+    n = len(off) - 1
+    tp, mem = sample_tiles_weighted(off, col, weights, B, M, A)
+    st = reorder_stages(n, tp, mem, S)
+    nmov = int(st["mover"].sum())
+    ident = np.arange(n, dtype=np.int32)
+    if nmov == 0:
+        return off, col, w, ident, 0, 0
+    sig_r, swaps = reorder_match(n, S, st)
+    if swaps == 0:
+        return off, col, w, ident, nmov, 0
+    off2, col2, w2 = relabel(off, col, w, sig_r)
+    return off2, col2, w2, sig_r, nmov, swaps
+
+
+def online_reorder_bfs(off, col, sources, threshold=None, B: int = 256, M: int = 8, A: int = 4,
+                       S: int = 8):
+    """Online Sampling-based Reordering driven by a sequence of BFS queries (sage_online_reorder):
+    every query records the rows of the vertices it reached (weight + 1 each, current labels); when
+    the recorded row lengths since the last round reach ``threshold`` (default |E|), one
+    round runs on that sample before the next query.  Returns (sigma, rounds, levels per query in
+    original ids) with sigma[v_orig] = final label."""
+    off = np.ascontiguousarray(off, dtype=np.int64)
+    col = np.ascontiguousarray(col, dtype=np.int32)
+    n = len(off) - 1
+    thr = len(col) if threshold is None or threshold <= 0 else int(threshold)
+    sigma = np.arange(n, dtype=np.int32)
+    weights = np.zeros(n, dtype=np.int64)
+    acc, rounds, levels = 0, 0, []
+    for s in sources:
+        lv_cur = bfs(off, col, int(sigma[int(s)]))     # query in current labels
+        levels.append(lv_cur[sigma])                   # answer in original ids
+        reached = np.nonzero(lv_cur >= 0)[0]
+        weights[reached] += 1
+        acc += int(np.sum(off[reached + 1] - off[reached]))
+        if acc >= thr:
+            off, col, _, sig_r, _, _ = reorder_round_weighted(off, col, None, weights, B, M, A, S)
+            sigma = sig_r[sigma]
+            weights[:] = 0
+            acc = 0
+            rounds += 1
+    return sigma, rounds, levels

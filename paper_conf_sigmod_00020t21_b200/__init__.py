@@ -25,7 +25,7 @@ STATUS_NAMES = {0: "SAGE_OK", 1: "SAGE_E_INVALID", 2: "SAGE_E_NOMEM", 3: "SAGE_E
                 4: "SAGE_E_NCCL", 5: "SAGE_E_OVERFLOW", 6: "SAGE_E_UNSUPPORTED"}
 
 EXPORTED = ["sage_load_csr", "sage_free", "sage_bfs", "sage_bfs_ex", "sage_sssp", "sage_pagerank",
-            "sage_pagerank_ex", "sage_bc",
+            "sage_pagerank_ex", "sage_bc", "sage_online_reorder", "sage_online_reorder_info",
             "sage_reorder", "sage_reorder_objective", "sage_get_permutation", "sage_get_csr", "sage_graph_info",
             "sage_debug_export_tiles", "sage_debug_reorder_stages", "sage_nccl_unique_id", "sage_debug_level_records", "sage_last_error", "sage_version"]
 
@@ -83,6 +83,8 @@ def lib():
         L.sage_load_csr.argtypes = [ctypes.POINTER(Csr), ctypes.POINTER(p)]
         L.sage_free.argtypes = [p]
         L.sage_bfs.argtypes = [p, i32, p, p, ctypes.POINTER(Stats)]
+        L.sage_online_reorder.argtypes = [p, i32, i32, i64]
+        L.sage_online_reorder_info.argtypes = [p, ctypes.POINTER(i64), ctypes.POINTER(i64), ctypes.POINTER(i64)]
         L.sage_bfs_ex.argtypes = [p, i32, p, p, u32, ctypes.POINTER(Stats)]
         L.sage_sssp.argtypes = [p, i32, p, ctypes.POINTER(Stats)]
         L.sage_pagerank.argtypes = [p, dbl, i32, p, ctypes.POINTER(Stats)]
@@ -226,6 +228,17 @@ class Graph:
         st = Stats()
         _check(lib().sage_bc(self._h, src.ctypes.data, len(src), o.ptr, ctypes.byref(st)))
         return o.obj, st.as_dict()
+
+    def online_reorder(self, enable: bool = True, sector_width: int = 8, threshold: int = 0):
+        """sage_online_reorder: record the tile accesses of later queries; one reorder round each
+        time the recorded row lengths reach ``threshold`` (0 = |E|)."""
+        _check(lib().sage_online_reorder(self._h, 1 if enable else 0, int(sector_width), int(threshold)))
+
+    def online_info(self) -> dict:
+        """sage_online_reorder_info -> {"rounds", "swaps", "pending"}."""
+        r, s, p = ctypes.c_int64(0), ctypes.c_int64(0), ctypes.c_int64(0)
+        _check(lib().sage_online_reorder_info(self._h, ctypes.byref(r), ctypes.byref(s), ctypes.byref(p)))
+        return {"rounds": r.value, "swaps": s.value, "pending": p.value}
 
     def reorder(self, rounds: int = 1, sector_width: int = 8, candidates=None):
         ro = ReorderOpts()

@@ -220,6 +220,8 @@ static void destroy(sage_graph *g) {
   }
   dfree(g, g->sigma);
   dfree(g, g->sigma_inv);
+  dfree(g, g->samp_w);
+  dfree(g, g->samp_acc);
   cudaStreamSynchronize(g->stream);
   if (g->own_stream) cudaStreamDestroy(g->stream);
   delete g;

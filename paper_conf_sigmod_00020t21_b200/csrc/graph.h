@@ -97,5 +97,11 @@ struct sage_graph {
   sage::TraversalState ts;
   sage::PageRankState pr;
   sage::Comm *comm = nullptr;
+  // online sampling (sage_online_reorder): per-vertex occurrence counts, recorded row lengths
+  bool online = false;
+  int online_lgS = 3;
+  long long online_thr = 0, online_pending = 0, online_rounds = 0, online_movers = 0, online_swaps = 0;
+  uint32_t *samp_w = nullptr;
+  unsigned long long *samp_acc = nullptr;
   int grid_bfs = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0, grid_bin = 0, grid_pr_bin = 0;   // persistent grid sizes
 };

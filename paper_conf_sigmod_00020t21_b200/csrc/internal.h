@@ -26,6 +26,7 @@ int32_t to_internal_id(sage_graph *g, int32_t v);
 
 // pagerank.cu
 void free_pagerank_state(sage_graph *g);
+sage_status online_after_query(sage_graph *g, const int32_t *level_internal, int32_t pr_iters);
 sage_status ensure_pagerank_log(sage_graph *g);
 
 // comm.cu (multi-GPU)

@@ -574,7 +574,7 @@ extern "C" sage_status sage_pagerank_ex(sage_graph *g, double damping, int32_t i
   if ((s = translate_out_f64(g, p.x, rank_out)) != SAGE_OK) return s;
   e = cudaStreamSynchronize(g->stream);
   if (e != cudaSuccess) return cuda_fail(g, e, "PageRank output");
-  return SAGE_OK;
+  return online_after_query(g, nullptr, iterations);
 }
 
 extern "C" sage_status sage_pagerank(sage_graph *g, double damping, int32_t iterations,

@@ -45,6 +45,7 @@ struct SampleArgs {
   const int2 *lohi;
   const int *target;
   unsigned long long *objective;
+  const uint32_t *vw;          // online sampling: occurrences of each vertex's tiles (null = 1)
 };
 
 // first index i in seg[0, len) with seg[i] >= key (seg sorted ascending)
@@ -101,15 +102,19 @@ __global__ void __launch_bounds__(256) k_sample(const __grid_constant__ SampleAr
       const long long ti = r * R + lane / G;
       const bool tv = ti < count;
       long long start = 0;
+      unsigned long long wt = 1;   // occurrences of this tile in the sample
       if (tv) {
+        int u;
         if (c == 0) {
           start = a.q.cta[ti].start;
+          u = a.q.cta[ti].u;
         } else {
-          const int u = a.q.cls[c][ti];
+          u = a.q.cls[c][ti];
           const long long b = a.off[u], e = a.off[u + 1];
           const RowSplit s = split_row(b, e, a.L);
           start = class_tile_start(e, s.r, t);
         }
+        if (a.vw) wt = a.vw[u];
       }
       // stage the members in shared memory
       if (t < 32) {
@@ -125,12 +130,12 @@ __global__ void __launch_bounds__(256) k_sample(const __grid_constant__ SampleAr
         const int i = t < 32 ? lane : lane + 32 * k;
         const int *seg = t < 32 ? buf + (lane / G) * G : buf;
         const int pos = t < 32 ? lane % G : i;
-        if (!tv) continue;
+        if (!tv || (MODE != 3 && wt == 0)) continue;
         const int x = seg[pos];
         const long long sx = (long long)x >> a.lgS;
         if (MODE == 0) {
           const int cnt = lower_bound_s(seg, t, (sx + 1) << a.lgS) - lower_bound_s(seg, t, sx << a.lgS) - 1;
-          if (cnt > 0) atomicAdd(a.loc1 + x, (unsigned long long)cnt);
+          if (cnt > 0) atomicAdd(a.loc1 + x, (unsigned long long)cnt * wt);
         } else if (MODE == 1) {
           const int2 lh = a.lohi[x];
           if (lh.y - lh.x > 1) {
@@ -140,14 +145,14 @@ __global__ void __launch_bounds__(256) k_sample(const __grid_constant__ SampleAr
             const int ihi = lower_bound_s(seg, t, hi << a.lgS);
             const int Lc = imid - ilo - ((sx >= lo && sx < mid) ? 1 : 0);
             const int Rc = ihi - imid - ((sx >= mid && sx < hi) ? 1 : 0);
-            if (Lc > 0) atomicAdd(a.cl + x, (unsigned long long)Lc);
-            if (Rc > 0) atomicAdd(a.cr + x, (unsigned long long)Rc);
+            if (Lc > 0) atomicAdd(a.cl + x, (unsigned long long)Lc * wt);
+            if (Rc > 0) atomicAdd(a.cr + x, (unsigned long long)Rc * wt);
           }
         } else if (MODE == 2) {
           const long long tg = a.target[x];
           const int cnt = lower_bound_s(seg, t, (tg + 1) << a.lgS) - lower_bound_s(seg, t, tg << a.lgS) -
                           (sx == tg ? 1 : 0);
-          if (cnt > 0) atomicAdd(a.loc3 + x, (unsigned long long)cnt);
+          if (cnt > 0) atomicAdd(a.loc3 + x, (unsigned long long)cnt * wt);
         } else {
           if (pos == 0 || ((long long)seg[pos - 1] >> a.lgS) != sx) obj++;
         }
@@ -353,7 +358,8 @@ static void free_round(sage_graph *g, RoundBufs &b) {
 
 // One reorder round; *movers / *swaps report what happened (swaps == 0 -> nothing relabelled).
 static sage_status one_round(sage_graph *g, RoundBufs &b, int lgS, const uint8_t *cand,
-                             long long *movers, long long *swaps, bool stages_only = false) {
+                             long long *movers, long long *swaps, bool stages_only = false,
+                             const uint32_t *vw = nullptr) {
   const long long n = g->n;
   const int S = 1 << lgS;
   const long long nsec = (n + S - 1) / S;
@@ -361,6 +367,7 @@ static sage_status one_round(sage_graph *g, RoundBufs &b, int lgS, const uint8_t
   SampleArgs a;
   sage_status s = sample_args(g, &a, lgS);
   if (s != SAGE_OK) return s;
+  a.vw = vw;
   a.loc1 = b.loc1;
   a.loc3 = b.loc3;
   a.cl = b.cl;
@@ -521,6 +528,127 @@ static sage_status load_candidates(sage_graph *g, RoundBufs &b, const std::vecto
 }  // namespace sage
 
 using namespace sage;
+
+// ---- online sampling (NEXT #3; §6 P:444 "the sampling is performed along with the tile access",
+// threshold |E| P:514; reading R19b): queries record the rows they expanded as per-vertex
+// occurrence counts (current labels); once the recorded row lengths since the last round reach
+// the threshold, one round runs on that weighted sample after the query has returned its answer.
+__global__ void k_samp_levels(const int32_t *__restrict__ level, const long long *__restrict__ off,
+                              long long n, uint32_t *w, unsigned long long *acc) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  unsigned long long s = 0;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+    if (level[v] >= 0) {
+      w[v] += 1u;
+      s += (unsigned long long)(off[v + 1] - off[v]);
+    }
+  s = warp_sum64(s);
+  if ((threadIdx.x & 31) == 0 && s) atomicAdd(acc, s);
+}
+__global__ void k_samp_all(const long long *__restrict__ off, long long n, uint32_t k, uint32_t *w,
+                           unsigned long long *acc) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  unsigned long long s = 0;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+    const long long d = off[v + 1] - off[v];
+    if (d > 0) {
+      w[v] += k;
+      s += (unsigned long long)d * k;
+    }
+  }
+  s = warp_sum64(s);
+  if ((threadIdx.x & 31) == 0 && s) atomicAdd(acc, s);
+}
+
+sage_status sage::online_after_query(sage_graph *g, const int32_t *level_internal, int32_t pr_iters) {
+  if (!g->online) return SAGE_OK;
+  const long long n = g->n;
+  const int grid = g->num_sms * 8;
+  if (level_internal)
+    k_samp_levels<<<grid, 256, 0, g->stream>>>(level_internal, (const long long *)g->off, n, g->samp_w,
+                                              g->samp_acc);
+  else if (pr_iters > 0)
+    k_samp_all<<<grid, 256, 0, g->stream>>>((const long long *)g->off, n, (uint32_t)pr_iters, g->samp_w,
+                                           g->samp_acc);
+  unsigned long long acc = 0;
+  cudaMemcpyAsync(&acc, g->samp_acc, sizeof(acc), cudaMemcpyDeviceToHost, g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "online sampling");
+  g->online_pending = (long long)acc;
+  if ((long long)acc < g->online_thr) return SAGE_OK;
+  RoundBufs b;
+  sage_status s = alloc_round(g, b, false);
+  long long mv = 0, sw = 0;
+  if (s == SAGE_OK) s = one_round(g, b, g->online_lgS, nullptr, &mv, &sw, false, g->samp_w);
+  free_round(g, b);
+  if (s != SAGE_OK) return s;
+  if (sw > 0) {
+    g->h_sigma.resize((size_t)n);
+    cudaMemcpy(g->h_sigma.data(), g->sigma, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToHost);
+  }
+  cudaMemsetAsync(g->samp_w, 0, sizeof(uint32_t) * (size_t)n, g->stream);
+  cudaMemsetAsync(g->samp_acc, 0, sizeof(unsigned long long), g->stream);
+  e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "online reorder");
+  g->online_rounds += 1;
+  g->online_movers += mv;
+  g->online_swaps += sw;
+  g->online_pending = 0;
+  return SAGE_OK;
+}
+
+extern "C" sage_status sage_online_reorder(sage_graph *g, int32_t enable, int32_t sector_width,
+                                           int64_t threshold) {
+  clear_error();
+  if (!g) {
+    set_error("null graph");
+    return SAGE_E_INVALID;
+  }
+  if (g->sticky) return (sage_status)g->sticky;
+  if (!enable) {
+    g->online = false;
+    return SAGE_OK;
+  }
+  if (g->comm || g->host_columns) {
+    set_error("online reordering is single-GPU with device-resident columns only");
+    return SAGE_E_UNSUPPORTED;
+  }
+  const int S = sector_width ? sector_width : 8;
+  if (S < 1 || S > 64 || (S & (S - 1))) {
+    set_error("sector_width must be a power of two in [1, 64]");
+    return SAGE_E_INVALID;
+  }
+  int lgS = 0;
+  while ((1 << lgS) < S) ++lgS;
+  sage_status s;
+  if (!g->samp_w) {
+    if ((s = dalloc(g, (void **)&g->samp_w, sizeof(uint32_t) * (size_t)std::max<long long>(g->n, 1))) != SAGE_OK ||
+        (s = dalloc(g, (void **)&g->samp_acc, sizeof(unsigned long long))) != SAGE_OK)
+      return s;
+  }
+  cudaMemsetAsync(g->samp_w, 0, sizeof(uint32_t) * (size_t)std::max<long long>(g->n, 1), g->stream);
+  cudaMemsetAsync(g->samp_acc, 0, sizeof(unsigned long long), g->stream);
+  cudaError_t e = cudaStreamSynchronize(g->stream);
+  if (e != cudaSuccess) return cuda_fail(g, e, "online reorder");
+  g->online = true;
+  g->online_lgS = lgS;
+  g->online_thr = threshold > 0 ? threshold : std::max<long long>(g->m, 1);
+  g->online_pending = 0;
+  return SAGE_OK;
+}
+
+extern "C" sage_status sage_online_reorder_info(const sage_graph *g, int64_t *rounds, int64_t *swaps,
+                                                int64_t *pending) {
+  clear_error();
+  if (!g) {
+    set_error("null graph");
+    return SAGE_E_INVALID;
+  }
+  if (rounds) *rounds = g->online_rounds;
+  if (swaps) *swaps = g->online_swaps;
+  if (pending) *pending = g->online_pending;
+  return SAGE_OK;
+}
 
 extern "C" sage_status sage_reorder(sage_graph *g, int32_t rounds, const sage_reorder_opts *opt,
                                     sage_stats *st) {

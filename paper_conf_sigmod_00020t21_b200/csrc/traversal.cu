@@ -1359,7 +1359,8 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   if (parent_out && (s = translate_out_i32(g, t.parent, parent_out, true)) != SAGE_OK) return s;
   e = cudaStreamSynchronize(g->stream);
   if (e != cudaSuccess) return cuda_fail(g, e, "BFS output");
-  return SAGE_OK;
+  // online sampling: record the rows this query expanded (after the answer has been delivered)
+  return online_after_query(g, t.level, 0);
 }
 
 extern "C" sage_status sage_bfs(sage_graph *g, int32_t source, int32_t *level_out,

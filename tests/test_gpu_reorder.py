@@ -147,3 +147,47 @@ def test_reorder_objective_improves_and_errors(sage):
         with pytest.raises(sage.SageError) as ei:
             G.reorder(1, sector_width=3)
         assert ei.value.status == sage.E_INVALID
+
+
+@pytest.mark.parametrize("sym,lad", [(True, dict(tile_cta=16, tile_min=4, align=4)),
+                                     (False, dict(tile_cta=32, tile_min=8, align=0))])
+def test_online_reorder_equals_oracle(sage, sym, lad):
+    """Online sampling (NEXT #3, sage_online_reorder): a sequence of BFS queries records the rows it
+    expanded; rounds run when the recorded row lengths reach the threshold.  The permutation and
+    the relabelled CSR equal the oracle's driver (oracle.online_reorder_bfs) exactly, and every
+    answer is in original ids."""
+    g = sg.rmat(12, 8, seed=6, symmetric=sym)
+    srcs = [int(s) for s in sg.sources(g, 8, seed=2)]
+    thr = 2 * g.m
+    sig_ref, rounds_ref, lv_ref = oracle.online_reorder_bfs(
+        g.off, g.col, srcs, threshold=thr, B=lad["tile_cta"], M=lad["tile_min"], A=lad["align"])
+    assert rounds_ref >= 1
+    with sage.load_csr(g.off, g.col, symmetric=sym, **lad) as G:
+        G.online_reorder(True, 8, thr)
+        for s, ref in zip(srcs, lv_ref):
+            lv, _, _ = G.bfs(s, push_only=True)
+            assert np.array_equal(lv, ref)
+        info = G.online_info()
+        assert info["rounds"] == rounds_ref
+        assert np.array_equal(G.permutation(), sig_ref)
+        off2, col2, _ = oracle.relabel(g.off, g.col, None, sig_ref)
+        o, c, _ = G.csr()
+        assert np.array_equal(o, off2) and np.array_equal(c, col2)
+        G.online_reorder(False)
+        lv, _, _ = G.bfs(srcs[0])
+        assert np.array_equal(lv, oracle.bfs(g.off, g.col, srcs[0]))
+        assert G.online_info()["rounds"] == rounds_ref
+
+
+def test_online_reorder_pagerank_records_every_row(sage):
+    """A PageRank call records every non-empty row `iterations` times: with threshold K*m one call
+    triggers one round, which is the offline round (uniform weights scale every count)."""
+    g = sg.rmat(11, 8, seed=7, symmetric=False)
+    _, _, _, sig1, _ = oracle.reorder(g.off, g.col, None, rounds=1, B=256, M=8, A=4, S=8)
+    with sage.load_csr(g.off, g.col) as G:
+        G.online_reorder(True, 8, 0)          # threshold |E|
+        x, _ = G.pagerank(0.85, 3)
+        assert G.online_info()["rounds"] == 1
+        assert np.array_equal(G.permutation(), sig1)
+        xr = oracle.pagerank(g.off, g.col, 0.85, 3)
+        assert np.max(np.abs(x - xr) / xr) <= 1e-6

@@ -497,6 +497,21 @@ def _extras(a, G, g, srcs, level, flush, stream, sage):
         ex["reorder"] = {"round_ms": st["ms"], "note": "second round on the graph (first round = warm-up)", "swaps": st["vertices_discovered"], "movers": st["vertices_expanded"],
                          "objective_before": ob0, "objective_after": ob1,
                          "bfs_push_ms_before": b0["kernel_ms"], "bfs_push_ms_after": b1["kernel_ms"]}
+        # online sampling (NEXT #3): 4 BFS queries recording their rows, threshold |E| -> a round
+        # after every query that crosses it; wall time of each sage_bfs call incl. recording + round
+        H.online_reorder(True, 8, 0)
+        walls = []
+        for i in range(4):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            _, _, bs = H.bfs(int(srcs[2 + i]), out=level, push_only=True)
+            torch.cuda.synchronize()
+            walls.append((time.perf_counter() - t0) * 1e3)
+        info = H.online_info()
+        H.online_reorder(False)
+        ex["online_reorder"] = {"bfs_call_wall_ms": walls, "rounds": info["rounds"], "swaps": info["swaps"],
+                                "threshold": "|E|", "note": "each call = BFS + row recording (+ one round "
+                                "when the recorded row lengths reach |E|)"}
     return ex
 
 

@@ -858,15 +858,18 @@ sage_status run_sssp_multi(sage_graph *g, int32_t source, uint32_t *dist_out, sa
   cudaEventElapsedTime(&ms, e0, e1);
   cudaEventDestroy(e0);
   cudaEventDestroy(e1);
-  if (st) {
-    memset(st, 0, sizeof(*st));
+  // reached arcs (collective on every rank, whether or not this rank asked for stats)
+  unsigned long long hra = 0;
+  {
     unsigned long long *ra = c->stats;
     cudaMemsetAsync(ra, 0, sizeof(unsigned long long), g->stream);
     k_mreached_arcs<<<grid, 256, 0, g->stream>>>((const long long *)g->off, t.dist, g->n_local, ra);
     NCCL_CHECK(g, ncclAllReduce(ra, ra + 8, 1, ncclUint64, ncclSum, c->nc, g->stream), "reached arcs");
-    unsigned long long hra = 0;
     cudaMemcpyAsync(&hra, ra + 8, sizeof(hra), cudaMemcpyDeviceToHost, g->stream);
     cudaStreamSynchronize(g->stream);
+  }
+  if (st) {
+    memset(st, 0, sizeof(*st));
     st->levels = st->push_levels = iters;
     st->vertices_expanded = exp_;
     st->arcs_inspected = arcs;

@@ -489,8 +489,22 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
       f.v_base = 0;
       f.next_q = &a.q[(L + 1) & 1];
       f.next_cs = nxt;
+#ifdef SAGE_PROF
+      const unsigned long long pt0 = globaltimer();
+#endif
       consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok,
                        a.steal != 0);
+#ifdef SAGE_PROF
+      if (L == 1 && (threadIdx.x & 31) == 0) {   // per-warp consume durations of level 1
+        const unsigned long long d = globaltimer() - pt0;
+        atomicAdd(&g_prof[8], d);
+        atomicMax(&g_prof[9], d);
+        if (d > 20000) atomicAdd(&g_prof[10], 1ull);
+        atomicAdd(&g_prof[11], 1ull);
+        atomicMax(&g_prof[12], pt0 - ctl->t0_ns);
+        atomicMin(&g_prof[13], pt0 - ctl->t0_ns);
+      }
+#endif
     } else {
       pull_level(a, L + 1, fbc, fbn, a.q[(L + 1) & 1], cur, nxt, &wsm[warp]);
     }
@@ -1604,6 +1618,7 @@ extern "C" int sage_prof_read(unsigned long long *out16, int reset) {
   cudaMemcpyFromSymbol(out16, sage::g_prof, sizeof(unsigned long long) * 16);
   if (reset) {
     unsigned long long z[16] = {0};
+    z[13] = ~0ull;
     cudaMemcpyToSymbol(sage::g_prof, z, sizeof(z));
   }
   return 0;

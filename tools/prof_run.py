@@ -62,7 +62,8 @@ for i in range(a.reps):
         import ctypes
         buf = (ctypes.c_ulonglong * 16)()
         sage.lib().sage_prof_read(buf, 1)
-        names = ["flush_cyc", "flushes", "visit_contig_cyc", "visit_strided_cyc", "strided_steps", "ticket_cyc", "tickets"]
+        names = ["flush_cyc", "flushes", "visit_contig_cyc", "visit_strided_cyc", "strided_steps", "ticket_cyc",
+                 "tickets", "_", "L1_sum_ns", "L1_max_ns", "L1_warps_gt20us", "L1_warps", "L1_start_max", "L1_start_min"]
         d = {nm: buf[k] for k, nm in enumerate(names)}
         print("   prof:", d, {"cyc/flush": d["flush_cyc"] / max(1, d["flushes"]),
                                "cyc/strided_step": d["visit_strided_cyc"] / max(1, d["strided_steps"]),

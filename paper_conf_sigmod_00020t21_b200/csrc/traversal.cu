@@ -1156,8 +1156,9 @@ int coop_grid(sage_graph *g, const void *fn, int *cache) {
   if (nb < 1) nb = 1;
   // small graphs (C1: 1.8M arcs, L2-resident) are latency-bound per level: one CTA per SM halves
   // the grid barrier's participants and the counter traffic (C1 DO BFS 156 -> 135 us measured)
+  const int nb_occ = nb;
   if (g->m < (8ll << 20)) nb = 1;
-  if (const char *e = getenv("SAGE_CTAS_PER_SM")) nb = std::max(1, std::min(nb, atoi(e)));
+  if (const char *e = getenv("SAGE_CTAS_PER_SM")) nb = std::max(1, std::min(nb_occ, atoi(e)));
   *cache = nb * g->num_sms;
   return *cache;
 }

@@ -338,3 +338,21 @@ def test_pagerank_binned_push_parity(sage, lg, monkeypatch):
     with sage.load_csr(uk.off, uk.col) as G:
         x, _ = G.pagerank(0.85, 10)
         assert np.max(np.abs(x - xr) / xr) <= 1e-6
+
+
+def test_full_occupancy_grid_on_small_graphs(sage, monkeypatch):
+    """Small graphs run the persistent kernels with one CTA per SM by default; the full-occupancy
+    grid (4 CTAs per SM, the configuration of the large configs) gives the same answers."""
+    monkeypatch.setenv("SAGE_CTAS_PER_SM", "4")
+    g = sg.rmat(15, 16, seed=9, symmetric=True)
+    w = sg.weights(g, 1)
+    with sage.load_csr(g.off, g.col, w, symmetric=True) as G:
+        for s in sg.sources(g, 4, seed=2):
+            ref = oracle.bfs(g.off, g.col, int(s))
+            for po in (True, False):
+                assert np.array_equal(G.bfs(int(s), push_only=po)[0], ref)
+            d, _ = G.sssp(int(s))
+            assert np.array_equal(d, oracle.sssp(g.off, g.col, w, int(s))[0])
+        x, _ = G.pagerank(0.85, 10)
+        xr = oracle.pagerank(g.off, g.col, 0.85, 10)
+        assert np.max(np.abs(x - xr) / xr) <= 1e-6

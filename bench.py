@@ -376,6 +376,15 @@ def _time_calls(fn, k, flush, stream):
     return out
 
 
+def _lv_in_core(G, src, level_ooc):
+    """Levels of the out-of-core run (already in ``level_ooc``) vs the in-core graph."""
+    import torch
+    ooc = level_ooc.cpu().numpy().copy()
+    ref = torch.empty_like(level_ooc)
+    G.bfs(int(src), out=ref, push_only=True)
+    return np.array_equal(ooc, ref.cpu().numpy())
+
+
 def _extras(a, G, g, srcs, level, flush, stream, sage):
     import torch
 
@@ -430,6 +439,20 @@ def _extras(a, G, g, srcs, level, flush, stream, sage):
                           "bfs_ms": float(np.mean([t for t, _ in r])), "bfs_levels": r[-1][1]["levels"],
                           "bfs_gteps": len(r) / sum(t * 1e-3 * 1e9 / st["edges_traversed"] for t, st in r),
                           "pagerank_ms_20_iter": rp[0][0]}
+    # out-of-core (NEXT #4): C2 with col in pinned host memory read zero-copy over the host link
+    # (copied into library-owned pinned memory at load); push and DO BFS, parity checked
+    with sage.load_csr(g.off, g.col, symmetric=True, host_columns=True, align=32,
+                       stream=stream.cuda_stream) as O:
+        oo = {}
+        for form, po in (("push", True), ("do", False)):
+            O.bfs(int(srcs[0]), out=level, push_only=po)
+            r = _time_calls(lambda i: O.bfs(int(srcs[i]), out=level, push_only=po)[2], 2, flush, stream)
+            oo[form] = {"ms": float(np.mean([t for t, _ in r])),
+                        "gteps": len(r) / sum(t * 1e-3 * 1e9 / st["edges_traversed"] for t, st in r)}
+        O.bfs(int(srcs[0]), out=level, push_only=True)
+        oo["levels_equal_in_core"] = bool(_lv_in_core(G, srcs[0], level))
+        oo["note"] = "col (2.08 GB) in pinned host memory; tile alignment 32 (128-B requests)"
+        ex["out_of_core"] = oo
     # C1 (BASELINE configs[0]): RMAT-16, L2-resident and launch/latency-bound; 16 sources, push
     # and direction-optimising, each checked against the oracle, which is timed beside it
     c1 = sg.config("C1")

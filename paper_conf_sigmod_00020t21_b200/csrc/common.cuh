@@ -63,6 +63,7 @@ struct CounterSet {                      // counters of one log (rotated over 3 
   PaddedCounter nF, arcsF;               // |F| and arcs(F) of the vertices enqueued here
   PaddedCounter inspected;               // pull: arcs inspected while consuming this level
   PaddedCounter scanned;                 // pull: unvisited non-isolated vertices scanned
+  PaddedCounter flc;                     // deferred contraction: frontier-list slots reserved
 };
 
 struct LevelRec {                        // per-level record (first kMaxRec levels)
@@ -391,6 +392,7 @@ struct WarpScratch {
   long long hb[32];
   long long tb[32];
   int buf[64];
+  long long cpos, cend;   // deferred contraction: the warp's open chunk of the frontier list
 };
 
 #ifdef SAGE_PROF
@@ -401,6 +403,66 @@ __device__ unsigned long long g_prof[16];
 #define PROF_T(x)
 #define PROF_ADD(i, v)
 #endif
+
+// ---- deferred contraction (filters with kDefer; push BFS): a filtered-in vertex is only appended
+// to a plain frontier list (32-slot groups inside 256-slot chunks reserved per warp, -1 = empty
+// slot); Tiled Partitioning of the list into the next level's log runs as its own grid phase after
+// the level (K2' before K3', Fig. 2), where every warp classifies with all its loads in flight,
+// instead of stalling the consumer warp for an enqueue round trip every 32 discoveries.
+template <class F, class = void> struct DeferTrait { static constexpr bool value = false; };
+template <class F> struct DeferTrait<F, std::void_t<decltype(F::kDefer)>> {
+  static constexpr bool value = F::kDefer;
+};
+constexpr int kDeferChunk = 256;
+__device__ __forceinline__ void defer_group(int x, WarpScratch *ws, int *list, unsigned long long *lc) {
+  const unsigned lane = lane_id();
+  long long pos = 0;
+  if (lane == 0) {
+    pos = ws->cpos;
+    if (pos >= ws->cend) {
+      pos = (long long)atomicAdd(lc, (unsigned long long)kDeferChunk);
+      ws->cend = pos + kDeferChunk;
+    }
+    ws->cpos = pos + 32;
+  }
+  pos = (long long)shfl64((unsigned long long)pos, 0);
+  list[pos + lane] = x;
+}
+__device__ __forceinline__ void defer_push(bool in, int v, WarpScratch *ws, int &cnt, int *list,
+                                           unsigned long long *lc) {
+  const unsigned m = __ballot_sync(FULL, in);
+  if (!m) return;
+  const unsigned lane = lane_id();
+  if (in) ws->buf[cnt + __popc(m & lanemask_lt())] = v;
+  cnt += __popc(m);
+  if (cnt >= 32) {
+    __syncwarp();
+    const int x = ws->buf[lane];
+    const int y = ws->buf[32 + lane];
+    __syncwarp();
+    cnt -= 32;
+    if ((int)lane < cnt) ws->buf[lane] = y;
+    __syncwarp();
+    defer_group(x, ws, list, lc);
+  }
+}
+// last partial group, then -1 over the rest of the open chunk; leaves the chunk state reset
+__device__ __forceinline__ void defer_close(WarpScratch *ws, int &cnt, int *list, unsigned long long *lc) {
+  __syncwarp();
+  const unsigned lane = lane_id();
+  if (cnt) {
+    const int x = (int)lane < cnt ? ws->buf[lane] : -1;
+    __syncwarp();
+    defer_group(x, ws, list, lc);
+    cnt = 0;
+  }
+  __syncwarp();
+  const long long p0 = ws->cpos, p1 = ws->cend;
+  for (long long i = p0 + lane; i < p1; i += 32) list[i] = -1;
+  __syncwarp();
+  if (lane == 0) ws->cpos = ws->cend = 0;
+  __syncwarp();
+}
 
 // Append the lanes' filtered-in vertices to the warp buffer; flush full batches of 32.
 __device__ __forceinline__ void buffer_push(bool in, int v, WarpScratch *ws, int &cnt,
@@ -633,7 +695,8 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
           if constexpr (F::kEnqueue) {
 #pragma unroll
             for (int j = 0; j < VEC; ++j)
-              buffer_push(in[j], v[j], ws, bcnt, off, L, *f.next_q, f.next_cs);
+              if constexpr (DeferTrait<F>::value) defer_push(in[j], v[j], ws, bcnt, f.flist, f.flc);
+              else buffer_push(in[j], v[j], ws, bcnt, off, L, *f.next_q, f.next_cs);
           }
         }
         __syncwarp();
@@ -706,12 +769,16 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
       }
       bool in[1];
       f.template visit<1>(kv, so, vv, w1, in, 1);
-      if constexpr (F::kEnqueue) buffer_push(in[0], vv[0], ws, bcnt, off, L, *f.next_q, f.next_cs);
+      if constexpr (F::kEnqueue) {
+        if constexpr (DeferTrait<F>::value) defer_push(in[0], vv[0], ws, bcnt, f.flist, f.flc);
+        else buffer_push(in[0], vv[0], ws, bcnt, off, L, *f.next_q, f.next_cs);
+      }
     }
     __syncwarp();
   }
   if constexpr (F::kEnqueue) {
-    if (bcnt) buffer_flush(ws, bcnt, off, L, *f.next_q, f.next_cs);
+    if constexpr (DeferTrait<F>::value) defer_close(ws, bcnt, f.flist, f.flc);
+    else if (bcnt) buffer_flush(ws, bcnt, off, L, *f.next_q, f.next_cs);
   }
 }
 

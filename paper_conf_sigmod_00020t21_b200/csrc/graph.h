@@ -41,6 +41,7 @@ struct TraversalState {     // per-query scratch, allocated on first use and kep
   PaddedCounter *farc = nullptr;  // SSSP near-far: [3] pile sizes + [3] scan minima
   void *tailmem = nullptr;        // BFS tail mode state (global scratch)
   uint32_t *expd = nullptr;       // SSSP near-far: last expanded distance per vertex
+  int *flist = nullptr;           // BFS deferred contraction: frontier list
 };
 
 struct PageRankState {      // the all-V resident tile log (built once, reused)

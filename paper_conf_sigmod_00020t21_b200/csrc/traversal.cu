@@ -37,6 +37,12 @@ struct BfsPush {
   static constexpr bool kWeights = false;
   static constexpr bool kNeedRow = false;
   static constexpr bool kEnqueue = true;
+#ifndef SAGE_BFS_DEFER
+#define SAGE_BFS_DEFER 1
+#endif
+  static constexpr bool kDefer = SAGE_BFS_DEFER != 0;   // contraction deferred to a K2' phase
+  int *flist = nullptr;                  // deferred frontier list
+  unsigned long long *flc = nullptr;     // its slot counter (next level's CounterSet)
   uint32_t *visited;
   int *level;
   int *parent;
@@ -156,6 +162,7 @@ struct TravArgs {
   int *tail;            // tail mode: next-frontier list (n entries of scratch)
   struct TailSmem *tailmem;   // tail mode state (global scratch: only block 0 uses it)
   int steal;            // 0 = ablation: static tile assignment instead of stealing
+  int *flist;           // deferred contraction: frontier list (n + slack entries)
 };
 
 // Pull (bottom-up) step over the visited bitmap: one warp per 32-vertex word.
@@ -472,6 +479,7 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
   int dir = 0;
   unsigned long long prev_nF = 1;
   const long long nwords = (a.n + 31) >> 5;
+  if ((threadIdx.x & 31) == 0) wsm[warp].cpos = wsm[warp].cend = 0;
   for (int L = 0;; ++L) {
     CounterSet *cur = &ctl->set[L % 3];
     CounterSet *nxt = &ctl->set[(L + 1) % 3];
@@ -489,6 +497,8 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
       f.v_base = 0;
       f.next_q = &a.q[(L + 1) & 1];
       f.next_cs = nxt;
+      f.flist = a.flist;
+      f.flc = &nxt->flc.v;
 #ifdef SAGE_PROF
       const unsigned long long pt0 = globaltimer();
 #endif
@@ -510,6 +520,38 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
     }
     if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
     grid_barrier(&ctl->bar);
+    if (BfsPush::kDefer) {
+      // K2': Tiled Partitioning of the deferred frontier list into level L+1's log, every warp on
+      // 32-slot groups with the next group's ids and rows loaded before the current enqueue
+      const unsigned long long fl = ldcg(&nxt->flc.v);
+      if (fl) {
+        const unsigned lane = threadIdx.x & 31;
+        const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+        const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+        long long base = gw * 32;
+        int v = base < (long long)fl ? ldcg(a.flist + base + lane) : -1;
+        long long b = 0, e = 0;
+        if (v >= 0) {
+          b = ld_off(a.off + v);
+          e = ld_off(a.off + v + 1);
+        }
+        while (base < (long long)fl) {
+          const long long nb = base + nw * 32;
+          int v2 = nb < (long long)fl ? ldcg(a.flist + nb + lane) : -1;
+          long long b2 = 0, e2 = 0;
+          if (v2 >= 0) {
+            b2 = ld_off(a.off + v2);
+            e2 = ld_off(a.off + v2 + 1);
+          }
+          enqueue_warp(v >= 0, v, b, e, a.L, a.q[(L + 1) & 1], nxt);
+          base = nb;
+          v = v2;
+          b = b2;
+          e = e2;
+        }
+        grid_barrier(&ctl->bar);
+      }
+    }
     const unsigned long long nF = ldcg(&nxt->nF.v);
     const unsigned long long aF = ldcg(&nxt->arcsF.v);
     if (blockIdx.x == 0 && threadIdx.x == 0) record_level(ctl, L, dir, cur, nxt);
@@ -1097,6 +1139,7 @@ void free_traversal_state(sage_graph *g) {
   dfree(g, t.expd);
   dfree(g, t.infar);
   dfree(g, t.farc);
+  dfree(g, t.flist);
   t = TraversalState();
 }
 
@@ -1118,6 +1161,12 @@ sage_status ensure_traversal_state(sage_graph *g) {
       free_traversal_state(g);
       return st;
     }
+  // deferred-contraction frontier list: n entries + one open 256-slot chunk per possible warp
+  if ((st = dalloc(g, (void **)&t.flist,
+                   sizeof(int) * (size_t)(n + (long long)g->num_sms * 64 * kDeferChunk + 64))) != SAGE_OK) {
+    free_traversal_state(g);
+    return st;
+  }
   if ((st = dalloc(g, &t.tailmem, sizeof(TailSmem))) != SAGE_OK) {
     free_traversal_state(g);
     return st;
@@ -1220,6 +1269,7 @@ static TravArgs make_args(sage_graph *g) {
   if (const char *e = getenv("SAGE_DEBUG_MAX_LEVELS")) a.max_levels = atoi(e);   // diagnostics only
   a.tail = (int *)g->ts.tmp_out;
   a.tailmem = reinterpret_cast<TailSmem *>(g->ts.tailmem);
+  a.flist = g->ts.flist;
   a.steal = 1;
   a.vec_ok = g->vec_ok ? 1 : 0;
   return a;

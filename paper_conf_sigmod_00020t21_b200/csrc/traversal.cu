@@ -175,7 +175,7 @@ struct TravArgs {
 // empty) into the next level's log; every warp takes groups grid-stride with the next group's ids
 // and rows loaded before the current enqueue.  Returns whether the list was non-empty (then the
 // caller must barrier before reading the log's counters).
-__device__ __noinline__ bool classify_deferred(const TravArgs &a, const unsigned long long *flc,
+__device__ __forceinline__ bool classify_deferred(const TravArgs &a, const unsigned long long *flc,
                                                const Queues &Q, CounterSet *cs) {
   const unsigned long long fl = ldcg(flc);
   if (!fl) return false;

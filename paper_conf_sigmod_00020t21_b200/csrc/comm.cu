@@ -91,6 +91,7 @@ struct MultiArgs {
   int vec_ok;
   int lvl;                         // current level L
   PartMap pm;
+  int *flist;                      // deferred contraction: frontier list
   // SSSP (frontier Bellman-Ford across ranks)
   const uint32_t *w;
   uint32_t *dist;                  // own rows' distances
@@ -107,6 +108,9 @@ struct BfsPushMulti {
   static constexpr bool kWeights = false;
   static constexpr bool kNeedRow = false;
   static constexpr bool kEnqueue = true;
+  static constexpr bool kDefer = true;   // contraction deferred to k_mclassify (see traversal.cu)
+  int *flist = nullptr;
+  unsigned long long *flc = nullptr;
   const MultiArgs *a;
   uint32_t *fb_next;
   const Queues *next_q;
@@ -145,13 +149,24 @@ __global__ void __launch_bounds__(kBlock, 4) k_mpush(const __grid_constant__ Mul
   __shared__ BfsPushMulti::Src fsrc[kWarps][32];
   const int warp = threadIdx.x >> 5;
   const int L = a.lvl;
+  if ((threadIdx.x & 31) == 0) wsm[warp].cpos = wsm[warp].cend = 0;
+  __syncwarp();
   BfsPushMulti f;
   f.a = &a;
   f.fb_next = a.do_enabled ? a.fb[(L + 1) % 3] : nullptr;
   f.next_q = &a.q[(L + 1) & 1];
   f.next_cs = &a.ctl->set[(L + 1) % 3];
+  f.flist = a.flist;
+  f.flc = &a.ctl->set[(L + 1) % 3].flc.v;
   consume_log<VEC>(f, a.L, a.q[L & 1], &a.ctl->set[L % 3], a.off, a.col, nullptr, &wsm[warp],
                    fsrc[warp], a.vec_ok);
+}
+
+// K2' of the deferred contraction for the vertices k_mpush claimed locally.
+__global__ void __launch_bounds__(kBlock) k_mclassify(const __grid_constant__ MultiArgs a) {
+  const int L = a.lvl;
+  classify_deferred(a.off, a.flist, &a.ctl->set[(L + 1) % 3].flc.v, a.L, a.q[(L + 1) & 1],
+                    &a.ctl->set[(L + 1) % 3]);
 }
 
 // Owners apply the candidates received from every other rank.
@@ -625,6 +640,7 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
   a.out = c->out;
   a.recv = c->recv;
   a.level = t.level;
+  a.flist = t.flist;
   a.do_enabled = do_enabled ? 1 : 0;
   a.vec_ok = g->vec_ok ? 1 : 0;
   a.pm = c->pm;
@@ -654,6 +670,7 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
     if (dir == 0) {
       if (g->vec == 4) k_mpush<4><<<grid_push, kBlock, 0, g->stream>>>(a);
       else k_mpush<1><<<grid_push, kBlock, 0, g->stream>>>(a);
+      k_mclassify<<<grid_push, kBlock, 0, g->stream>>>(a);
       // dense alltoall of the owners' candidate slices
       NCCL_CHECK(g, ncclGroupStart(), "group");
       for (int r = 0; r < c->world; ++r) {

@@ -464,6 +464,43 @@ __device__ __forceinline__ void defer_close(WarpScratch *ws, int &cnt, int *list
   __syncwarp();
 }
 
+// K2' of the deferred contraction: Tiled Partitioning of the frontier list (32-slot groups, -1 =
+// empty) into the next level's log; every warp takes groups grid-stride with the next group's ids
+// and rows loaded before the current enqueue.  Returns whether the list was non-empty (then the
+// caller must barrier before reading the log's counters).  Must stay inlined (an out-of-line call
+// cost k_bfs its register allocation).
+__device__ __forceinline__ bool classify_deferred(const long long *__restrict__ off, const int *flist,
+                                                  const unsigned long long *flc, const Ladder &L,
+                                                  const Queues &Q, CounterSet *cs) {
+  const unsigned long long fl = ldcg(flc);
+  if (!fl) return false;
+  const unsigned lane = threadIdx.x & 31;
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  long long base = gw * 32;
+  int v = base < (long long)fl ? ldcg(flist + base + lane) : -1;
+  long long b = 0, e = 0;
+  if (v >= 0) {
+    b = ld_off(off + v);
+    e = ld_off(off + v + 1);
+  }
+  while (base < (long long)fl) {
+    const long long nb = base + nw * 32;
+    const int v2 = nb < (long long)fl ? ldcg(flist + nb + lane) : -1;
+    long long b2 = 0, e2 = 0;
+    if (v2 >= 0) {
+      b2 = ld_off(off + v2);
+      e2 = ld_off(off + v2 + 1);
+    }
+    enqueue_warp(v >= 0, v, b, e, L, Q, cs);
+    base = nb;
+    v = v2;
+    b = b2;
+    e = e2;
+  }
+  return true;
+}
+
 // Append the lanes' filtered-in vertices to the warp buffer; flush full batches of 32.
 __device__ __forceinline__ void buffer_push(bool in, int v, WarpScratch *ws, int &cnt,
                                             const long long *__restrict__ off, const Ladder &L,

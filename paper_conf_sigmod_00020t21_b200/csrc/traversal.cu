@@ -171,41 +171,6 @@ struct TravArgs {
   int *flist;           // deferred contraction: frontier list (n + slack entries)
 };
 
-// K2' of the deferred contraction: Tiled Partitioning of the frontier list (32-slot groups, -1 =
-// empty) into the next level's log; every warp takes groups grid-stride with the next group's ids
-// and rows loaded before the current enqueue.  Returns whether the list was non-empty (then the
-// caller must barrier before reading the log's counters).
-__device__ __forceinline__ bool classify_deferred(const TravArgs &a, const unsigned long long *flc,
-                                               const Queues &Q, CounterSet *cs) {
-  const unsigned long long fl = ldcg(flc);
-  if (!fl) return false;
-  const unsigned lane = threadIdx.x & 31;
-  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
-  long long base = gw * 32;
-  int v = base < (long long)fl ? ldcg(a.flist + base + lane) : -1;
-  long long b = 0, e = 0;
-  if (v >= 0) {
-    b = ld_off(a.off + v);
-    e = ld_off(a.off + v + 1);
-  }
-  while (base < (long long)fl) {
-    const long long nb = base + nw * 32;
-    const int v2 = nb < (long long)fl ? ldcg(a.flist + nb + lane) : -1;
-    long long b2 = 0, e2 = 0;
-    if (v2 >= 0) {
-      b2 = ld_off(a.off + v2);
-      e2 = ld_off(a.off + v2 + 1);
-    }
-    enqueue_warp(v >= 0, v, b, e, a.L, Q, cs);
-    base = nb;
-    v = v2;
-    b = b2;
-    e = e2;
-  }
-  return true;
-}
-
 // Pull (bottom-up) step over the visited bitmap: one warp per 32-vertex word.
 __device__ __forceinline__ void pull_level(const TravArgs &a, int next_level, const uint32_t *fbc,
                                            uint32_t *fbn, const Queues &Qn, CounterSet *cur,
@@ -561,7 +526,7 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
     }
     if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
     grid_barrier(&ctl->bar);
-    if (BfsPush::kDefer && classify_deferred(a, &nxt->flc.v, a.q[(L + 1) & 1], nxt))
+    if (BfsPush::kDefer && classify_deferred(a.off, a.flist, &nxt->flc.v, a.L, a.q[(L + 1) & 1], nxt))
       grid_barrier(&ctl->bar);
     const unsigned long long nF = ldcg(&nxt->nF.v);
     const unsigned long long aF = ldcg(&nxt->arcsF.v);
@@ -956,7 +921,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
     consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok);
     if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
     grid_barrier(&ctl->bar);
-    if (SsspPush::kDefer && classify_deferred(a, &nxt->flc.v, a.q[(L + 1) & 1], nxt))
+    if (SsspPush::kDefer && classify_deferred(a.off, a.flist, &nxt->flc.v, a.L, a.q[(L + 1) & 1], nxt))
       grid_barrier(&ctl->bar);
     unsigned long long nF = ldcg(&nxt->nF.v);
     // near frontier exhausted: raise the threshold and pull the far pile forward

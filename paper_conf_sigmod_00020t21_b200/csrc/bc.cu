@@ -41,6 +41,7 @@ struct BcArgs {
   int src;
   int vec_ok;
   int max_levels;
+  int *flist;           // deferred contraction: frontier list
 };
 
 struct BcFwd {
@@ -50,6 +51,9 @@ struct BcFwd {
   static constexpr bool kWeights = false;
   static constexpr bool kNeedRow = false;
   static constexpr bool kEnqueue = true;
+  static constexpr bool kDefer = true;   // contraction deferred to a K2' phase (see traversal.cu)
+  int *flist = nullptr;
+  unsigned long long *flc = nullptr;
   int *level;
   double *sigma;
   int next_level;
@@ -115,6 +119,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_bc_fwd(const __grid_constant__ Bc
   __shared__ BcFwd::Src fsrc[kWarps][32];
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
+  if ((threadIdx.x & 31) == 0) wsm[warp].cpos = wsm[warp].cend = 0;
   for (int L = 0;; ++L) {
     CounterSet *cur = &ctl->set[L % 3];
     CounterSet *nxt = &ctl->set[(L + 1) % 3];
@@ -122,6 +127,8 @@ __global__ void __launch_bounds__(kBlock, 4) k_bc_fwd(const __grid_constant__ Bc
     if (blockIdx.x == 0 && threadIdx.x < (int)(sizeof(CounterSet) / sizeof(PaddedCounter)))
       reinterpret_cast<PaddedCounter *>(&ctl->set[(L + 2) % 3])[threadIdx.x].v = 0ull;
     BcFwd f;
+    f.flist = a.flist;
+    f.flc = &nxt->flc.v;
     f.level = a.level;
     f.sigma = a.sigma;
     f.next_level = L + 1;
@@ -129,6 +136,8 @@ __global__ void __launch_bounds__(kBlock, 4) k_bc_fwd(const __grid_constant__ Bc
     f.next_cs = nxt;
     consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, nullptr, &wsm[warp], fsrc[warp], a.vec_ok);
     grid_barrier(&ctl->bar);
+    if (classify_deferred(a.off, a.flist, &nxt->flc.v, a.L, a.q[(L + 1) & 1], nxt))
+      grid_barrier(&ctl->bar);
     const unsigned long long nF = ldcg(&nxt->nF.v);
     if (blockIdx.x == 0 && threadIdx.x == 0) {
       ctl->levels = L + 1;
@@ -263,6 +272,7 @@ extern "C" sage_status sage_bc(sage_graph *g, const int32_t *sources, int64_t n_
   a.seg = seg;
   a.vec_ok = g->vec_ok ? 1 : 0;
   a.max_levels = kMaxRec;
+  a.flist = t.flist;
   const void *ffn = g->vec == 4 ? (const void *)k_bc_fwd<4> : (const void *)k_bc_fwd<1>;
   const void *bfn = g->vec == 4 ? (const void *)k_bc_bwd<4> : (const void *)k_bc_bwd<1>;
   static int grid_f = 0, grid_b = 0;

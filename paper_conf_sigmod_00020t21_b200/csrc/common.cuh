@@ -404,7 +404,9 @@ __device__ unsigned long long g_prof[16];
 #define PROF_ADD(i, v)
 #endif
 
-// ---- deferred contraction (filters with kDefer; push BFS): a filtered-in vertex is only appended
+// ---- deferred contraction (filters with kDefer and a non-null flist; the kernels leave flist null
+// on small levels, where the second grid barrier would cost more than the enqueue stalls it
+// saves): a filtered-in vertex is only appended
 // to a plain frontier list (32-slot groups inside 256-slot chunks reserved per warp, -1 = empty
 // slot); Tiled Partitioning of the list into the next level's log runs as its own grid phase after
 // the level (K2' before K3', Fig. 2), where every warp classifies with all its loads in flight,
@@ -559,6 +561,33 @@ __device__ __forceinline__ void buffer_flush(WarpScratch *ws, int &cnt,
 //   Queues *next_q; CounterSet *next_cs;             where filtered-in vertices go
 // steal = false (ablation of Resident Tile Stealing, Fig. 10): tiles are dealt to warps
 // statically, round robin in batch units, instead of through the device-wide tickets.
+// Contraction of a filtered-in vertex: deferred (frontier list) or immediate (warp buffer -> log).
+#ifndef SAGE_DEFER_RUNTIME
+#define SAGE_DEFER_RUNTIME 0   // 1: small levels contract immediately (measured slower: the second path costs k_bfs 130 B of spills)
+#endif
+template <class F>
+__device__ __forceinline__ void push_filtered(const F &f, bool in, int v, WarpScratch *ws, int &cnt,
+                                              const long long *__restrict__ off, const Ladder &L) {
+  if constexpr (DeferTrait<F>::value) {
+    if (!SAGE_DEFER_RUNTIME || f.flist) {
+      defer_push(in, v, ws, cnt, f.flist, f.flc);
+      return;
+    }
+  }
+  buffer_push(in, v, ws, cnt, off, L, *f.next_q, f.next_cs);
+}
+template <class F>
+__device__ __forceinline__ void close_filtered(const F &f, WarpScratch *ws, int &cnt,
+                                               const long long *__restrict__ off, const Ladder &L) {
+  if constexpr (DeferTrait<F>::value) {
+    if (!SAGE_DEFER_RUNTIME || f.flist) {
+      defer_close(ws, cnt, f.flist, f.flc);
+      return;
+    }
+  }
+  if (cnt) buffer_flush(ws, cnt, off, L, *f.next_q, f.next_cs);
+}
+
 // Column-prefetch depth of a filter (F::kPrefetch, default 1 step ahead).
 template <class F, class = void> struct PrefetchDepth { static constexpr int value = 1; };
 template <class F> struct PrefetchDepth<F, std::void_t<decltype(F::kPrefetch)>> {
@@ -732,8 +761,7 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
           if constexpr (F::kEnqueue) {
 #pragma unroll
             for (int j = 0; j < VEC; ++j)
-              if constexpr (DeferTrait<F>::value) defer_push(in[j], v[j], ws, bcnt, f.flist, f.flc);
-              else buffer_push(in[j], v[j], ws, bcnt, off, L, *f.next_q, f.next_cs);
+              push_filtered(f, in[j], v[j], ws, bcnt, off, L);
           }
         }
         __syncwarp();
@@ -807,15 +835,13 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
       bool in[1];
       f.template visit<1>(kv, so, vv, w1, in, 1);
       if constexpr (F::kEnqueue) {
-        if constexpr (DeferTrait<F>::value) defer_push(in[0], vv[0], ws, bcnt, f.flist, f.flc);
-        else buffer_push(in[0], vv[0], ws, bcnt, off, L, *f.next_q, f.next_cs);
+        push_filtered(f, in[0], vv[0], ws, bcnt, off, L);
       }
     }
     __syncwarp();
   }
   if constexpr (F::kEnqueue) {
-    if constexpr (DeferTrait<F>::value) defer_close(ws, bcnt, f.flist, f.flc);
-    else if (bcnt) buffer_flush(ws, bcnt, off, L, *f.next_q, f.next_cs);
+    close_filtered(f, ws, bcnt, off, L);
   }
 }
 

@@ -169,6 +169,7 @@ struct TravArgs {
   struct TailSmem *tailmem;   // tail mode state (global scratch: only block 0 uses it)
   int steal;            // 0 = ablation: static tile assignment instead of stealing
   int *flist;           // deferred contraction: frontier list (n + slack entries)
+  unsigned long long defer_min_arcs;   // defer only on levels with arcs(F) >= this
 };
 
 // Pull (bottom-up) step over the visited bitmap: one warp per 32-vertex word.
@@ -503,7 +504,7 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
       f.v_base = 0;
       f.next_q = &a.q[(L + 1) & 1];
       f.next_cs = nxt;
-      f.flist = a.flist;
+      f.flist = (!SAGE_DEFER_RUNTIME || ldcg(&cur->arcsF.v) >= a.defer_min_arcs) ? a.flist : nullptr;
       f.flc = &nxt->flc.v;
 #ifdef SAGE_PROF
       const unsigned long long pt0 = globaltimer();
@@ -916,7 +917,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
     f.far = fa.far[k % 3];
     f.far_cnt = &fa.cnt[k % 3].v;
     f.expd = fa.delta == ~0ull ? nullptr : fa.expd;
-    f.flist = a.flist;
+    f.flist = (!SAGE_DEFER_RUNTIME || ldcg(&cur->arcsF.v) >= a.defer_min_arcs) ? a.flist : nullptr;
     f.flc = &nxt->flc.v;
     consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok);
     if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
@@ -1251,6 +1252,8 @@ static TravArgs make_args(sage_graph *g) {
   a.tail = (int *)g->ts.tmp_out;
   a.tailmem = reinterpret_cast<TailSmem *>(g->ts.tailmem);
   a.flist = g->ts.flist;
+  a.defer_min_arcs = 1ull << 16;   // SAGE_DEFER_MIN_ARCS overrides (tests: 0 = every level)
+  if (const char *e = getenv("SAGE_DEFER_MIN_ARCS")) a.defer_min_arcs = strtoull(e, nullptr, 10);
   a.steal = 1;
   a.vec_ok = g->vec_ok ? 1 : 0;
   return a;

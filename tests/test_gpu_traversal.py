@@ -356,3 +356,18 @@ def test_full_occupancy_grid_on_small_graphs(sage, monkeypatch):
         x, _ = G.pagerank(0.85, 10)
         xr = oracle.pagerank(g.off, g.col, 0.85, 10)
         assert np.max(np.abs(x - xr) / xr) <= 1e-6
+
+
+@pytest.mark.parametrize("min_arcs", ["0", "100000000000"])
+def test_deferred_and_immediate_contraction(sage, min_arcs, monkeypatch):
+    """Push BFS / SSSP with the deferred frontier list + K2' phase; SAGE_DEFER_MIN_ARCS selects
+    immediate contraction on small levels in builds with SAGE_DEFER_RUNTIME=1 (off by default):
+    exact either way."""
+    monkeypatch.setenv("SAGE_DEFER_MIN_ARCS", min_arcs)
+    for sym in (True, False):
+        g = sg.rmat(14, 16, seed=12, symmetric=sym)
+        w = sg.weights(g, 1)
+        with sage.load_csr(g.off, g.col, w, symmetric=sym) as G:
+            for s in sg.sources(g, 3, seed=2):
+                assert np.array_equal(G.bfs(int(s), push_only=True)[0], oracle.bfs(g.off, g.col, int(s)))
+                assert np.array_equal(G.sssp(int(s))[0], oracle.sssp(g.off, g.col, w, int(s))[0])

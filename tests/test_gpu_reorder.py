@@ -191,3 +191,21 @@ def test_online_reorder_pagerank_records_every_row(sage):
         assert np.array_equal(G.permutation(), sig1)
         xr = oracle.pagerank(g.off, g.col, 0.85, 3)
         assert np.max(np.abs(x - xr) / xr) <= 1e-6
+
+
+def test_online_reorder_errors(sage):
+    g = sg.rmat(10, 8, seed=1, symmetric=True)
+    with sage.load_csr(g.off, g.col, symmetric=True, host_columns=True) as G:
+        with pytest.raises(sage.SageError) as ei:
+            G.online_reorder(True)
+        assert ei.value.status == sage.E_UNSUPPORTED
+    with sage.load_csr(g.off, g.col, symmetric=True) as G:
+        with pytest.raises(sage.SageError) as ei:
+            G.online_reorder(True, sector_width=3)
+        assert ei.value.status == sage.E_INVALID
+        G.online_reorder(True, 8, 10 ** 15)        # threshold never reached: no round, identity
+        s = int(sg.sources(g, 1, seed=2)[0])
+        assert np.array_equal(G.bfs(s)[0], oracle.bfs(g.off, g.col, s))
+        info = G.online_info()
+        assert info["rounds"] == 0 and info["pending"] > 0
+        assert np.array_equal(G.permutation(), np.arange(g.n))

@@ -126,6 +126,10 @@ __device__ __forceinline__ uint32_t ld_stream1u(const uint32_t *p) {
   return r;
 }
 __device__ __forceinline__ long long ld_off(const long long *p) { return __ldg(p); }
+__device__ __forceinline__ void ld_row_pair(const long long *off, int v, long long *b, long long *e) {
+  *b = __ldg(off + v);
+  *e = __ldg(off + v + 1);
+}
 
 // L2 cache policies: the column / weight stream is read once per level -> evict_first; the
 // status words (visited bitmap, dist) are re-read at random all level long -> evict_last.
@@ -371,6 +375,86 @@ __device__ __forceinline__ void enqueue_warp(bool active, int v, long long b, lo
   }
 }
 
+// Two-pass form of enqueue_warp for a warp that classifies many 32-vertex groups (the K2' phase):
+// enqueue_count accumulates what the groups need (lane 0: CTA tiles, lane c: entries of queue c,
+// lane 29: order-list entries; nF / arcs warp-uniform), the warp reserves everything with ONE
+// round of atomics, and enqueue_write writes each group at the running bases (no atomics).
+__device__ __forceinline__ void enqueue_count(bool active, long long b, long long e, const Ladder &L,
+                                              unsigned long long &tot, unsigned long long &nf,
+                                              unsigned long long &arcs) {
+  const unsigned am = __ballot_sync(FULL, active);
+  if (!am) return;
+  const unsigned lane = lane_id();
+  RowSplit s{0, 0, 0, 0};
+  if (active) s = split_row(b, e, L);
+  const unsigned long long totq = warp_sum64(active ? (unsigned long long)s.q : 0ull);
+  arcs += warp_sum64(active ? (unsigned long long)(e - b) : 0ull);
+  nf += (unsigned long long)__popc(am);
+#pragma unroll
+  for (int c = 1; c < kQueues; ++c) {
+    unsigned cm = 0;
+    if (c < L.ncls) cm = __ballot_sync(FULL, active && (s.r & (L.B >> c)));
+    else if (c == L.ncls) cm = __ballot_sync(FULL, active && (s.h > 0 || (s.r & (L.M - 1)) != 0));
+    if ((int)lane == c) tot += (unsigned long long)__popc(cm);
+  }
+  if (lane == 0) tot += totq;
+  if (lane == 29) tot += (unsigned long long)__popc(am);
+}
+__device__ __forceinline__ void enqueue_write(bool active, int v, long long b, long long e, const Ladder &L,
+                                              const Queues &Q, unsigned long long &run) {
+  const unsigned am = __ballot_sync(FULL, active);
+  if (!am) return;
+  const unsigned lane = lane_id();
+  const unsigned lt = lanemask_lt();
+  RowSplit s{0, 0, 0, 0};
+  if (active) s = split_row(b, e, L);
+  unsigned long long q = active ? (unsigned long long)s.q : 0ull;
+  unsigned long long incq = q;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    unsigned long long y = __shfl_up_sync(FULL, incq, o);
+    if ((int)lane >= o) incq += y;
+  }
+  const unsigned long long totq = shfl64(incq, 31);
+  if (Q.order) {
+    const unsigned long long ob = shfl64(run, 29);
+    if (active) Q.order[ob + __popc(am & lt)] = v;
+    if (lane == 29) run += (unsigned long long)__popc(am);
+  }
+#pragma unroll
+  for (int c = 1; c < kQueues; ++c) {
+    if (c > L.ncls) break;
+    unsigned cm;
+    if (c < L.ncls) cm = __ballot_sync(FULL, active && (s.r & (L.B >> c)));
+    else cm = __ballot_sync(FULL, active && (s.h > 0 || (s.r & (L.M - 1)) != 0));
+    const unsigned long long base = shfl64(run, c);
+    if (cm & (1u << lane)) {
+      int *qp = (c == L.ncls) ? Q.frag : Q.cls[c];
+      qp[base + __popc(cm & lt)] = v;
+    }
+    if ((int)lane == c) run += (unsigned long long)__popc(cm);
+  }
+  if (totq) {
+    const unsigned long long base0 = shfl64(run, 0);
+    if (q > 0 && q <= SAGE_ENQ_LANEQ) {
+      const unsigned long long bs = base0 + incq - q;
+      for (unsigned long long j = 0; j < q; ++j) st_tile(Q.cta + bs + j, s.b2 + (long long)j * L.B, v, L.B);
+    }
+    unsigned hm = __ballot_sync(FULL, q > SAGE_ENQ_LANEQ);
+    while (hm) {
+      const int src = __ffs(hm) - 1;
+      hm &= hm - 1;
+      const unsigned long long qs = shfl64(q, src);
+      const unsigned long long bs = base0 + shfl64(incq, src) - qs;
+      const long long b2 = (long long)shfl64((unsigned long long)s.b2, src);
+      const int vv = __shfl_sync(FULL, v, src);
+      for (unsigned long long j = lane; j < qs; j += 32)
+        st_tile(Q.cta + bs + j, b2 + (long long)j * L.B, vv, L.B);
+    }
+    if (lane == 0) run += totq;
+  }
+}
+
 // enqueue_warp for vertex ids only: loads the rows first (one round of loads for the warp).
 // Not inlined: it is the cold path of the consumer (once per 32 filtered-in vertices) and
 // inlining it at every call site multiplies the kernel's code size (I-cache misses).
@@ -479,26 +563,55 @@ __device__ __forceinline__ bool classify_deferred(const long long *__restrict__ 
   const unsigned lane = threadIdx.x & 31;
   const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
-  long long base = gw * 32;
-  int v = base < (long long)fl ? ldcg(flist + base + lane) : -1;
-  long long b = 0, e = 0;
-  if (v >= 0) {
-    b = ld_off(off + v);
-    e = ld_off(off + v + 1);
-  }
-  while (base < (long long)fl) {
-    const long long nb = base + nw * 32;
-    const int v2 = nb < (long long)fl ? ldcg(flist + nb + lane) : -1;
-    long long b2 = 0, e2 = 0;
-    if (v2 >= 0) {
-      b2 = ld_off(off + v2);
-      e2 = ld_off(off + v2 + 1);
+  const long long first = gw * 32, step = nw * 32;
+  // pass A: what this warp's groups need (next group's ids and rows loaded ahead)
+  unsigned long long tot = 0, nf = 0, arcs = 0;
+  {
+    long long base = first;
+    int v = base < (long long)fl ? ldcg(flist + base + lane) : -1;
+    long long b = 0, e = 0;
+    if (v >= 0) ld_row_pair(off, v, &b, &e);
+    while (base < (long long)fl) {
+      const long long nb = base + step;
+      const int v2 = nb < (long long)fl ? ldcg(flist + nb + lane) : -1;
+      long long b2 = 0, e2 = 0;
+      if (v2 >= 0) ld_row_pair(off, v2, &b2, &e2);
+      enqueue_count(v >= 0, b, e, L, tot, nf, arcs);
+      base = nb;
+      v = v2;
+      b = b2;
+      e = e2;
     }
-    enqueue_warp(v >= 0, v, b, e, L, Q, cs);
-    base = nb;
-    v = v2;
-    b = b2;
-    e = e2;
+  }
+  if (nf == 0) return true;
+  // one round of reservations for all of them
+  unsigned long long run = 0;
+  if (lane == 0 || ((int)lane <= L.ncls)) {
+    if (tot) run = atomicAdd(&cs->cnt[lane].v, tot);
+  } else if (lane == 29) {
+    if (Q.order && tot) run = atomicAdd(Q.order_cnt, tot);
+  } else if (lane == 30) {
+    atomicAdd(&cs->nF.v, nf);
+  } else if (lane == 31) {
+    if (arcs) atomicAdd(&cs->arcsF.v, arcs);
+  }
+  // pass B: the same groups again (rows now in L1/L2), written at the running bases
+  {
+    long long base = first;
+    int v = base < (long long)fl ? ldcg(flist + base + lane) : -1;
+    long long b = 0, e = 0;
+    if (v >= 0) ld_row_pair(off, v, &b, &e);
+    while (base < (long long)fl) {
+      const long long nb = base + step;
+      const int v2 = nb < (long long)fl ? ldcg(flist + nb + lane) : -1;
+      long long b2 = 0, e2 = 0;
+      if (v2 >= 0) ld_row_pair(off, v2, &b2, &e2);
+      enqueue_write(v >= 0, v, b, e, L, Q, run);
+      base = nb;
+      v = v2;
+      b = b2;
+      e = e2;
+    }
   }
   return true;
 }

@@ -169,6 +169,14 @@ __device__ __forceinline__ uint32_t ld_colu(const uint32_t *p, unsigned long lon
 }
 // status word load (kept in L2).  SAGE_STATUS_NC selects the non-coherent path: a stale read
 // is harmless for the visited bitmap (bits only go 0 -> 1 within a kernel, atomicOr decides).
+// stealing ticket batches (`consume_log`): grabs per warp per class, column elements per grab
+#ifndef SAGE_TK_GRABS
+#define SAGE_TK_GRABS 2
+#endif
+#ifndef SAGE_TK_ELEMS
+#define SAGE_TK_ELEMS 4096
+#endif
+
 __device__ __forceinline__ uint32_t ld_status(const uint32_t *p, unsigned long long pol) {
   uint32_t r;
 #if defined(SAGE_STATUS_NC) && SAGE_STATUS_NC
@@ -729,8 +737,8 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
     const int spt = (t / VEC) > 32 ? (t / (32 * VEC)) : 1;  // steps per tile
     // adaptive ticket batch: ~2 grabs per warp, <= 16 KB of columns per grab; warps beyond the
     // number of grabs skip the class (no ticket traffic on small levels)
-    unsigned long long batch = (count + 2 * nwarps - 1) / (2 * nwarps);
-    const unsigned long long bmax = (4096 / t) > (unsigned)tps ? (4096 / t) : tps;
+    unsigned long long batch = (count + SAGE_TK_GRABS * nwarps - 1) / (SAGE_TK_GRABS * nwarps);
+    const unsigned long long bmax = (SAGE_TK_ELEMS / t) > (unsigned)tps ? (SAGE_TK_ELEMS / t) : tps;
     if (batch > bmax) batch = bmax;
     batch = ((batch + tps - 1) / tps) * tps;
     const unsigned long long grabs = (count + batch - 1) / batch;

@@ -125,7 +125,21 @@ __device__ __forceinline__ uint32_t ld_stream1u(const uint32_t *p) {
   asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
   return r;
 }
+#if defined(SAGE_OFF_L1) && SAGE_OFF_L1 == 1
+__device__ __forceinline__ long long ld_off(const long long *p) {
+  long long r;
+  asm volatile("ld.global.nc.L1::evict_last.s64 %0, [%1];" : "=l"(r) : "l"(p));
+  return r;
+}
+#elif defined(SAGE_OFF_L1) && SAGE_OFF_L1 == 2
+__device__ __forceinline__ long long ld_off(const long long *p) {
+  long long r;
+  asm volatile("ld.global.nc.L1::no_allocate.s64 %0, [%1];" : "=l"(r) : "l"(p));
+  return r;
+}
+#else
 __device__ __forceinline__ long long ld_off(const long long *p) { return __ldg(p); }
+#endif
 __device__ __forceinline__ void ld_row_pair(const long long *off, int v, long long *b, long long *e) {
   *b = __ldg(off + v);
   *e = __ldg(off + v + 1);

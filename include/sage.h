@@ -60,10 +60,8 @@ enum {
                               every tile request line-aligned.  sage_reorder is unsupported.     */
   SAGE_F_PUSH_ONLY = 16u,  /* disable direction switching: every level is the paper's push
                               expansion (Alg. 2/3).  Can also be set per call (sage_bfs_ex).     */
-  SAGE_F_BINNED = 32u,     /* per call (sage_bfs_ex), experimental: two-phase push levels (neighbour
-                              ids binned by vertex slice, then filtered against shared-memory
-                              slices of the visited bitmap).  Results identical;
-                              slower than the default direct filter on B200 as measured.        */
+                           /* 32u: reserved (an experimental binned push level of round 1, removed;
+                              DESIGN.md §5 keeps its measurements)                                */
   SAGE_F_NO_STEALING = 64u /* per call (sage_bfs_ex), ablation (Fig. 10): tiles are dealt to
                               warps statically instead of through Resident Tile Stealing        */
 };
@@ -91,6 +89,8 @@ typedef struct {
                         else a power of two in [1, 64]; default 4 (16 B, one int4 load)          */
   double alpha;      /* Beamer push->pull threshold: pull when arcs(F) > arcs(unvisited)/alpha; 15 */
   double beta;       /* pull->push threshold: push when |F| < n/beta; default 18                     */
+  int32_t ctas_per_sm; /* resident CTAs per SM of the persistent kernels; 0 = automatic (the
+                        occupancy limit, one CTA per SM on graphs under 8M arcs)                  */
 } sage_options;
 
 /* CSR input of sage_load_csr (Fig. 1: u_offset / v arrays).                         */
@@ -237,10 +237,11 @@ sage_status sage_debug_reorder_stages(sage_graph *g, int32_t sector_width, const
                                       int64_t *loc3_out, uint8_t *mover_out);
 
 /* Diagnostic entry point: per-level records of the last BFS / SSSP query on this graph, 9 int64 per
- * level: direction (0 push, 1 pull), |F|, arcs(F), arcs inspected, vertices scanned (pull),
- * vertices discovered, device time since the kernel started at the end of the level (ns), and
- * the time at which the last warp finished the level's work, before the grid barrier (ns), and
- * (binned push levels) the end of the expansion phase (ns, microsecond resolution; 0 otherwise).
+ * level (rec_out must hold 9 * cap int64): direction (0 push, 1 pull), |F|, arcs(F), arcs
+ * inspected, vertices scanned (pull), vertices discovered, device time since the kernel started
+ * at the end of the level (ns), the time at which the last warp finished the level's work,
+ * before the grid barrier (ns), and the end of the level's expansion phase before Tiled
+ * Partitioning of the next frontier (ns; 0 when not recorded).
  * Writes min(levels, cap) records to host memory; *n_out = number of levels (<= 4096 kept).     */
 sage_status sage_debug_level_records(const sage_graph *g, int64_t *rec_out, int32_t cap,
                                      int32_t *n_out);

@@ -19,7 +19,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, os.environ.get("SAGE_LIB", "libsage.so"))
 
 OK, E_INVALID, E_NOMEM, E_CUDA, E_NCCL, E_OVERFLOW, E_UNSUPPORTED = range(7)
-F_SYMMETRIC, F_DEVICE_PTRS, F_BORROW, F_NO_VALIDATE, F_PUSH_ONLY, F_BINNED, F_NO_STEALING = 1, 2, 4, 8, 16, 32, 64
+F_SYMMETRIC, F_DEVICE_PTRS, F_BORROW, F_NO_VALIDATE, F_PUSH_ONLY, F_NO_STEALING = 1, 2, 4, 8, 16, 64
 F_HOST_COLUMNS = 128
 STATUS_NAMES = {0: "SAGE_OK", 1: "SAGE_E_INVALID", 2: "SAGE_E_NOMEM", 3: "SAGE_E_CUDA",
                 4: "SAGE_E_NCCL", 5: "SAGE_E_OVERFLOW", 6: "SAGE_E_UNSUPPORTED"}
@@ -38,7 +38,7 @@ class SageError(RuntimeError):
 
 class Options(ctypes.Structure):
     _fields_ = [("tile_cta", ctypes.c_int32), ("tile_min", ctypes.c_int32), ("align", ctypes.c_int32),
-                ("alpha", ctypes.c_double), ("beta", ctypes.c_double)]
+                ("alpha", ctypes.c_double), ("beta", ctypes.c_double), ("ctas_per_sm", ctypes.c_int32)]
 
 
 class Dist(ctypes.Structure):
@@ -196,14 +196,14 @@ class Graph:
 
     # ------------------------------------------------------------------ queries
     def bfs(self, source: int, out=None, parent_out=None, parents: bool = False, push_only: bool = False,
-            binning: bool = False, stealing: bool = True):
+            stealing: bool = True):
         """sage_bfs_ex -> (level int32[n_local], parent or None, stats dict)."""
         o = _out(out, self.n_local, np.int32)
         po = None
         if parents or parent_out is not None:
             po = _out(parent_out, self.n_local, np.int32)
         st = Stats()
-        fl = (F_PUSH_ONLY if push_only else 0) | (F_BINNED if binning else 0) | (0 if stealing else F_NO_STEALING)
+        fl = (F_PUSH_ONLY if push_only else 0) | (0 if stealing else F_NO_STEALING)
         _check(lib().sage_bfs_ex(self._h, int(source), o.ptr, po.ptr if po else None, fl, ctypes.byref(st)))
         return o.obj, (po.obj if po else None), st.as_dict()
 
@@ -284,8 +284,9 @@ class Graph:
         return off, col[:self.m], w[:self.m]
 
     def level_records(self) -> np.ndarray:
-        """sage_debug_level_records -> int64[levels, 8] (dir, |F|, arcs(F), inspected, scanned,
-        discovered, t_ns at level end, t_ns when the last warp finished) of the last BFS/SSSP query."""
+        """sage_debug_level_records -> int64[levels, 9] (dir, |F|, arcs(F), inspected, scanned,
+        discovered, t_ns at level end, t_ns when the last warp finished, t_ns at the end of the
+        expansion phase) of the last BFS/SSSP query."""
         n = ctypes.c_int32(0)
         buf = np.zeros(9 * 4096, dtype=np.int64)
         _check(lib().sage_debug_level_records(self._h, buf.ctypes.data, 4096, ctypes.byref(n)))
@@ -311,7 +312,7 @@ def nccl_unique_id() -> bytes:
 
 def load_csr(off, col, w=None, n: int | None = None, symmetric: bool = False, push_only: bool = False,
              borrow: bool = False, validate: bool = True, tile_cta: int = 256, tile_min: int = 8,
-             align: int = 4, alpha: float = 15.0, beta: float = 18.0, stream=None,
+             align: int = 4, alpha: float = 15.0, beta: float = 18.0, stream=None, ctas_per_sm: int = 0,
              rank: int = 0, world: int = 1, nccl_unique_id: bytes | None = None,
              v_begin: int = 0, v_end: int | None = None, host_columns: bool = False) -> Graph:
     """sage_load_csr.  ``off``/``col``/``w`` are host arrays or tensors, or CUDA tensors."""
@@ -337,8 +338,12 @@ def load_csr(off, col, w=None, n: int | None = None, symmetric: bool = False, pu
     csr.col_indices = pc
     csr.weights = pw
     csr.flags = flags
+    if stream is None and dev:
+        # device inputs: order the library's work after the caller's producing work (torch stream)
+        import torch
+        stream = torch.cuda.current_stream().cuda_stream
     csr.cuda_stream = stream
-    opts = Options(tile_cta, tile_min, align, alpha, beta)
+    opts = Options(tile_cta, tile_min, align, alpha, beta, ctas_per_sm)
     csr.opts = ctypes.pointer(opts)
     dist = None
     if nccl_unique_id is not None:

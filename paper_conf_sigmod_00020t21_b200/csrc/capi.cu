@@ -68,8 +68,7 @@ static cudaMemPool_t pool_for(int dev) {
 sage_status dalloc(sage_graph *g, void **p, size_t bytes) {
   *p = nullptr;
   if (bytes == 0) bytes = 16;
-  static const bool use_pool = getenv("SAGE_NO_POOL") == nullptr;
-  cudaMemPool_t pool = use_pool ? pool_for(g->device) : nullptr;
+  cudaMemPool_t pool = pool_for(g->device);
   cudaError_t e = pool ? cudaMallocFromPoolAsync(p, bytes, pool, g->stream)
                        : cudaMallocAsync(p, bytes, g->stream);
   if (e != cudaSuccess) {
@@ -167,7 +166,7 @@ static int ilog2(long long x) {
 static bool is_pow2(long long x) { return x > 0 && (x & (x - 1)) == 0; }
 
 static sage_status make_ladder(const sage_options *o, sage_graph *g) {
-  int B = 256, M = 8, A = 4;
+  int B = 256, M = 8, A = 4, cps = 0;
   double alpha = 15.0, beta = 18.0;
   if (o) {
     B = o->tile_cta;
@@ -175,6 +174,11 @@ static sage_status make_ladder(const sage_options *o, sage_graph *g) {
     A = o->align;
     alpha = o->alpha;
     beta = o->beta;
+    cps = o->ctas_per_sm;
+  }
+  if (cps < 0 || cps > 32) {
+    set_error("ctas_per_sm must be in [0, 32]");
+    return SAGE_E_INVALID;
   }
   if (!is_pow2(B) || B > 4096) {
     set_error("tile_cta must be a power of two in [1, 4096]");
@@ -199,6 +203,7 @@ static sage_status make_ladder(const sage_options *o, sage_graph *g) {
   g->ladder.ncls = ilog2(B / M) + 1;
   g->alpha = alpha;
   g->beta = beta;
+  g->ctas_per_sm = cps;
   return SAGE_OK;
 }
 
@@ -288,6 +293,16 @@ sage_status sage_load_csr(const sage_csr *in, sage_graph **out) {
   } else {
     cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking);
     g->own_stream = true;
+    if (devptrs) {
+      // device inputs were produced on the caller's (legacy default) stream: order the copy,
+      // the validation pass and every later read of borrowed arrays after that work
+      cudaEvent_t ev;
+      if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) == cudaSuccess) {
+        cudaEventRecord(ev, cudaStreamLegacy);
+        cudaStreamWaitEvent(g->stream, ev, 0);
+        cudaEventDestroy(ev);
+      }
+    }
   }
   sage_status st = make_ladder(in->opts, g);
   if (st != SAGE_OK) {

@@ -68,10 +68,11 @@ struct CounterSet {                      // counters of one log (rotated over 3 
 
 struct LevelRec {                        // per-level record (first kMaxRec levels)
   int dir;                               // 0 push, 1 pull
-  int t_mid_us;                          // binned push: phase-1 end (us after the level start)
+  int pad_;
   unsigned long long nF, arcsF, inspected, scanned, discovered;
   unsigned long long t_ns;               // %globaltimer at the end of the level
   unsigned long long t_work;             // %globaltimer when the last warp finished its work
+  unsigned long long t_mid;              // %globaltimer after the expansion's grid barrier (K2' start)
 };
 constexpr int kMaxRec = 4096;
 
@@ -125,24 +126,12 @@ __device__ __forceinline__ uint32_t ld_stream1u(const uint32_t *p) {
   asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
   return r;
 }
-#if defined(SAGE_OFF_L1) && SAGE_OFF_L1 == 1
-__device__ __forceinline__ long long ld_off(const long long *p) {
-  long long r;
-  asm volatile("ld.global.nc.L1::evict_last.s64 %0, [%1];" : "=l"(r) : "l"(p));
-  return r;
-}
-#elif defined(SAGE_OFF_L1) && SAGE_OFF_L1 == 2
-__device__ __forceinline__ long long ld_off(const long long *p) {
-  long long r;
-  asm volatile("ld.global.nc.L1::no_allocate.s64 %0, [%1];" : "=l"(r) : "l"(p));
-  return r;
-}
-#else
+// row offsets: read-only, re-read by the K2' passes and the consumer's metadata round -> L1-
+// allocating non-coherent loads (round 1 A/B: L1::evict_last equal, L1::no_allocate +3%)
 __device__ __forceinline__ long long ld_off(const long long *p) { return __ldg(p); }
-#endif
 __device__ __forceinline__ void ld_row_pair(const long long *off, int v, long long *b, long long *e) {
-  *b = __ldg(off + v);
-  *e = __ldg(off + v + 1);
+  *b = ld_off(off + v);
+  *e = ld_off(off + v + 1);
 }
 
 // L2 cache policies: the column / weight stream is read once per level -> evict_first; the
@@ -181,9 +170,8 @@ __device__ __forceinline__ uint32_t ld_colu(const uint32_t *p, unsigned long lon
                : "=r"(r) : "l"(p), "l"(pol));
   return r;
 }
-// status word load (kept in L2).  SAGE_STATUS_NC selects the non-coherent path: a stale read
-// is harmless for the visited bitmap (bits only go 0 -> 1 within a kernel, atomicOr decides).
-// status loads' L1 policy: 2 = L1::evict_last (default; hub status words stay in L1, measured
+// status word load (kept in L2; a stale read is harmless for the visited bitmap: bits only go
+// 0 -> 1 within a kernel and the atomicOr claim decides).  Status loads' L1 policy: 2 = L1::evict_last (default; hub status words stay in L1, measured
 // 2.767 -> 2.742 ms on C2 push BFS), 1 = L1::no_allocate (2.786), 0 = default allocation
 #ifndef SAGE_STATUS_L1
 #define SAGE_STATUS_L1 2
@@ -198,9 +186,7 @@ __device__ __forceinline__ uint32_t ld_colu(const uint32_t *p, unsigned long lon
 
 __device__ __forceinline__ uint32_t ld_status(const uint32_t *p, unsigned long long pol) {
   uint32_t r;
-#if defined(SAGE_STATUS_NC) && SAGE_STATUS_NC
-  asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
-#elif defined(SAGE_STATUS_L1) && SAGE_STATUS_L1 == 1
+#if defined(SAGE_STATUS_L1) && SAGE_STATUS_L1 == 1
   asm volatile("ld.global.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
 #elif defined(SAGE_STATUS_L1) && SAGE_STATUS_L1 == 2
   asm volatile("ld.global.L1::evict_last.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
@@ -492,10 +478,7 @@ __device__ __forceinline__ void enqueue_write(bool active, int v, long long b, l
 static __device__ __noinline__ void enqueue_ids(bool active, int v, const long long *__restrict__ off,
                                             const Ladder &L, const Queues &Q, CounterSet *cs) {
   long long b = 0, e = 0;
-  if (active) {
-    b = __ldg(off + v);
-    e = __ldg(off + v + 1);
-  }
+  if (active) ld_row_pair(off, v, &b, &e);
   enqueue_warp(active, v, b, e, L, Q, cs);
 }
 

@@ -32,15 +32,7 @@ struct TraversalState {     // per-query scratch, allocated on first use and kep
   Queues q[2];                    // double-buffered per-level tile logs
   Ctl *ctl = nullptr;             // device control block
   int32_t *tmp_out = nullptr;     // ID-translation scratch (n_local)
-  int *bins = nullptr;            // binned push: nslices x bin_cap neighbour ids
-  long long bin_cap = 0;
-  PaddedCounter *fill = nullptr;  // binned push: [2][kMaxSlices] bin fill counters
-  int nslices = 0;
-  int *far[3] = {nullptr, nullptr, nullptr};  // SSSP near-far: rotating far piles
-  uint32_t *infar = nullptr;      // SSSP near-far: far-pile membership bitmap
-  PaddedCounter *farc = nullptr;  // SSSP near-far: [3] pile sizes + [3] scan minima
   void *tailmem = nullptr;        // BFS tail mode state (global scratch)
-  uint32_t *expd = nullptr;       // SSSP near-far: last expanded distance per vertex
   int *flist = nullptr;           // BFS deferred contraction: frontier list
 };
 
@@ -53,14 +45,6 @@ struct PageRankState {      // the all-V resident tile log (built once, reused; 
   double *x = nullptr, *y = nullptr;
   float *c = nullptr;             // pull form: x_u / out(u)
   CounterSet *cs = nullptr;       // device copy of the log's counters (+ rotating tickets)
-  // binned push form (pagerank.cu, PrPushBin); bin_lg == 0 = not set up
-  int bin_lg = 0, nbin = 0;
-  long long bin_warps = 0;
-  long long *bstart = nullptr;
-  unsigned long long *bfill = nullptr;
-  int *ev = nullptr;
-  double *ec = nullptr;
-  unsigned *wpos = nullptr, *wend = nullptr;
 };
 
 }  // namespace sage
@@ -87,7 +71,7 @@ struct sage_graph {
   int64_t n_isolated = 0;
   sage::Ladder ladder{};
   double alpha = 15.0, beta = 18.0;
-  double w_mean = 0.0;        // mean arc weight (SSSP near-far threshold step), lazily computed
+  int ctas_per_sm = 0;        // sage_options.ctas_per_sm (0 = automatic)
   int vec = 4;                // neighbours per lane per step (4; 1 when tile_min < 4)
   bool vec_ok = true;         // sub-warp tiles use 16-B loads (align % 4 == 0, aligned arrays)
   // reordering: sigma[v_orig] = current label; sigma_inv[label] = v_orig (null = identity)
@@ -104,5 +88,5 @@ struct sage_graph {
   long long online_thr = 0, online_pending = 0, online_rounds = 0, online_movers = 0, online_swaps = 0;
   uint32_t *samp_w = nullptr;
   unsigned long long *samp_acc = nullptr;
-  int grid_bfs = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0, grid_bin = 0, grid_pr_bin = 0;   // persistent grid sizes
+  int grid_bfs = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0;   // persistent grid sizes
 };

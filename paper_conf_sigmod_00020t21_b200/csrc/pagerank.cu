@@ -98,81 +98,6 @@ struct PrArgs {
   float *c;           // pull form: x_u / out(u) in fp32
   Ctl *ctl;
   int vec_ok;
-  // binned push (PrPushBin): far contributions staged per target block, applied block by block
-  int bin_lg;                     // block = vertex >> bin_lg
-  int nbin;
-  const long long *bstart;        // bin b's entries live at [bstart[b], bstart[b] + cap)
-  unsigned long long *bfill;      // reserved entries per bin (multiple of kPrChunk)
-  int *ev;                        // entry target (-1 = pad)
-  double *ec;                     // entry contribution
-  unsigned *wpos, *wend;          // per (warp, bin) open chunk [wpos, wend) relative to bstart[b]
-};
-constexpr int kPrChunk = 64;      // entries reserved per (warp, bin) at a time
-
-// Binned push form (B200 addition; same arithmetic as Alg. 1 l.26-29): on a graph
-// whose y does not fit L2, every arc whose target lies outside the source's 2^bin_lg-vertex block
-// would cost a DRAM read-modify-write of a y sector.  Such contributions (v, c_u) are appended to
-// the bin of v's block instead (12 B written + 12 B read later) and applied after the sweep, bin
-// by bin, while that block of y is L2-resident; near targets are added directly.
-struct PrPushBin {
-  struct Src {
-    double c;
-    int ublk;
-  };
-  static constexpr bool kWeights = false;
-  static constexpr bool kNeedRow = true;
-  static constexpr bool kEnqueue = false;
-  static constexpr bool kSplit = false;
-  const Queues *next_q = nullptr;
-  CounterSet *next_cs = nullptr;
-  const PrArgs *a;
-  unsigned *wpos, *wend;          // this warp's chunk state (nbin entries each)
-
-  __device__ __forceinline__ Src src(bool valid, int u, long long b, long long e) const {
-    return Src{(valid && e > b) ? ldcg(a->x + u) / (double)(e - b) : 0.0, u >> a->bin_lg};
-  }
-  // warp-collective: lanes with `far` append (v, c) to bin v >> bin_lg (consecutive slots per bin)
-  __device__ __forceinline__ void append(bool far, int v, double c) const {
-    const unsigned fm = __ballot_sync(FULL, far);
-    if (!fm) return;
-    const unsigned lane = lane_id();
-    const int b = far ? (v >> a->bin_lg) : -1 - (int)lane;
-    const unsigned peers = __match_any_sync(FULL, b);
-    const int leader = __ffs(peers) - 1;
-    const int cnt = __popc(peers), rank = __popc(peers & lanemask_lt());
-    unsigned pos = 0, room = 0, nbase = 0;
-    if (far && (int)lane == leader) {
-      pos = wpos[b];
-      const unsigned end = wend[b];
-      room = end - pos;
-      if (room >= (unsigned)cnt) {
-        wpos[b] = pos + cnt;
-      } else {   // open a new chunk; the first `room` entries still fill the old one
-        nbase = (unsigned)atomicAdd(a->bfill + b, (unsigned long long)kPrChunk);
-        wpos[b] = nbase + (cnt - room);
-        wend[b] = nbase + kPrChunk;
-      }
-    }
-    pos = __shfl_sync(FULL, pos, leader);
-    room = __shfl_sync(FULL, room, leader);
-    nbase = __shfl_sync(FULL, nbase, leader);
-    if (far) {
-      const long long i = a->bstart[b] + (long long)((unsigned)rank < room ? pos + rank : nbase + (rank - room));
-      a->ev[i] = v;
-      a->ec[i] = c;
-    }
-  }
-  template <int N>
-  __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N],
-                                        const uint32_t (&)[N], bool (&in)[N], int) const {
-#pragma unroll
-    for (int j = 0; j < N; ++j) {
-      in[j] = false;
-      const bool far = valid && (v[j] >> a->bin_lg) != s.ublk;
-      if (valid && !far) atomicAdd(a->y + v[j], s.c);
-      append(far, v[j], s.c);
-    }
-  }
 };
 
 // Build the all-V resident log: one thread per vertex, warp-aggregated classification.
@@ -201,25 +126,6 @@ __global__ void k_build_log(const long long *__restrict__ off, long long n, Ladd
   }
 }
 
-// Arcs whose target lies outside the source's block, per target block (binned push capacities).
-__global__ void k_far_count(const long long *__restrict__ off, const int *__restrict__ col, long long n,
-                            int lg, int nbin, unsigned long long *cnt) {
-  extern __shared__ unsigned long long hc[];
-  for (int i = threadIdx.x; i < nbin; i += blockDim.x) hc[i] = 0ull;
-  __syncthreads();
-  const long long stride = (long long)gridDim.x * (blockDim.x / 32);
-  for (long long u = (long long)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); u < n; u += stride) {
-    const int ub = (int)(u >> lg);
-    for (long long k = off[u] + lane_id(); k < off[u + 1]; k += 32) {
-      const int vb = col[k] >> lg;
-      if (vb != ub) atomicAdd(&hc[vb], 1ull);
-    }
-  }
-  __syncthreads();
-  for (int i = threadIdx.x; i < nbin; i += blockDim.x)
-    if (hc[i]) atomicAdd(cnt + i, hc[i]);
-}
-
 __global__ void k_pr_init(double *x, double *y, long long n, double v0) {
   const long long stride = (long long)gridDim.x * blockDim.x;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
@@ -228,10 +134,10 @@ __global__ void k_pr_init(double *x, double *y, long long n, double v0) {
   }
 }
 
-template <int VEC, bool BIN>
+template <int VEC>
 __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ PrArgs a) {
   __shared__ WarpScratch wsm[kWarps];
-  __shared__ PrPushBin::Src fsrc_raw[kWarps][32];
+  __shared__ PrPush::Src fsrc[kWarps][32];
   __shared__ double red[kWarps];
   const int warp = threadIdx.x >> 5;
   const unsigned lane = lane_id();
@@ -244,37 +150,10 @@ __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ 
     if (blockIdx.x == 0 && threadIdx.x < kQueues) a.sets[(it + 2) % 3].tk[threadIdx.x].v = 0ull;
     if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->D[(it + 2) % 3] = 0.0;
     // push phase over the resident log
-    if constexpr (BIN) {
-      PrPushBin f;
-      f.a = &a;
-      const long long gw = tid >> 5;
-      f.wpos = a.wpos + gw * a.nbin;
-      f.wend = a.wend + gw * a.nbin;
-      consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &wsm[warp], fsrc_raw[warp], a.vec_ok);
-      // close this warp's open chunks: pad [wpos, wend) with -1 and reset the chunk state
-      __syncwarp();
-      for (int b = 0; b < a.nbin; ++b) {
-        const unsigned p0 = f.wpos[b], p1 = f.wend[b];
-        for (unsigned i = p0 + lane; i < p1; i += 32) a.ev[a.bstart[b] + i] = -1;
-        __syncwarp();
-        if (lane == 0) f.wpos[b] = f.wend[b] = 0u;
-      }
-      grid_barrier(&a.ctl->bar);
-      // apply the far contributions bin by bin (all warps on the same bin: its y block stays in L2)
-      for (int b = 0; b < a.nbin; ++b) {
-        const long long s0 = a.bstart[b], cnt = (long long)ldcg(a.bfill + b);
-        for (long long i = tid; i < cnt; i += stride) {
-          const int v = ldcg(a.ev + s0 + i);
-          if (v >= 0) atomicAdd(a.y + v, ldcg(a.ec + s0 + i));
-        }
-      }
-    } else {
-      PrPush f;
-      f.x = a.x;
-      f.y = a.y;
-      consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &wsm[warp],
-                       reinterpret_cast<PrPush::Src *>(fsrc_raw[warp]), a.vec_ok);
-    }
+    PrPush f;
+    f.x = a.x;
+    f.y = a.y;
+    consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &wsm[warp], fsrc[warp], a.vec_ok);
     // dangling mass of this iteration's x
     double dsum = 0.0;
     for (long long i = tid; i < a.n_dangling; i += stride) dsum += ldcg(a.x + a.dangling[i]);
@@ -295,7 +174,6 @@ __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ 
       a.x[v] = add + a.d * yv;
       a.y[v] = 0.0;
     }
-    if (BIN && tid < a.nbin) a.bfill[tid] = 0ull;   // every bin was applied before the barrier above
     grid_barrier(&a.ctl->bar);
   }
 }
@@ -351,26 +229,8 @@ __global__ void k_pr_init_c(const long long *__restrict__ off, float *c, long lo
   }
 }
 
-void free_pr_bins(sage_graph *g) {
-  PageRankState &p = g->pr;
-  dfree(g, p.bstart);
-  dfree(g, p.bfill);
-  dfree(g, p.ev);
-  dfree(g, p.ec);
-  dfree(g, p.wpos);
-  dfree(g, p.wend);
-  p.bstart = nullptr;
-  p.bfill = nullptr;
-  p.ev = nullptr;
-  p.ec = nullptr;
-  p.wpos = p.wend = nullptr;
-  p.bin_lg = p.nbin = 0;
-  p.bin_warps = 0;
-}
-
 void free_pagerank_state(sage_graph *g) {
   PageRankState &p = g->pr;
-  free_pr_bins(g);
   free_queues(g, &p.q);
   dfree(g, p.dangling);
   dfree(g, p.x);
@@ -398,7 +258,6 @@ sage_status ensure_pagerank_log(sage_graph *g) {
     free_pagerank_state(g);
     return s;
   }
-  free_pr_bins(g);   // capacities follow the labels (rebuilt after sage_reorder)
   unsigned long long *nd = reinterpret_cast<unsigned long long *>(p.cs + 3);
   cudaMemsetAsync(p.cs, 0, sizeof(CounterSet) * 3 + 64, g->stream);
   k_build_log<<<g->num_sms * 8, 256, 0, g->stream>>>((const long long *)g->off, n, g->ladder,
@@ -415,53 +274,6 @@ sage_status ensure_pagerank_log(sage_graph *g) {
   for (int i = 0; i < kQueues; ++i) p.cnt[i] = h.cnt[i].v;
   p.n_dangling = (long long)hnd;
   p.valid = true;
-  return SAGE_OK;
-}
-
-// Binned-push state (see PrPushBin): per-bin capacities from the static far-arc counts (one pass
-// over col per graph), entry arrays, and the per-(warp, bin) chunk state.  Rebuilt with the log.
-static sage_status ensure_pr_bins(sage_graph *g, long long nwarps) {
-  PageRankState &p = g->pr;
-  if (p.bin_lg && p.bin_warps == nwarps) return SAGE_OK;
-  free_pr_bins(g);
-  int lg = 20;
-  if (const char *e = getenv("SAGE_PR_BIN_LG")) lg = std::max(10, std::min(30, atoi(e)));
-  const long long n = g->n_local;
-  const int nbin = (int)(((n > 0 ? n - 1 : 0) >> lg) + 1);
-  sage_status s;
-  unsigned long long *cnt = nullptr;
-  if ((s = dalloc(g, (void **)&cnt, sizeof(unsigned long long) * (size_t)nbin)) != SAGE_OK) return s;
-  cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * (size_t)nbin, g->stream);
-  k_far_count<<<g->num_sms * 4, 256, sizeof(unsigned long long) * (size_t)nbin, g->stream>>>(
-      (const long long *)g->off, g->col, n, lg, nbin, cnt);
-  std::vector<unsigned long long> h((size_t)nbin);
-  cudaMemcpyAsync(h.data(), cnt, sizeof(unsigned long long) * (size_t)nbin, cudaMemcpyDeviceToHost, g->stream);
-  cudaError_t e = cudaStreamSynchronize(g->stream);
-  dfree(g, cnt);
-  if (e != cudaSuccess) return cuda_fail(g, e, "PageRank bins");
-  std::vector<long long> bs((size_t)nbin);
-  long long tot = 0;
-  for (int b = 0; b < nbin; ++b) {
-    bs[(size_t)b] = tot;
-    tot += (long long)h[(size_t)b] + nwarps * kPrChunk;   // + one partial chunk per warp
-  }
-  if ((s = dalloc(g, (void **)&p.bstart, sizeof(long long) * (size_t)nbin)) != SAGE_OK ||
-      (s = dalloc(g, (void **)&p.bfill, sizeof(unsigned long long) * (size_t)nbin)) != SAGE_OK ||
-      (s = dalloc(g, (void **)&p.ev, sizeof(int) * (size_t)tot)) != SAGE_OK ||
-      (s = dalloc(g, (void **)&p.ec, sizeof(double) * (size_t)tot)) != SAGE_OK ||
-      (s = dalloc(g, (void **)&p.wpos, sizeof(unsigned) * (size_t)(nwarps * nbin))) != SAGE_OK ||
-      (s = dalloc(g, (void **)&p.wend, sizeof(unsigned) * (size_t)(nwarps * nbin))) != SAGE_OK) {
-    free_pr_bins(g);
-    return s;
-  }
-  cudaMemcpyAsync(p.bstart, bs.data(), sizeof(long long) * (size_t)nbin, cudaMemcpyHostToDevice, g->stream);
-  cudaMemsetAsync(p.wpos, 0, sizeof(unsigned) * (size_t)(nwarps * nbin), g->stream);
-  cudaMemsetAsync(p.wend, 0, sizeof(unsigned) * (size_t)(nwarps * nbin), g->stream);
-  e = cudaStreamSynchronize(g->stream);
-  if (e != cudaSuccess) return cuda_fail(g, e, "PageRank bins");
-  p.bin_lg = lg;
-  p.nbin = nbin;
-  p.bin_warps = nwarps;
   return SAGE_OK;
 }
 
@@ -524,29 +336,11 @@ extern "C" sage_status sage_pagerank_ex(sage_graph *g, double damping, int32_t i
                                                       1.0 / (double)g->n);
     a.c = p.c;
   }
-  // binned push: opt-in (SAGE_PR_BINNED=1; SAGE_PR_BIN_LG = block).  Measured on full C4 (y = 840
-  // MB, 29% far arcs): 82-95 ms per iteration vs 57 ms for the direct form, so it is off by default.
-  bool binned = false;
-  if (!pull && iterations > 0)
-    if (const char *e = getenv("SAGE_PR_BINNED")) binned = atoi(e) != 0;
   if (iterations > 0) {
     const void *fn = pull ? (g->vec == 4 ? (const void *)k_pagerank_pull<4> : (const void *)k_pagerank_pull<1>)
-                   : binned ? (g->vec == 4 ? (const void *)k_pagerank<4, true> : (const void *)k_pagerank<1, true>)
-                            : (g->vec == 4 ? (const void *)k_pagerank<4, false> : (const void *)k_pagerank<1, false>);
-    int *cache = pull ? &g->grid_pr_pull : binned ? &g->grid_pr_bin : &g->grid_pr;
+                          : (g->vec == 4 ? (const void *)k_pagerank<4> : (const void *)k_pagerank<1>);
+    int *cache = pull ? &g->grid_pr_pull : &g->grid_pr;
     const int grid = coop_grid(g, fn, cache);
-    if (binned) {
-      if ((s = ensure_pr_bins(g, grid * (kBlock / 32))) != SAGE_OK) return s;
-      a.bin_lg = p.bin_lg;
-      a.nbin = p.nbin;
-      a.bstart = p.bstart;
-      a.bfill = p.bfill;
-      a.ev = p.ev;
-      a.ec = p.ec;
-      a.wpos = p.wpos;
-      a.wend = p.wend;
-      cudaMemsetAsync(p.bfill, 0, sizeof(unsigned long long) * (size_t)p.nbin, g->stream);
-    }
     void *args[] = {&a};
     if ((s = launch_coop(g, fn, grid, args, "PageRank kernel")) != SAGE_OK) return s;
   }

@@ -37,10 +37,7 @@ struct BfsPush {
   static constexpr bool kWeights = false;
   static constexpr bool kNeedRow = false;
   static constexpr bool kEnqueue = true;
-#ifndef SAGE_BFS_DEFER
-#define SAGE_BFS_DEFER 1
-#endif
-  static constexpr bool kDefer = SAGE_BFS_DEFER != 0;   // contraction deferred to a K2' phase
+  static constexpr bool kDefer = true;   // contraction deferred to a K2' phase
   int *flist = nullptr;                  // deferred frontier list
   unsigned long long *flc = nullptr;     // its slot counter (next level's CounterSet)
   uint32_t *visited;
@@ -89,10 +86,7 @@ struct SsspPush {
   static constexpr bool kWeights = true;
   static constexpr bool kNeedRow = false;
   static constexpr bool kEnqueue = true;
-#ifndef SAGE_SSSP_DEFER
-#define SAGE_SSSP_DEFER 1
-#endif
-  static constexpr bool kDefer = SAGE_SSSP_DEFER != 0;   // contraction deferred (see BfsPush)
+  static constexpr bool kDefer = true;   // contraction deferred to the K2' phase (see BfsPush)
   int *flist = nullptr;
   unsigned long long *flc = nullptr;
   uint32_t *dist;
@@ -100,20 +94,13 @@ struct SsspPush {
   int *overflow;
   const Queues *next_q;
   CounterSet *next_cs;
-  // near-far ordering: improvements at distance >= T go to the far pile instead of the frontier
-  unsigned long long T;
-  uint32_t *infar;      // far-pile membership bitmap
-  int *far;             // far pile being appended to
-  unsigned long long *far_cnt;
-  uint32_t *expd;       // distance at which each vertex was last expanded (near-far only)
 
   __device__ __forceinline__ Src src(bool valid, int u, long long, long long) const {
     // dist[u] may have been lowered by another SM in an earlier iteration: read through L2
-    const uint32_t du = valid ? ldcg(dist + u) : 0xffffffffu;
-    if (valid && expd) expd[u] = du;
-    return Src{du};
+    return Src{valid ? ldcg(dist + u) : 0xffffffffu};
   }
 
+  // nd = dist[u] + w(u,v); if nd < dist[v]: dist[v] = nd and v enters the next frontier
   template <int N>
   __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N],
                                         const uint32_t (&w)[N], bool (&in)[N], int) const {
@@ -128,17 +115,10 @@ struct SsspPush {
       if (valid && nd >= 0xffffffffull) {
         if (s.du != 0xffffffffu) *overflow = 1;  // possible overflow: resolved after the traversal
       } else if (valid && nd < cur[j]) {
-        {
-          const uint32_t old = atomicMin(dist + v[j], (uint32_t)nd);
-          if ((uint32_t)nd < old) {
-            const uint32_t bit = 1u << (v[j] & 31);
-            if (nd < T) {
-              const uint32_t o2 = atomicOr(inq_next + (v[j] >> 5), bit);
-              in[j] = !(o2 & bit);
-            } else if (!(atomicOr(infar + (v[j] >> 5), bit) & bit)) {
-              far[atomicAdd(far_cnt, 1ull)] = v[j];
-            }
-          }
+        const uint32_t old = atomicMin(dist + v[j], (uint32_t)nd);
+        if ((uint32_t)nd < old) {
+          const uint32_t bit = 1u << (v[j] & 31);
+          in[j] = !(atomicOr(inq_next + (v[j] >> 5), bit) & bit);
         }
       }
     }
@@ -169,7 +149,6 @@ struct TravArgs {
   struct TailSmem *tailmem;   // tail mode state (global scratch: only block 0 uses it)
   int steal;            // 0 = ablation: static tile assignment instead of stealing
   int *flist;           // deferred contraction: frontier list (n + slack entries)
-  unsigned long long defer_min_arcs;   // defer only on levels with arcs(F) >= this
 };
 
 // Pull (bottom-up) step over the visited bitmap: one warp per 32-vertex word.
@@ -469,9 +448,6 @@ __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
 }
 
 // ============================================================================ BFS kernel
-#ifndef SAGE_BFS_VEC8
-#define SAGE_BFS_VEC8 0   // push BFS with 8 neighbours per lane per step (more loads in flight)
-#endif
 template <int VEC>
 #ifndef SAGE_BFS_MINB
 #define SAGE_BFS_MINB 4
@@ -504,7 +480,7 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
       f.v_base = 0;
       f.next_q = &a.q[(L + 1) & 1];
       f.next_cs = nxt;
-      f.flist = (!SAGE_DEFER_RUNTIME || ldcg(&cur->arcsF.v) >= a.defer_min_arcs) ? a.flist : nullptr;
+      f.flist = a.flist;
       f.flc = &nxt->flc.v;
 #ifdef SAGE_PROF
       const unsigned long long pt0 = globaltimer();
@@ -527,7 +503,7 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
     }
     if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
     grid_barrier(&ctl->bar);
-    if (BfsPush::kDefer && classify_deferred(a.off, a.flist, &nxt->flc.v, a.L, a.q[(L + 1) & 1], nxt))
+    if (classify_deferred(a.off, a.flist, &nxt->flc.v, a.L, a.q[(L + 1) & 1], nxt))
       grid_barrier(&ctl->bar);
     const unsigned long long nF = ldcg(&nxt->nF.v);
     const unsigned long long aF = ldcg(&nxt->arcsF.v);
@@ -566,331 +542,9 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
   }
 }
 
-// ============================================================================ binned push BFS
-// B200 restructuring of the push filter: a scattered 4-B status read costs about one
-// L1TEX cycle per SM from L2-resident global memory but ~0.2 from shared memory (measured,
-// tools/micro/status_reads.cu).  A push level therefore runs in two phases:
-//   phase 1: the unchanged TP + RTS expansion; every neighbour id is stored into the bin of its
-//            vertex slice (1M ids = 128 KB of bitmap), in a chunk reserved per (warp, slice);
-//   phase 2: each CTA stages the visited bits of one slice in shared memory and runs Alg. 1's
-//            filter on its share of that slice's bin; a vertex new to the CTA is claimed with a
-//            global atomicOr (other CTAs of the slice), and filtered-in vertices are classified
-//            into the next level's log exactly as before.
-constexpr int kBinBlock = 1024;
-constexpr int kBinWarps = kBinBlock / 32;
-constexpr int kMaxSlices = 40;
-constexpr int kSliceLg = 20;         // 2^20 vertices per slice
-constexpr int kBinRes = 512;         // entries reserved per (warp, slice) with one atomic
-
-struct BinArgs {
-  int *bins;                         // nslices x cap
-  long long cap;
-  PaddedCounter *fill;               // [2][kMaxSlices]
-  int nslices;
-  int slice_lg;
-};
-
-struct BinPush {
-  struct Src {
-    int u;
-  };
-  static constexpr bool kWeights = false;
-  static constexpr bool kNeedRow = false;
-  static constexpr bool kEnqueue = false;
-  const Queues *next_q = nullptr;
-  CounterSet *next_cs = nullptr;
-  // phase-1 context
-  const TravArgs *a;
-  const BinArgs *b;
-  int *rpos, *rend;                  // this warp's reserved bin range per slice
-  int fillset;
-  int next_level;
-  int nbits;                         // bits of a slice id
-  const Queues *qn;
-  CounterSet *csn;
-  __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
-
-  // end of phase 1: pad the unused part of every reservation
-  __device__ __forceinline__ void close_reservations() const {
-    const unsigned lane = lane_id();
-    for (int s = 0; s < b->nslices; ++s) {
-      const int pos = rpos[s], end = rend[s];
-      for (int i = pos + (int)lane; i < end; i += 32) b->bins[(long long)s * b->cap + i] = -1;
-    }
-  }
-
-  // Warp multi-split of 32 ids into their slices without staging: lanes of one slice are found
-  // with one ballot per slice-id bit, ranked with popc, and stored straight into this warp's
-  // reserved chunk of the slice's bin (one global atomic per kBinRes ids and slice).
-  __device__ __forceinline__ void append(bool valid, int v) const {
-    const unsigned lane = lane_id();
-    const int sl = valid ? (v >> b->slice_lg) : 0;
-    unsigned grp = __ballot_sync(FULL, valid);
-    if (!grp) return;
-#pragma unroll
-    for (int bit = 0; bit < 6; ++bit) {
-      if (bit < nbits) {
-        const bool on = (sl >> bit) & 1;
-        const unsigned bb = __ballot_sync(FULL, on);
-        grp &= on ? bb : ~bb;
-      }
-    }
-    const unsigned lt = lanemask_lt();
-    const int rank = __popc(grp & lt), c = __popc(grp);
-    const bool leader = valid && rank == 0;
-    int pos = valid ? rpos[sl] : 0;
-    const int end = valid ? rend[sl] : 0;
-    unsigned nm = __ballot_sync(FULL, leader && end - pos < c);
-    while (nm) {   // new reservation for the slices whose chunk is too small (rare)
-      const int ld = __ffs(nm) - 1;
-      nm &= nm - 1;
-      const int s2 = __shfl_sync(FULL, sl, ld);
-      const int p2 = rpos[s2], e2 = rend[s2];
-      for (int i = p2 + (int)lane; i < e2; i += 32) b->bins[(long long)s2 * b->cap + i] = -1;
-      unsigned long long np = 0;
-      if (lane == 0) np = atomicAdd(&b->fill[fillset * kMaxSlices + s2].v, (unsigned long long)kBinRes);
-      np = shfl64(np, 0);
-      __syncwarp();
-      if (lane == 0) {
-        rpos[s2] = (int)min(np, (unsigned long long)b->cap);
-        rend[s2] = (int)min(np + kBinRes, (unsigned long long)b->cap);
-      }
-      __syncwarp();
-    }
-    pos = valid ? rpos[sl] : 0;
-    const bool fits = valid && pos + c <= rend[sl];
-    if (fits) b->bins[(long long)sl * b->cap + pos + rank] = v;
-    __syncwarp();
-    if (leader && fits) rpos[sl] = pos + c;
-    __syncwarp();
-    // bin capacity exhausted (skewed ids): Alg. 1's filter on the global bitmap directly
-    const bool direct = valid && !fits;
-    if (__any_sync(FULL, direct)) {
-      bool disc = false;
-      if (direct) {
-        const uint32_t bit = 1u << (v & 31);
-        disc = !(atomicOr(a->visited + (v >> 5), bit) & bit);
-        if (disc) {
-          a->level[v] = next_level;
-          if (a->do_enabled) atomicOr(a->fb[next_level % 3] + (v >> 5), bit);
-        }
-      }
-      enqueue_ids(disc, v, a->off, a->L, *qn, csn);
-    }
-  }
-
-  template <int N>
-  __device__ __forceinline__ void visit(bool valid, const Src &, int (&v)[N], const uint32_t (&)[N],
-                                        bool (&in)[N], int) const {
-#pragma unroll
-    for (int j = 0; j < N; ++j) {
-      in[j] = false;
-      append(valid, v[j]);
-    }
-  }
-};
-
-// phase 2: Alg. 1's filter against a shared-memory copy of one slice of the visited bitmap
-__device__ __forceinline__ void bin_check(const TravArgs &a, const BinArgs &b, int fillset, int L,
-                                          uint32_t *sbm, WarpScratch *ws, const Queues &Qn,
-                                          CounterSet *csn) {
-  const unsigned lane = lane_id();
-  const int warp = threadIdx.x >> 5;
-  const int nw = blockDim.x >> 5;
-  const int ns = b.nslices;
-  int bcnt = 0;
-  uint32_t *fbn = a.do_enabled ? a.fb[(L + 1) % 3] : nullptr;
-  const int G = gridDim.x;
-  const int first = (int)blockIdx.x % ns;
-  const int nparts = G >= ns ? (G - first + ns - 1) / ns : 1;
-  const int part = G >= ns ? (int)blockIdx.x / ns : 0;
-  for (int s = first; s < ns; s += (G >= ns ? ns : G)) {
-    const long long v0 = (long long)s << b.slice_lg;
-    const long long v1 = min(a.n, v0 + (1ll << b.slice_lg));
-    const long long nwd = (v1 - v0 + 31) >> 5;
-    for (long long i = threadIdx.x; i < nwd; i += blockDim.x) sbm[i] = ldcg(a.visited + (v0 >> 5) + i);
-    __syncthreads();
-    const long long fill = (long long)ldcg(&b.fill[fillset * kMaxSlices + s].v);
-    const long long tot = fill < b.cap ? fill : b.cap;
-    const long long lo = tot * part / nparts, hi = tot * (part + 1) / nparts;
-    const int *bin = b.bins + (long long)s * b.cap;
-    for (long long base = lo + (long long)warp * 128; base < hi; base += (long long)nw * 128) {
-      int vv[4];
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const long long i = base + j * 32 + lane;
-        vv[j] = i < hi ? ldcg(bin + i) : -1;
-      }
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int v = vv[j];
-        bool disc = false;
-        if (v >= 0) {
-          const int lb = (int)(v - v0);
-          const uint32_t bit = 1u << (lb & 31);
-          if (!(sbm[lb >> 5] & bit)) {
-            if (!(atomicOr(sbm + (lb >> 5), bit) & bit)) {
-              disc = !(atomicOr(a.visited + (v >> 5), bit) & bit);
-              if (disc) {
-                a.level[v] = L + 1;
-                if (fbn) atomicOr(fbn + (v >> 5), bit);
-              }
-            }
-          }
-        }
-        buffer_push(disc, v, &ws[warp], bcnt, a.off, a.L, Qn, csn);
-      }
-    }
-    __syncthreads();
-  }
-  if (bcnt) buffer_flush(&ws[warp], bcnt, a.off, a.L, Qn, csn);
-}
-
-template <int VEC>
-__global__ void __launch_bounds__(kBinBlock, 1) k_bfs_bin(const __grid_constant__ TravArgs a,
-                                                          const __grid_constant__ BinArgs b) {
-  extern __shared__ __align__(16) unsigned char dsm[];
-  WarpScratch *wsm = reinterpret_cast<WarpScratch *>(dsm);
-  BinPush::Src *fsrc = reinterpret_cast<BinPush::Src *>(dsm + sizeof(WarpScratch) * kBinWarps);
-  int *rps = reinterpret_cast<int *>(dsm + sizeof(WarpScratch) * kBinWarps + sizeof(BinPush::Src) * 32 * kBinWarps);
-  int *res = rps + kMaxSlices * kBinWarps;
-  unsigned char *U = dsm + sizeof(WarpScratch) * kBinWarps + sizeof(BinPush::Src) * 32 * kBinWarps +
-                     2 * sizeof(int) * kMaxSlices * kBinWarps;
-  const int warp = threadIdx.x >> 5;
-  const unsigned lane = lane_id();
-  Ctl *ctl = a.ctl;
-  double mU = (double)a.m - (double)ldcg(&ctl->set[0].arcsF.v);
-  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t0_ns = globaltimer();
-  int dir = 0;
-  unsigned long long prev_nF = 1;
-  const long long nwords = (a.n + 31) >> 5;
-  for (int L = 0;; ++L) {
-    CounterSet *cur = &ctl->set[L % 3];
-    CounterSet *nxt = &ctl->set[(L + 1) % 3];
-    __syncthreads();
-    zero_counterset(&ctl->set[(L + 2) % 3]);
-    if (blockIdx.x == 0 && threadIdx.x < kMaxSlices) b.fill[((L + 1) & 1) * kMaxSlices + threadIdx.x].v = 0ull;
-    if (a.do_enabled) clear_words(a.fb[(L + 2) % 3], nwords);
-    if (dir == 0) {
-      // phase 1: expansion into slice bins
-      for (int i = lane; i < b.nslices; i += 32) {
-        rps[warp * kMaxSlices + i] = 0;
-        res[warp * kMaxSlices + i] = 0;
-      }
-      __syncwarp();
-      BinPush f;
-      f.a = &a;
-      f.b = &b;
-      f.rpos = rps + warp * kMaxSlices;
-      f.rend = res + warp * kMaxSlices;
-      f.fillset = L & 1;
-      f.next_level = L + 1;
-      f.nbits = 0;
-      while ((1 << f.nbits) < b.nslices) ++f.nbits;
-      f.qn = &a.q[(L + 1) & 1];
-      f.csn = nxt;
-      consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc + warp * 32, a.vec_ok);
-      f.close_reservations();
-      grid_barrier(&ctl->bar);
-      if (blockIdx.x == 0 && threadIdx.x == 0 && L < kMaxRec)
-        ctl->rec[L].t_mid_us = (int)((globaltimer() - ctl->t0_ns) / 1000);
-      // phase 2: filter against shared-memory slices of the visited bitmap
-      bin_check(a, b, L & 1, L, reinterpret_cast<uint32_t *>(U), wsm, a.q[(L + 1) & 1], nxt);
-    } else {
-      pull_level(a, L + 1, a.fb[L % 3], a.fb[(L + 1) % 3], a.q[(L + 1) & 1], cur, nxt, &wsm[warp]);
-    }
-    if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
-    grid_barrier(&ctl->bar);
-    const unsigned long long nF = ldcg(&nxt->nF.v);
-    const unsigned long long aF = ldcg(&nxt->arcsF.v);
-    if (blockIdx.x == 0 && threadIdx.x == 0) record_level(ctl, L, dir, cur, nxt);
-    if (nF == 0) break;
-    if (L + 1 >= a.max_levels) {
-      if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = 1;
-      break;
-    }
-    mU -= (double)aF;
-    if (a.do_enabled) {
-      if (dir == 0) {
-        if ((double)aF > mU / a.alpha) dir = 1;
-      } else {
-        if (!(nF >= prev_nF || (double)nF > (double)a.n / a.beta)) dir = 0;
-      }
-    }
-    prev_nF = nF;
-  }
-}
-
-static size_t bin_smem_bytes(int nslices, long long n) {
-  const size_t fixed = sizeof(WarpScratch) * kBinWarps + sizeof(int) * 32 * kBinWarps +
-                       2 * sizeof(int) * kMaxSlices * kBinWarps;
-  const long long sw = std::min<long long>(n, 1ll << kSliceLg);
-  const size_t bm = sizeof(uint32_t) * (size_t)((sw + 31) / 32 + 1);
-  (void)nslices;
-  return fixed + bm;
-}
-
 // ============================================================================ SSSP kernel
-struct FarArgs {                      // near-far state of k_sssp
-  int *far[3];                       // three rotating far piles (append / scan / spare)
-  uint32_t *infar;                   // far-pile membership bitmap
-  uint32_t *expd;                    // last expanded distance per vertex (stale far entries)
-  PaddedCounter *cnt;                // [3] far pile sizes
-  PaddedCounter *fmin;               // [3] min distance seen in a scan
-  unsigned long long delta;          // threshold step; 0xffff... = plain Bellman-Ford
-};
-
-// Advance phase of near-far SSSP: move far-pile vertices with dist < T into the next log.
-__device__ __forceinline__ void far_scan(const TravArgs &a, const FarArgs &fa, int k, unsigned long long T,
-                                         uint32_t *inq_next, const Queues &Qn, CounterSet *csn,
-                                         WarpScratch *ws) {
-  const unsigned lane = lane_id();
-  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
-  const int *src = fa.far[k % 3];
-  int *dst = fa.far[(k + 1) % 3];
-  const long long cnt = (long long)ldcg(&fa.cnt[k % 3].v);
-  unsigned long long mn = ~0ull;
-  int bcnt = 0;
-  for (long long base = gw * 32; base < cnt; base += nw * 32) {
-    const long long i = base + lane;
-    bool move = false, keep = false;
-    int v = 0;
-    if (i < cnt) {
-      v = ldcg(src + i);
-      const uint32_t d = ldcg(a.dist + v);
-      const uint32_t bit = 1u << (v & 31);
-      if (d < T) {
-        atomicAnd(fa.infar + (v >> 5), ~bit);
-        // skip entries whose vertex was already expanded at its current distance
-        move = ldcg(fa.expd + v) != d && !(atomicOr(inq_next + (v >> 5), bit) & bit);
-      } else {
-        keep = true;
-        if (d < mn) mn = d;
-      }
-    }
-    const unsigned km = __ballot_sync(FULL, keep);
-    if (km) {
-      const int leader = __ffs(km) - 1;
-      unsigned long long p = 0;
-      if ((int)lane == leader) p = atomicAdd(&fa.cnt[(k + 1) % 3].v, (unsigned long long)__popc(km));
-      p = shfl64(p, leader);
-      if (keep) dst[p + __popc(km & lanemask_lt())] = v;
-    }
-    buffer_push(move, v, ws, bcnt, a.off, a.L, Qn, csn);
-  }
-  if (bcnt) buffer_flush(ws, bcnt, a.off, a.L, Qn, csn);
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    const unsigned long long y = __shfl_xor_sync(FULL, mn, o);
-    mn = y < mn ? y : mn;
-  }
-  if (lane == 0 && mn != ~0ull) atomicMin(&fa.fmin[k % 3].v, mn);
-}
-
 template <int VEC>
-__global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ TravArgs a, int *overflow,
-                                                    const __grid_constant__ FarArgs fa) {
+__global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ TravArgs a, int *overflow) {
   __shared__ WarpScratch wsm[kWarps];
   __shared__ SsspPush::Src fsrc[kWarps][32];
   const int warp = threadIdx.x >> 5;
@@ -898,8 +552,6 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
   const long long nwords = (a.n + 31) >> 5;
   if ((threadIdx.x & 31) == 0) wsm[warp].cpos = wsm[warp].cend = 0;
   if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t0_ns = globaltimer();
-  unsigned long long T = fa.delta;   // near threshold
-  int k = 0;                         // far scans done; the current far pile is far[k % 3]
   for (int L = 0;; ++L) {
     CounterSet *cur = &ctl->set[L % 3];
     CounterSet *nxt = &ctl->set[(L + 1) % 3];
@@ -912,33 +564,14 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
     f.overflow = overflow;
     f.next_q = &a.q[(L + 1) & 1];
     f.next_cs = nxt;
-    f.T = T;
-    f.infar = fa.infar;
-    f.far = fa.far[k % 3];
-    f.far_cnt = &fa.cnt[k % 3].v;
-    f.expd = fa.delta == ~0ull ? nullptr : fa.expd;
-    f.flist = (!SAGE_DEFER_RUNTIME || ldcg(&cur->arcsF.v) >= a.defer_min_arcs) ? a.flist : nullptr;
+    f.flist = a.flist;
     f.flc = &nxt->flc.v;
     consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok);
     if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
     grid_barrier(&ctl->bar);
-    if (SsspPush::kDefer && classify_deferred(a.off, a.flist, &nxt->flc.v, a.L, a.q[(L + 1) & 1], nxt))
+    if (classify_deferred(a.off, a.flist, &nxt->flc.v, a.L, a.q[(L + 1) & 1], nxt))
       grid_barrier(&ctl->bar);
-    unsigned long long nF = ldcg(&nxt->nF.v);
-    // near frontier exhausted: raise the threshold and pull the far pile forward
-    while (nF == 0 && ldcg(&fa.cnt[k % 3].v) != 0) {
-      if (blockIdx.x == 0 && threadIdx.x == 0) {
-        fa.cnt[(k + 2) % 3].v = 0ull;     // scan k-1's source pile, no longer read
-        fa.fmin[(k + 1) % 3].v = ~0ull;   // written by scan k+1, not read before it
-      }
-      const unsigned long long fm = k > 0 ? ldcg(&fa.fmin[(k + 2) % 3].v) : ~0ull;  // scan k-1's
-      T = (T + fa.delta > T) ? T + fa.delta : ~0ull;
-      if (fm != ~0ull && fm >= T) T = (fm / fa.delta + 1) * fa.delta;   // skip empty buckets
-      far_scan(a, fa, k, T, a.fb[(L + 1) % 3], a.q[(L + 1) & 1], nxt, &wsm[warp]);
-      grid_barrier(&ctl->bar);
-      ++k;
-      nF = ldcg(&nxt->nF.v);
-    }
+    const unsigned long long nF = ldcg(&nxt->nF.v);
     if (blockIdx.x == 0 && threadIdx.x == 0) record_level(ctl, L, 0, cur, nxt);
     if (nF == 0) break;
     if (L + 1 >= a.max_levels) {
@@ -1114,13 +747,7 @@ void free_traversal_state(sage_graph *g) {
   free_queues(g, &t.q[1]);
   dfree(g, t.ctl);
   dfree(g, t.tmp_out);
-  dfree(g, t.bins);
-  dfree(g, t.fill);
-  for (int i = 0; i < 3; ++i) dfree(g, t.far[i]);
   dfree(g, t.tailmem);
-  dfree(g, t.expd);
-  dfree(g, t.infar);
-  dfree(g, t.farc);
   dfree(g, t.flist);
   t = TraversalState();
 }
@@ -1165,31 +792,29 @@ sage_status ensure_traversal_state(sage_graph *g) {
 int coop_grid(sage_graph *g, const void *fn, int *cache) {
   if (*cache) return *cache;
   // shared-memory carveout: the persistent kernels use <= 10 KB of shared memory per CTA; the rest
-  // of the SM's 256 KB goes to L1, which caches status words and row offsets (SAGE_CARVEOUT = %)
-  // (measured on C2 push BFS: driver default 3.40 ms, smallest carveout for 4 CTAs 3.15 ms)
-  {
-    const char *e = getenv("SAGE_CARVEOUT");
-    int pct = e ? atoi(e) : -1;
-    if (!e) {   // smallest carveout that still holds kMinBlocks CTAs (+1 KB reserved per CTA)
-      cudaFuncAttributes fa;
-      if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) {
-        int dev = 0, smem_sm = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
-        const size_t need = 4 * (fa.sharedSizeBytes + 1024);
-        if (smem_sm > 0) pct = (int)std::min<size_t>(100, (need * 100 + smem_sm - 1) / smem_sm);
-      }
-    }
-    if (pct >= 0) cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
-  }
+  // of the SM's 256 KB goes to L1, which caches status words and row offsets.  The smallest
+  // carveout that still holds the occupancy limit's CTAs (+1 KB reserved per CTA) is requested
+  // (measured on C2 push BFS: driver default 3.40 ms, smallest carveout 3.15 ms).
   int nb = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, kBlock, 0);
   if (nb < 1) nb = 1;
+  {
+    cudaFuncAttributes fa;
+    if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) {
+      int smem_sm = 0;
+      cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, g->device);
+      const size_t need = (size_t)nb * (fa.sharedSizeBytes + 1024);
+      if (smem_sm > 0) {
+        const int pct = (int)std::min<size_t>(100, (need * 100 + smem_sm - 1) / smem_sm);
+        cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+      }
+    }
+  }
+  const int nb_occ = nb;
   // small graphs (C1: 1.8M arcs, L2-resident) are latency-bound per level: one CTA per SM halves
   // the grid barrier's participants and the counter traffic (C1 DO BFS 156 -> 135 us measured)
-  const int nb_occ = nb;
   if (g->m < (8ll << 20)) nb = 1;
-  if (const char *e = getenv("SAGE_CTAS_PER_SM")) nb = std::max(1, std::min(nb_occ, atoi(e)));
+  if (g->ctas_per_sm > 0) nb = std::max(1, std::min(nb_occ, g->ctas_per_sm));
   *cache = nb * g->num_sms;
   return *cache;
 }
@@ -1248,12 +873,9 @@ static TravArgs make_args(sage_graph *g) {
   a.alpha = g->alpha;
   a.beta = g->beta;
   a.max_levels = (int)std::min<long long>(g->n + 1, 0x7fffffffll);
-  if (const char *e = getenv("SAGE_DEBUG_MAX_LEVELS")) a.max_levels = atoi(e);   // diagnostics only
   a.tail = (int *)g->ts.tmp_out;
   a.tailmem = reinterpret_cast<TailSmem *>(g->ts.tailmem);
   a.flist = g->ts.flist;
-  a.defer_min_arcs = 1ull << 16;   // SAGE_DEFER_MIN_ARCS overrides (tests: 0 = every level)
-  if (const char *e = getenv("SAGE_DEFER_MIN_ARCS")) a.defer_min_arcs = strtoull(e, nullptr, 10);
   a.steal = 1;
   a.vec_ok = g->vec_ok ? 1 : 0;
   return a;
@@ -1346,41 +968,9 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   a.do_enabled = (symmetric && !push_only) ? 1 : 0;
   a.steal = (call_flags & SAGE_F_NO_STEALING) ? 0 : 1;
   k_seed<<<1, 32, 0, g->stream>>>(a, src, 0);
-  const int nslices = (int)((g->n + (1ll << kSliceLg) - 1) >> kSliceLg);
-  const bool binned = !parent_out && (call_flags & SAGE_F_BINNED) && nslices <= kMaxSlices;
-  if (binned && !t.bins) {
-    // per-slice capacity: 1.5x the average share of all arcs plus staging slack; a full bin
-    // spills to the direct filter, so the capacity only affects speed
-    t.nslices = nslices;
-    t.bin_cap = (long long)(1.5 * (double)g->m / nslices) + (long long)kBinRes * kBinWarps * g->num_sms + 1024;
-    if ((s = dalloc(g, (void **)&t.bins, sizeof(int) * (size_t)t.bin_cap * nslices)) != SAGE_OK ||
-        (s = dalloc(g, (void **)&t.fill, sizeof(PaddedCounter) * 2 * kMaxSlices)) != SAGE_OK)
-      return s;
-  }
-  if (binned) cudaMemsetAsync(t.fill, 0, sizeof(PaddedCounter) * 2 * kMaxSlices, g->stream);
   cudaEventRecord(e1, g->stream);
-  if (binned) {
-    BinArgs b;
-    b.bins = t.bins;
-    b.cap = t.bin_cap;
-    b.fill = t.fill;
-    b.nslices = nslices;
-    b.slice_lg = kSliceLg;
-    const void *fn = g->vec == 4 ? (const void *)k_bfs_bin<4> : (const void *)k_bfs_bin<1>;
-    const size_t smem = bin_smem_bytes(nslices, g->n);
-    cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (!g->grid_bin) {
-      int nb = 0;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, kBinBlock, smem);
-      g->grid_bin = std::max(1, nb) * g->num_sms;
-    }
-    void *args[] = {&a, &b};
-    cudaError_t le = cudaLaunchCooperativeKernel(fn, dim3(g->grid_bin), dim3(kBinBlock), args, smem, g->stream);
-    if (le != cudaSuccess) return cuda_fail(g, le, "binned BFS kernel");
-  } else {
-    static const int bfs_vec8 = getenv("SAGE_BFS_VEC") ? atoi(getenv("SAGE_BFS_VEC")) == 8 : SAGE_BFS_VEC8;
-    const void *fn = g->vec == 4 ? (bfs_vec8 && g->ladder.M >= 8 ? (const void *)k_bfs<8> : (const void *)k_bfs<4>)
-                                 : (const void *)k_bfs<1>;
+  {
+    const void *fn = g->vec == 4 ? (const void *)k_bfs<4> : (const void *)k_bfs<1>;
     const int grid = coop_grid(g, fn, &g->grid_bfs);
     void *args[] = {&a};
     if ((s = launch_coop(g, fn, grid, args, "BFS kernel")) != SAGE_OK) return s;
@@ -1396,7 +986,7 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   cudaEventDestroy(e0);
   cudaEventDestroy(e1);
   cudaEventDestroy(e2);
-  if (h.status == 1 && !getenv("SAGE_DEBUG_MAX_LEVELS")) {
+  if (h.status == 1) {
     set_error("BFS exceeded the level cap (internal error)");
     g->sticky = SAGE_E_CUDA;
     return SAGE_E_CUDA;
@@ -1443,52 +1033,12 @@ extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_o
   cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
   for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
   cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);
-  // near-far state (SSSP ordering); delta from the mean weight and degree
-  if (!t.far[0]) {
-    for (int i = 0; i < 3; ++i)
-      if ((s = dalloc(g, (void **)&t.far[i], sizeof(int) * (size_t)(g->n_local + 1))) != SAGE_OK) return s;
-    if ((s = dalloc(g, (void **)&t.infar, sizeof(uint32_t) * words)) != SAGE_OK ||
-        (s = dalloc(g, (void **)&t.farc, sizeof(PaddedCounter) * 6)) != SAGE_OK)
-      return s;
-  }
-  if (g->w_mean <= 0.0) {
-    unsigned long long *dsum = reinterpret_cast<unsigned long long *>(t.farc);
-    unsigned long long hsum = 0;
-    cudaMemsetAsync(dsum, 0, sizeof(unsigned long long), g->stream);
-    k_sum_u32<<<g->num_sms * 8, 256, 0, g->stream>>>(g->w, g->m, dsum);
-    cudaMemcpyAsync(&hsum, dsum, sizeof(hsum), cudaMemcpyDeviceToHost, g->stream);
-    cudaStreamSynchronize(g->stream);
-    g->w_mean = g->m ? (double)hsum / (double)g->m : 1.0;
-  }
-  FarArgs fa;
-  for (int i = 0; i < 3; ++i) fa.far[i] = t.far[i];
-  fa.infar = t.infar;
-  fa.expd = reinterpret_cast<uint32_t *>(t.far[2]) + 0;   // placeholder, set below
-  fa.cnt = t.farc;
-  fa.fmin = t.farc + 3;
-  {
-    const double avgdeg = g->n_local ? (double)g->m / (double)g->n_local : 1.0;
-    double dl = 32.0 * g->w_mean / std::max(1.0, avgdeg);
-    const char *env = getenv("SAGE_SSSP_DELTA");
-    if (env) dl = atof(env);
-    fa.delta = dl <= 0.0 ? ~0ull : (unsigned long long)std::max(1.0, std::floor(dl + 0.5));
-    if (!env) fa.delta = ~0ull;   // default: plain frontier Bellman-Ford (near-far measured slower)
-  }
-  if (fa.delta != ~0ull) {
-    if (!t.expd && (s = dalloc(g, (void **)&t.expd, sizeof(uint32_t) * (size_t)g->n_local)) != SAGE_OK)
-      return s;
-    cudaMemsetAsync(t.expd, 0xff, sizeof(uint32_t) * (size_t)g->n_local, g->stream);
-  }
-  fa.expd = t.expd;
-  cudaMemsetAsync(t.infar, 0, sizeof(uint32_t) * words, g->stream);
-  cudaMemsetAsync(t.farc, 0, sizeof(PaddedCounter) * 3, g->stream);
-  cudaMemsetAsync(t.farc + 3, 0xff, sizeof(PaddedCounter) * 3, g->stream);
   TravArgs a = make_args(g);
   k_seed<<<1, 32, 0, g->stream>>>(a, src, 1);
   cudaEventRecord(e1, g->stream);
   const void *fn = g->vec == 4 ? (const void *)k_sssp<4> : (const void *)k_sssp<1>;
   const int grid = coop_grid(g, fn, &g->grid_sssp);
-  void *args[] = {&a, &ovf, &fa};
+  void *args[] = {&a, &ovf};
   if ((s = launch_coop(g, fn, grid, args, "SSSP kernel")) != SAGE_OK) {
     dfree(g, ovf);
     return s;
@@ -1609,7 +1159,8 @@ extern "C" sage_status sage_debug_export_tiles(sage_graph *g, const int32_t *ver
 
 extern "C" sage_status sage_debug_level_records(const sage_graph *gc, int64_t *rec_out, int32_t cap,
                                                 int32_t *n_out) {
-  // 8 int64 per level (the 8th = device time at which the last warp finished the level's work)
+  // 9 int64 per level (include/sage.h): dir, |F|, arcs(F), inspected, scanned, discovered,
+  // level end, last warp's work end, expansion end (K2' start); times in ns since kernel start
   clear_error();
   sage_graph *g = const_cast<sage_graph *>(gc);
   if (!g || !n_out || (cap > 0 && !rec_out)) {
@@ -1640,7 +1191,7 @@ extern "C" sage_status sage_debug_level_records(const sage_graph *gc, int64_t *r
     o[5] = (int64_t)r.discovered;
     o[6] = (int64_t)(r.t_ns - h->t0_ns);
     o[7] = r.t_work ? (int64_t)(r.t_work - h->t0_ns) : 0;
-    o[8] = (int64_t)r.t_mid_us * 1000;
+    o[8] = r.t_mid ? (int64_t)(r.t_mid - h->t0_ns) : 0;
   }
   delete h;
   return SAGE_OK;

@@ -271,9 +271,9 @@ def test_error_conventions(sage):
         sage.load_csr(g.off, g.col, tile_cta=100)
 
 
-def test_binned_and_direct_push_agree(sage):
-    """The two-phase binned push level (slice bins + shared-memory bitmap slices) and the direct
-    per-arc filter give the oracle's levels, including multi-slice graphs (n > 2^20)."""
+def test_push_parity_multi_slice_and_skewed(sage):
+    """Push and direction-optimising BFS on graphs above 2^20 vertices, and on a skewed graph whose
+    arcs all target the first 2^20 vertices: the oracle's levels."""
     graphs = [sg.rmat(12, 16, seed=21, symmetric=True), sg.rmat(21, 8, seed=22, symmetric=True),
               sg.rmat(21, 8, seed=23, symmetric=False)]
     for g in graphs:
@@ -281,13 +281,8 @@ def test_binned_and_direct_push_agree(sage):
             for s in sg.sources(g, 2, seed=2):
                 ref = oracle.bfs(g.off, g.col, int(s))
                 for po in (True, False):
-                    for binning in (True, False):
-                        lv, _, st = G.bfs(int(s), push_only=po, binning=binning)
-                        assert np.array_equal(lv, ref), (g.name, int(s), po, binning)
-
-
-def test_binned_push_bin_overflow(sage):
-    """Every arc targets the first slice: bins overflow and spill to the direct filter."""
+                    lv, _, st = G.bfs(int(s), push_only=po)
+                    assert np.array_equal(lv, ref), (g.name, int(s), po)
     n = 3 << 20
     rng = np.random.default_rng(5)
     src = rng.integers(0, n, size=400000)
@@ -298,7 +293,7 @@ def test_binned_push_bin_overflow(sage):
     with sage.load_csr(g.off, g.col) as G:
         for s in [int(src[0]), 0]:
             ref = oracle.bfs(g.off, g.col, s)
-            lv, _, _ = G.bfs(s, push_only=True, binning=True)
+            lv, _, _ = G.bfs(s, push_only=True)
             assert np.array_equal(lv, ref)
 
 
@@ -316,13 +311,10 @@ def test_no_stealing_ablation_parity(sage):
         assert np.array_equal(G.bfs(s, push_only=True)[0], oracle.bfs(g.off, g.col, s))
 
 
-@pytest.mark.parametrize("lg", [10, 12])
-def test_pagerank_binned_push_parity(sage, lg, monkeypatch):
-    """Binned push PageRank (far contributions staged per target block) forced on
-    small graphs with small blocks (SAGE_PR_BIN_LG): within 1e-6 of the oracle on directed and
-    symmetric inputs, repeated calls, and after a reorder (bins rebuilt for the new labels)."""
-    monkeypatch.setenv("SAGE_PR_BINNED", "1")
-    monkeypatch.setenv("SAGE_PR_BIN_LG", str(lg))
+def test_pagerank_push_parity_repeat_and_reorder(sage):
+    """Push PageRank (Alg. 1 l.26-29) within 1e-6 of the oracle on directed and symmetric inputs,
+    repeated calls (the resident log is reused) and after a reorder (log rebuilt for the new
+    labels), and on a UK-like (crawl order, tendrils) graph."""
     for sym, seed in ((False, 3), (True, 4)):
         g = sg.rmat(15, 16, seed=seed, symmetric=sym)
         xr = oracle.pagerank(g.off, g.col, 0.85, 20)
@@ -340,13 +332,13 @@ def test_pagerank_binned_push_parity(sage, lg, monkeypatch):
         assert np.max(np.abs(x - xr) / xr) <= 1e-6
 
 
-def test_full_occupancy_grid_on_small_graphs(sage, monkeypatch):
+def test_full_occupancy_grid_on_small_graphs(sage):
     """Small graphs run the persistent kernels with one CTA per SM by default; the full-occupancy
-    grid (4 CTAs per SM, the configuration of the large configs) gives the same answers."""
-    monkeypatch.setenv("SAGE_CTAS_PER_SM", "4")
+    grid (sage_options.ctas_per_sm = 4, the configuration of the large configs) gives the same
+    answers."""
     g = sg.rmat(15, 16, seed=9, symmetric=True)
     w = sg.weights(g, 1)
-    with sage.load_csr(g.off, g.col, w, symmetric=True) as G:
+    with sage.load_csr(g.off, g.col, w, symmetric=True, ctas_per_sm=4) as G:
         for s in sg.sources(g, 4, seed=2):
             ref = oracle.bfs(g.off, g.col, int(s))
             for po in (True, False):
@@ -358,12 +350,8 @@ def test_full_occupancy_grid_on_small_graphs(sage, monkeypatch):
         assert np.max(np.abs(x - xr) / xr) <= 1e-6
 
 
-@pytest.mark.parametrize("min_arcs", ["0", "100000000000"])
-def test_deferred_and_immediate_contraction(sage, min_arcs, monkeypatch):
-    """Push BFS / SSSP with the deferred frontier list + K2' phase; SAGE_DEFER_MIN_ARCS selects
-    immediate contraction on small levels in builds with SAGE_DEFER_RUNTIME=1 (off by default):
-    exact either way."""
-    monkeypatch.setenv("SAGE_DEFER_MIN_ARCS", min_arcs)
+def test_deferred_contraction_every_level(sage):
+    """Push BFS / SSSP with the deferred frontier list + K2' phase on every level: exact."""
     for sym in (True, False):
         g = sg.rmat(14, 16, seed=12, symmetric=sym)
         w = sg.weights(g, 1)

@@ -4,6 +4,8 @@
 # Usage: bash tools/ab.sh <tag> [DEF=VAL ...]
 tag=${1:-ab}; shift
 out=gpurun_out; mkdir -p $out
+# leave the default library in the tree whatever happens (the stamp makes this a real rebuild)
+trap 'python tools/build.py > /dev/null' EXIT
 python tools/build.py > /dev/null || exit 1
 timeout 900 python -m pytest tests -m gpu -q -x > $out/pytest_gpu_$tag.txt 2>&1
 tail -2 $out/pytest_gpu_$tag.txt

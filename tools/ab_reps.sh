@@ -2,6 +2,8 @@
 # Repeated A/B of push-BFS kernel time (median over 3 bench runs per variant, alternating).
 # Usage: bash tools/ab_reps.sh "DEF=VAL[,DEF=VAL]" ...   (first variant = default build)
 out=gpurun_out; mkdir -p $out
+# leave the default library in the tree whatever happens (the stamp makes this a real rebuild)
+trap 'python tools/build.py > /dev/null' EXIT
 build_variant() {
   local d=$1; envs=()
   if [ "$d" != "base" ]; then IFS=',' read -ra kv <<< "$d"; for x in "${kv[@]}"; do envs+=("SAGE_DEF_${x%%=*}=${x#*=}"); done; fi

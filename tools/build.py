@@ -74,6 +74,16 @@ def build_sage(force=False, verbose=False):
             [os.path.join(ROOT, "include", "sage.h")])
     prof = os.environ.get("SAGE_PROF") == "1"
     out = os.path.join(PKG, "libsage_prof.so" if prof else "libsage.so")
+    # compile-time variants (SAGE_DEF_NAME=VALUE -> -DNAME=VALUE, used by the A/B scripts): the
+    # active set is stamped next to the library and its objects, and a different set is stale
+    defs = sorted(f"-D{k[len('SAGE_DEF_'):]}={v}" for k, v in os.environ.items() if k.startswith("SAGE_DEF_"))
+    if prof:
+        defs.append("-DSAGE_PROF=1")
+    stamp = out + ".defs"
+    want = " ".join(defs) + "\n"
+    have = open(stamp).read() if os.path.exists(stamp) else None
+    if have != want:
+        force = True
     if not (force or _stale(out, cus + hdrs)):
         return out
     nccl_inc, nccl_lib = _nccl_paths()
@@ -81,9 +91,7 @@ def build_sage(force=False, verbose=False):
     os.makedirs(objdir, exist_ok=True)
     common = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC",
               "-I", os.path.join(ROOT, "include"), "-I", csrc, "-I", nccl_inc,
-              "--expt-relaxed-constexpr", "-Xptxas", "-v" if verbose else "-O3"] + (["-DSAGE_PROF=1"] if prof else []) + \
-             [f"-D{k}={v}" for k, v in os.environ.items() if k.startswith("SAGE_DEF_")
-              for k in [k[len("SAGE_DEF_"):]]]
+              "--expt-relaxed-constexpr", "-Xptxas", "-v" if verbose else "-O3"] + defs
     objs = []
     for cu in cus:
         obj = os.path.join(objdir, os.path.basename(cu)[:-3] + ".o")
@@ -92,8 +100,12 @@ def build_sage(force=False, verbose=False):
             if verbose:
                 sys.stdout.write(log)
         objs.append(obj)
+    if os.path.exists(stamp):
+        os.remove(stamp)
     _run([NVCC, *ARCH, "-shared", "-o", out, *objs, "-L", nccl_lib, "-l:libnccl.so.2",
           "-Xlinker", "-rpath=" + nccl_lib])
+    with open(stamp, "w") as f:
+        f.write(want)
     return out
 
 

@@ -18,7 +18,6 @@ p.add_argument("--op", default="bfs_push", choices=["bfs_push", "bfs_do", "sssp"
 p.add_argument("--reps", type=int, default=3)
 p.add_argument("--tile-cta", type=int, default=256)
 p.add_argument("--align", type=int, default=4)
-p.add_argument("--binned", action="store_true", help="experimental two-phase binned push level")
 a = p.parse_args()
 if a.graph == "rmat":
     g = sg.rmat(a.scale, 16, 1, True)
@@ -34,9 +33,9 @@ src = sg.sources(g, a.reps, seed=2)
 lv = torch.empty(g.n, dtype=torch.int32, device="cuda")
 for i in range(a.reps):
     if a.op == "bfs_push":
-        _, _, st = G.bfs(int(src[i]), out=lv, push_only=True, binning=a.binned)
+        _, _, st = G.bfs(int(src[i]), out=lv, push_only=True)
     elif a.op == "bfs_do":
-        _, _, st = G.bfs(int(src[i]), out=lv, binning=a.binned)
+        _, _, st = G.bfs(int(src[i]), out=lv)
     elif a.op == "sssp":
         _, st = G.sssp(int(src[i]), out=lv.view(torch.uint32))
     elif a.op == "reorder":

@@ -91,6 +91,9 @@ typedef struct {
   double beta;       /* pull->push threshold: push when |F| < n/beta; default 18                     */
   int32_t ctas_per_sm; /* resident CTAs per SM of the persistent kernels; 0 = automatic (the
                         occupancy limit, one CTA per SM on graphs under 8M arcs)                  */
+  int32_t hub_filter;  /* push BFS hub filter (a shared-memory table of visited
+                        high-degree vertices skips their status reads; results identical):
+                        0 = automatic (graphs with >= 32M arcs), 1 = always, -1 = never        */
 } sage_options;
 
 /* CSR input of sage_load_csr (Fig. 1: u_offset / v arrays).                         */

@@ -166,7 +166,7 @@ static int ilog2(long long x) {
 static bool is_pow2(long long x) { return x > 0 && (x & (x - 1)) == 0; }
 
 static sage_status make_ladder(const sage_options *o, sage_graph *g) {
-  int B = 256, M = 8, A = 4, cps = 0;
+  int B = 256, M = 8, A = 4, cps = 0, hub = 0;
   double alpha = 15.0, beta = 18.0;
   if (o) {
     B = o->tile_cta;
@@ -175,6 +175,11 @@ static sage_status make_ladder(const sage_options *o, sage_graph *g) {
     alpha = o->alpha;
     beta = o->beta;
     cps = o->ctas_per_sm;
+    hub = o->hub_filter;
+  }
+  if (hub < -1 || hub > 1) {
+    set_error("hub_filter must be -1, 0 or 1");
+    return SAGE_E_INVALID;
   }
   if (cps < 0 || cps > 32) {
     set_error("ctas_per_sm must be in [0, 32]");
@@ -204,6 +209,7 @@ static sage_status make_ladder(const sage_options *o, sage_graph *g) {
   g->alpha = alpha;
   g->beta = beta;
   g->ctas_per_sm = cps;
+  g->hub_filter = hub;
   return SAGE_OK;
 }
 

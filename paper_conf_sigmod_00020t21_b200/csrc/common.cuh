@@ -569,9 +569,31 @@ __device__ __forceinline__ void defer_close(WarpScratch *ws, int &cnt, int *list
 // and rows loaded before the current enqueue.  Returns whether the list was non-empty (then the
 // caller must barrier before reading the log's counters).  Must stay inlined (an out-of-line call
 // cost k_bfs its register allocation).
+// Hub table inserts (BFS, DESIGN.md §5 "hub filter"): every classified vertex of degree >= thr is
+// offered to slot v & mask of a global direct-mapped table with atomicMax of (degree, key + 1), so
+// a slot ends up holding the highest-degree VISITED vertex mapped to it (visited bits only rise).
+// 0 = empty slot; a vertex whose key + 1 does not fit the key field is never inserted.
+struct HubIns {
+  uint32_t *g = nullptr;   // T packed entries (0 = empty); null = no table
+  uint32_t mask = 0;       // T - 1
+  int lgT = 0;             // key = v >> lgT
+  int kbits = 0;           // key field bits (8 or 16); degree in the upper 32 - kbits bits
+  long long thr = 0;       // minimum degree of an inserted vertex
+};
+__device__ __forceinline__ void hub_insert(const HubIns &h, int v, long long deg) {
+  if (h.g && v >= 0 && deg >= h.thr) {
+    const uint32_t k1 = ((uint32_t)v >> h.lgT) + 1u;
+    if (k1 >> h.kbits) return;
+    const unsigned long long dmax = (1ull << (32 - h.kbits)) - 1;
+    const uint32_t d = (uint32_t)((unsigned long long)deg < dmax ? (unsigned long long)deg : dmax);
+    atomicMax(h.g + ((uint32_t)v & h.mask), (d << h.kbits) | k1);
+  }
+}
+
 __device__ __forceinline__ bool classify_deferred(const long long *__restrict__ off, const int *flist,
                                                   const unsigned long long *flc, const Ladder &L,
-                                                  const Queues &Q, CounterSet *cs) {
+                                                  const Queues &Q, CounterSet *cs,
+                                                  const HubIns &hub = HubIns()) {
   const unsigned long long fl = ldcg(flc);
   if (!fl) return false;
   const unsigned lane = threadIdx.x & 31;
@@ -591,6 +613,7 @@ __device__ __forceinline__ bool classify_deferred(const long long *__restrict__ 
       long long b2 = 0, e2 = 0;
       if (v2 >= 0) ld_row_pair(off, v2, &b2, &e2);
       enqueue_count(v >= 0, b, e, L, tot, nf, arcs);
+      hub_insert(hub, v, e - b);
       base = nb;
       v = v2;
       b = b2;

@@ -34,6 +34,7 @@ struct TraversalState {     // per-query scratch, allocated on first use and kep
   int32_t *tmp_out = nullptr;     // ID-translation scratch (n_local)
   void *tailmem = nullptr;        // BFS tail mode state (global scratch)
   int *flist = nullptr;           // BFS deferred contraction: frontier list
+  uint32_t *hub_g = nullptr;      // BFS hub filter: global table of visited hubs (T packed entries)
 };
 
 struct PageRankState {      // the all-V resident tile log (built once, reused)
@@ -43,7 +44,8 @@ struct PageRankState {      // the all-V resident tile log (built once, reused; 
   int32_t *dangling = nullptr;    // vertices with out-degree 0
   long long n_dangling = 0;
   double *x = nullptr, *y = nullptr;
-  float *c = nullptr;             // pull form: x_u / out(u)
+  void *c = nullptr;              // pull form: x_u / out(u) (fp32, or fp64 when damping > 0.9)
+  size_t c_bytes = 0;
   CounterSet *cs = nullptr;       // device copy of the log's counters (+ rotating tickets)
 };
 
@@ -72,6 +74,7 @@ struct sage_graph {
   sage::Ladder ladder{};
   double alpha = 15.0, beta = 18.0;
   int ctas_per_sm = 0;        // sage_options.ctas_per_sm (0 = automatic)
+  int hub_filter = 0;         // sage_options.hub_filter (0 auto, 1 on, -1 off)
   int vec = 4;                // neighbours per lane per step (4; 1 when tile_min < 4)
   bool vec_ok = true;         // sub-warp tiles use 16-B loads (align % 4 == 0, aligned arrays)
   // reordering: sigma[v_orig] = current label; sigma_inv[label] = v_orig (null = identity)
@@ -88,5 +91,5 @@ struct sage_graph {
   long long online_thr = 0, online_pending = 0, online_rounds = 0, online_movers = 0, online_swaps = 0;
   uint32_t *samp_w = nullptr;
   unsigned long long *samp_acc = nullptr;
-  int grid_bfs = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0;   // persistent grid sizes
+  int grid_bfs = 0, grid_bfs_hub = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0, grid_pr_pull64 = 0;   // persistent grid sizes
 };

@@ -34,7 +34,8 @@ sage_status init_comm(sage_graph *g, const sage_dist *ds);
 void free_comm(sage_graph *g);
 
 // cooperative persistent launch helper
-sage_status launch_coop(sage_graph *g, const void *fn, int grid, void **args, const char *what);
-int coop_grid(sage_graph *g, const void *fn, int *cache);
+sage_status launch_coop(sage_graph *g, const void *fn, int grid, void **args, const char *what,
+                        int block = kBlock, size_t dyn_smem = 0);
+int coop_grid(sage_graph *g, const void *fn, int *cache, int block = kBlock, size_t dyn_smem = 0);
 
 }  // namespace sage

@@ -30,7 +30,34 @@
 namespace sage {
 
 // ============================================================================ filters
-struct BfsPush {
+// Hub filter (B200 addition): a push level examines the status of every arc's
+// target, and on a scale-free graph most arcs of the heavy levels point at a few high-degree
+// vertices that are already visited.  A scattered global status read costs one L1TEX wavefront
+// per lane (32 per warp instruction) and holds an L1 line while it waits for L2; a shared-memory
+// read of a random byte costs ~4 wavefronts per warp instruction.  Each CTA therefore keeps a
+// direct-mapped table of visited hubs in shared memory (slot = v & (T-1), entry = (v >> lgT) + 1,
+// 0 = empty) and skips the global read when the slot holds v.  The table only ever holds visited
+// vertices, so a hit is exact (visited bits only rise); a miss falls back to Alg. 1's test.
+// HT selects (lgT, key bits): 1 = (17, 8) and 2 = (16, 16): 128 KB; 3 = (16, 8) and 4 = (15, 16): 64 KB.
+template <int HT> struct HubGeom;
+template <> struct HubGeom<0> { static constexpr int lgT = 0, kbits = 0, bytes = 0; };
+template <> struct HubGeom<1> { static constexpr int lgT = 17, kbits = 8, bytes = 1 << 17; };
+template <> struct HubGeom<2> { static constexpr int lgT = 16, kbits = 16, bytes = 2 << 16; };
+template <> struct HubGeom<3> { static constexpr int lgT = 16, kbits = 8, bytes = 1 << 16; };
+template <> struct HubGeom<4> { static constexpr int lgT = 15, kbits = 16, bytes = 2 << 15; };
+__device__ __forceinline__ uint32_t ld_shared_u8(uint32_t addr) {
+  uint32_t r;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(r) : "r"(addr));
+  return r;
+}
+__device__ __forceinline__ uint32_t ld_shared_u16(uint32_t addr) {
+  uint32_t r;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=r"(r) : "r"(addr));
+  return r;
+}
+
+template <int HT>
+struct BfsPushT {
   struct Src {
     int u;
   };
@@ -48,6 +75,7 @@ struct BfsPush {
   int v_base;          // global id of local row 0 (0 on one GPU)
   const Queues *next_q;
   CounterSet *next_cs;
+  uint32_t ht = 0;     // shared-memory address of the hub table (HT > 0)
 
   __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
 
@@ -55,10 +83,22 @@ struct BfsPush {
   template <int N>
   __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N],
                                         const uint32_t (&)[N], bool (&in)[N], int) const {
+    bool hit[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      hit[j] = false;
+      if constexpr (HT > 0) {
+        constexpr int lg = HubGeom<HT>::lgT;
+        const uint32_t slot = (uint32_t)v[j] & ((1u << lg) - 1u), k1 = ((uint32_t)v[j] >> lg) + 1u;
+        if constexpr (HubGeom<HT>::kbits == 8) hit[j] = ld_shared_u8(ht + slot) == k1;
+        else hit[j] = ld_shared_u16(ht + 2u * slot) == k1;
+      }
+    }
     uint32_t wd[N];
     const unsigned long long keep = policy_evict_last();
 #pragma unroll
-    for (int j = 0; j < N; ++j) wd[j] = valid ? ld_status(visited + (v[j] >> 5), keep) : 0xffffffffu;
+    for (int j = 0; j < N; ++j)
+      wd[j] = (valid && !hit[j]) ? ld_status(visited + (v[j] >> 5), keep) : 0xffffffffu;
     // claims of all N neighbours in flight together (predicated, no branch between them)
     uint32_t old[N];
 #pragma unroll
@@ -78,6 +118,7 @@ struct BfsPush {
     }
   }
 };
+using BfsPush = BfsPushT<0>;
 
 struct SsspPush {
   struct Src {
@@ -149,6 +190,8 @@ struct TravArgs {
   struct TailSmem *tailmem;   // tail mode state (global scratch: only block 0 uses it)
   int steal;            // 0 = ablation: static tile assignment instead of stealing
   int *flist;           // deferred contraction: frontier list (n + slack entries)
+  HubIns hub;           // hub filter: global table + insert rule (hub.g null = off)
+  unsigned long long hub_min_arcs;   // reload the CTA's table before levels with arcs(F) >= this
 };
 
 // Pull (bottom-up) step over the visited bitmap: one warp per 32-vertex word.
@@ -267,12 +310,12 @@ struct TailSmem {
   int d[2][kTailV];                  // its out-degree
   int pre[kTailV + 1];
   int buf[kTailCollect];
-  int wsum[kWarps];
+  int wsum[32];
   int nnext;
   unsigned long long anext;
 };
 
-// exclusive block scan of x (one value per thread, 256 threads); returns the total
+// exclusive block scan of x (one value per thread, <= 1024 threads); returns the total
 __device__ __forceinline__ int block_scan_excl(int x, int *out_excl, int *wsum) {
   const int lane = (int)lane_id(), warp = threadIdx.x >> 5;
   int inc = x;
@@ -284,7 +327,8 @@ __device__ __forceinline__ int block_scan_excl(int x, int *out_excl, int *wsum) 
   if (lane == 31) wsum[warp] = inc;
   __syncthreads();
   int base = 0, total = 0;
-  for (int w = 0; w < kWarps; ++w) {
+  const int nw = blockDim.x >> 5;
+  for (int w = 0; w < nw; ++w) {
     if (w < warp) base += wsum[w];
     total += wsum[w];
   }
@@ -448,13 +492,28 @@ __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
 }
 
 // ============================================================================ BFS kernel
-template <int VEC>
-#ifndef SAGE_BFS_MINB
-#define SAGE_BFS_MINB 4
-#endif
-__global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_constant__ TravArgs a) {
-  __shared__ WarpScratch wsm[kWarps];
-  __shared__ BfsPush::Src fsrc[kWarps][32];
+// Load the CTA's hub table from the global one (after the K2' phase that inserted into it).
+template <int HT>
+__device__ __forceinline__ void hub_load(const TravArgs &a, uint8_t *ht) {
+  const uint4 *g4 = reinterpret_cast<const uint4 *>(a.hub.g);
+  constexpr int nvec = (1 << HubGeom<HT>::lgT) >> 2;
+  constexpr uint32_t km = (1u << HubGeom<HT>::kbits) - 1u;
+  for (int i = threadIdx.x; i < nvec; i += blockDim.x) {
+    const uint4 p = __ldcg(g4 + i);
+    const uint32_t k0 = p.x & km, k1 = p.y & km, k2 = p.z & km, k3 = p.w & km;
+    if constexpr (HubGeom<HT>::kbits == 8) {
+      reinterpret_cast<uint32_t *>(ht)[i] = k0 | (k1 << 8) | (k2 << 16) | (k3 << 24);
+    } else {
+      reinterpret_cast<uint2 *>(ht)[i] = make_uint2(k0 | (k1 << 16), k2 | (k3 << 16));
+    }
+  }
+}
+
+// The BFS level loop (one persistent cooperative launch per query).  HT > 0: hub filter on (the
+// CTA holds the table in `ht`, HubGeom<HT>::bytes of shared memory).
+template <int VEC, int HT>
+__device__ __forceinline__ void bfs_body(const TravArgs &a, WarpScratch *wsm, typename BfsPushT<HT>::Src (*fsrc)[32],
+                                         uint8_t *ht) {
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
   double mU = (double)a.m - (double)ldcg(&ctl->set[0].arcsF.v);
@@ -463,6 +522,9 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
   unsigned long long prev_nF = 1;
   const long long nwords = (a.n + 31) >> 5;
   if ((threadIdx.x & 31) == 0) wsm[warp].cpos = wsm[warp].cend = 0;
+  if constexpr (HT > 0) {   // empty table
+    for (int i = threadIdx.x; i < HubGeom<HT>::bytes / 4; i += blockDim.x) reinterpret_cast<uint32_t *>(ht)[i] = 0u;
+  }
   for (int L = 0;; ++L) {
     CounterSet *cur = &ctl->set[L % 3];
     CounterSet *nxt = &ctl->set[(L + 1) % 3];
@@ -471,7 +533,13 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
     uint32_t *fbc = a.fb[L % 3], *fbn = a.fb[(L + 1) % 3];
     if (a.do_enabled) clear_words(a.fb[(L + 2) % 3], nwords);
     if (dir == 0) {
-      BfsPush f;
+      if constexpr (HT > 0) {
+        if (ldcg(&cur->arcsF.v) >= a.hub_min_arcs) {
+          hub_load<HT>(a, ht);
+          __syncthreads();
+        }
+      }
+      BfsPushT<HT> f;
       f.visited = a.visited;
       f.level = a.level;
       f.parent = a.parent;
@@ -482,28 +550,16 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
       f.next_cs = nxt;
       f.flist = a.flist;
       f.flc = &nxt->flc.v;
-#ifdef SAGE_PROF
-      const unsigned long long pt0 = globaltimer();
-#endif
+      if constexpr (HT > 0) f.ht = (uint32_t)__cvta_generic_to_shared(ht);
       consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok,
                        a.steal != 0);
-#ifdef SAGE_PROF
-      if (L == 1 && (threadIdx.x & 31) == 0) {   // per-warp consume durations of level 1
-        const unsigned long long d = globaltimer() - pt0;
-        atomicAdd(&g_prof[8], d);
-        atomicMax(&g_prof[9], d);
-        if (d > 20000) atomicAdd(&g_prof[10], 1ull);
-        atomicAdd(&g_prof[11], 1ull);
-        atomicMax(&g_prof[12], pt0 - ctl->t0_ns);
-        atomicMin(&g_prof[13], pt0 - ctl->t0_ns);
-      }
-#endif
     } else {
       pull_level(a, L + 1, fbc, fbn, a.q[(L + 1) & 1], cur, nxt, &wsm[warp]);
     }
     if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
     grid_barrier(&ctl->bar);
-    if (classify_deferred(a.off, a.flist, &nxt->flc.v, a.L, a.q[(L + 1) & 1], nxt))
+    if (blockIdx.x == 0 && threadIdx.x == 0 && L < kMaxRec) ctl->rec[L].t_mid = globaltimer();
+    if (classify_deferred(a.off, a.flist, &nxt->flc.v, a.L, a.q[(L + 1) & 1], nxt, a.hub))
       grid_barrier(&ctl->bar);
     const unsigned long long nF = ldcg(&nxt->nF.v);
     const unsigned long long aF = ldcg(&nxt->arcsF.v);
@@ -540,6 +596,23 @@ __global__ void __launch_bounds__(kBlock, SAGE_BFS_MINB) k_bfs(const __grid_cons
     }
     prev_nF = nF;
   }
+}
+
+template <int VEC>
+__global__ void __launch_bounds__(kBlock, 4) k_bfs(const __grid_constant__ TravArgs a) {
+  __shared__ WarpScratch wsm[kWarps];
+  __shared__ BfsPush::Src fsrc[kWarps][32];
+  bfs_body<VEC, 0>(a, wsm, fsrc, nullptr);
+}
+
+// Hub-filter variant: one 1024-thread CTA per SM (one table per SM, not per CTA).
+constexpr int kHubBlock = 1024;
+template <int VEC, int HT>
+__global__ void __launch_bounds__(kHubBlock, 1) k_bfs_hub(const __grid_constant__ TravArgs a) {
+  __shared__ WarpScratch wsm[kHubBlock / 32];
+  __shared__ typename BfsPushT<HT>::Src fsrc[kHubBlock / 32][32];
+  extern __shared__ __align__(16) uint8_t hub_smem[];
+  bfs_body<VEC, HT>(a, wsm, fsrc, hub_smem);
 }
 
 // ============================================================================ SSSP kernel
@@ -749,6 +822,7 @@ void free_traversal_state(sage_graph *g) {
   dfree(g, t.tmp_out);
   dfree(g, t.tailmem);
   dfree(g, t.flist);
+  dfree(g, t.hub_g);
   t = TraversalState();
 }
 
@@ -789,21 +863,21 @@ sage_status ensure_traversal_state(sage_graph *g) {
   return SAGE_OK;
 }
 
-int coop_grid(sage_graph *g, const void *fn, int *cache) {
+int coop_grid(sage_graph *g, const void *fn, int *cache, int block, size_t dyn_smem) {
   if (*cache) return *cache;
-  // shared-memory carveout: the persistent kernels use <= 10 KB of shared memory per CTA; the rest
-  // of the SM's 256 KB goes to L1, which caches status words and row offsets.  The smallest
-  // carveout that still holds the occupancy limit's CTAs (+1 KB reserved per CTA) is requested
-  // (measured on C2 push BFS: driver default 3.40 ms, smallest carveout 3.15 ms).
+  // shared-memory carveout: the smallest that still holds the occupancy limit's CTAs (+1 KB
+  // reserved per CTA); the rest of the SM's 256 KB goes to L1, which caches status words and row
+  // offsets (measured on C2 push BFS: driver default 3.40 ms, smallest carveout 3.15 ms)
+  if (dyn_smem) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn_smem);
   int nb = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, kBlock, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, block, dyn_smem);
   if (nb < 1) nb = 1;
   {
     cudaFuncAttributes fa;
     if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) {
       int smem_sm = 0;
       cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, g->device);
-      const size_t need = (size_t)nb * (fa.sharedSizeBytes + 1024);
+      const size_t need = (size_t)nb * (fa.sharedSizeBytes + dyn_smem + 1024);
       if (smem_sm > 0) {
         const int pct = (int)std::min<size_t>(100, (need * 100 + smem_sm - 1) / smem_sm);
         cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
@@ -819,8 +893,9 @@ int coop_grid(sage_graph *g, const void *fn, int *cache) {
   return *cache;
 }
 
-sage_status launch_coop(sage_graph *g, const void *fn, int grid, void **args, const char *what) {
-  cudaError_t e = cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kBlock), args, 0, g->stream);
+sage_status launch_coop(sage_graph *g, const void *fn, int grid, void **args, const char *what, int block,
+                        size_t dyn_smem) {
+  cudaError_t e = cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(block), args, dyn_smem, g->stream);
   if (e != cudaSuccess) return cuda_fail(g, e, what);
   return SAGE_OK;
 }
@@ -852,6 +927,27 @@ sage_status translate_out_f64(sage_graph *g, const double *src, double *dst_user
   k_gather_f64<<<g->num_sms * 8, 256, 0, g->stream>>>(src, g->sigma, tmp, g->n_local);
   return copy_out(g, dst_user, tmp, bytes);
 }
+
+// Hub filter (BfsPushT): on graphs with >= 32M arcs the push BFS runs the 1024-thread variant with
+// a table of visited hubs per SM.  SAGE_HUB_KB (compile time) = 64 or 128 KB tables; 8-bit keys
+// when every key + 1 fits a byte (n <= 255 * T), else 16-bit keys.
+#ifndef SAGE_HUB_KB
+#define SAGE_HUB_KB 64
+#endif
+constexpr long long kHubMinGraphArcs = 32ll << 20;
+constexpr unsigned long long kHubMinLevelArcs = 4ull << 20;   // reload the tables before such levels
+static int hub_mode(const sage_graph *g) {
+#ifdef SAGE_NO_HUB
+  return 0;
+#else
+  if (g->vec != 4 || g->hub_filter < 0 || (g->hub_filter == 0 && g->m < kHubMinGraphArcs)) return 0;
+  if (SAGE_HUB_KB == 128) return g->n <= 255ll << 17 ? 1 : 2;
+  return g->n <= 255ll << 16 ? 3 : 4;
+#endif
+}
+static int hub_lgT(int ht) { return ht == 1 ? 17 : ht == 4 ? 15 : 16; }
+static int hub_kbits(int ht) { return (ht == 1 || ht == 3) ? 8 : 16; }
+static size_t hub_bytes(int ht) { return ht == 1 || ht == 2 ? (128u << 10) : (64u << 10); }
 
 static TravArgs make_args(sage_graph *g) {
   TravArgs a;
@@ -967,13 +1063,38 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   a.parent = parent_out ? t.parent : nullptr;
   a.do_enabled = (symmetric && !push_only) ? 1 : 0;
   a.steal = (call_flags & SAGE_F_NO_STEALING) ? 0 : 1;
+  if (const int ht = hub_mode(g)) {
+    const int lgT = hub_lgT(ht);
+    if (!t.hub_g && (s = dalloc(g, (void **)&t.hub_g, sizeof(uint32_t) << 17)) != SAGE_OK) return s;
+    cudaMemsetAsync(t.hub_g, 0, sizeof(uint32_t) << lgT, g->stream);
+    a.hub.g = t.hub_g;
+    a.hub.lgT = lgT;
+    a.hub.mask = (1u << lgT) - 1u;
+    a.hub.kbits = hub_kbits(ht);
+    a.hub.thr = std::max<long long>(2, 2 * ((g->m + g->n_local - 1) / std::max<long long>(1, g->n_local)));
+    a.hub_min_arcs = kHubMinLevelArcs;
+  }
   k_seed<<<1, 32, 0, g->stream>>>(a, src, 0);
   cudaEventRecord(e1, g->stream);
   {
-    const void *fn = g->vec == 4 ? (const void *)k_bfs<4> : (const void *)k_bfs<1>;
-    const int grid = coop_grid(g, fn, &g->grid_bfs);
+    const int ht = hub_mode(g);
+    const void *fn = ht == 1 ? (const void *)k_bfs_hub<4, 1>
+                   : ht == 2 ? (const void *)k_bfs_hub<4, 2>
+                   : ht == 3 ? (const void *)k_bfs_hub<4, 3>
+                   : ht == 4 ? (const void *)k_bfs_hub<4, 4>
+                   : g->vec == 4 ? (const void *)k_bfs<4> : (const void *)k_bfs<1>;
+    int block = ht ? kHubBlock : kBlock;
+    size_t dyn = ht ? hub_bytes(ht) : 0;
+#ifdef SAGE_HUB_NOTABLE   // A/B: the 1024-thread configuration without the table (1: same smem, 2: no smem)
+    if (ht) {
+      fn = (const void *)k_bfs_hub<4, 0>;
+      if (SAGE_HUB_NOTABLE == 2) dyn = 0;
+    }
+#endif
+    const int grid = coop_grid(g, fn, ht ? &g->grid_bfs_hub : &g->grid_bfs, block, dyn);
     void *args[] = {&a};
-    if ((s = launch_coop(g, fn, grid, args, "BFS kernel")) != SAGE_OK) return s;
+    if ((s = launch_coop(g, fn, grid, args, "BFS kernel", block, dyn)) != SAGE_OK) return s;
+    (void)block;
   }
   cudaEventRecord(e2, g->stream);
   Ctl h;
@@ -1037,9 +1158,9 @@ extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_o
   k_seed<<<1, 32, 0, g->stream>>>(a, src, 1);
   cudaEventRecord(e1, g->stream);
   const void *fn = g->vec == 4 ? (const void *)k_sssp<4> : (const void *)k_sssp<1>;
-  const int grid = coop_grid(g, fn, &g->grid_sssp);
+  const int grid = coop_grid(g, fn, &g->grid_sssp, kBlock, 0);
   void *args[] = {&a, &ovf};
-  if ((s = launch_coop(g, fn, grid, args, "SSSP kernel")) != SAGE_OK) {
+  if ((s = launch_coop(g, fn, grid, args, "SSSP kernel", kBlock, 0)) != SAGE_OK) {
     dfree(g, ovf);
     return s;
   }

@@ -6,8 +6,9 @@ ladder B=256 M=8 A=4).
   and direction-optimising.
 * SSSP: the exact certificate of SURVEY §8(c) c2 (dist(s)=0, no arc can be relaxed, every reached
   vertex has a tight in-arc) — it accepts iff dist is the true shortest-distance vector.
-* PageRank: x_20 from the GPU equals one oracle power-iteration step applied to the GPU's x_19,
-  at every vertex, within 1e-6 relative (the property x_K = step(x_{K-1}) holds at any size).
+* PageRank: the full 20-iteration oracle run (fp64, serial) vs the GPU's pull (default on this
+  symmetric graph) and push (Alg. 1) forms, within 1e-6 relative at every vertex; and x_20 equals
+  one oracle step applied to the GPU's x_19.
 * Reorder: after one round, BFS answers in original ids are unchanged.
 """
 import numpy as np
@@ -54,6 +55,13 @@ def test_c2_sssp_certificate(c2, G):
     d, st = G.sssp(s)
     assert oracle.check_sssp(c2.off, c2.col, c2.w, s, d) == 0
     assert st["levels"] > 5
+
+
+def test_c2_pagerank_full_oracle(c2, G):
+    ref = oracle.pagerank(c2.off, c2.col, 0.85, 20)
+    for po in (False, True):
+        x, _ = G.pagerank(0.85, 20, push_only=po)
+        assert np.max(np.abs(x - ref) / ref) <= 1e-6, po
 
 
 def test_c2_pagerank_step_property(c2, G):

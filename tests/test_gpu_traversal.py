@@ -204,6 +204,18 @@ def test_pagerank_parity(sage, lad):
             assert np.max(np.abs(x2 - oracle.pagerank(g.off, g.col, 0.85, 20)) / x2) <= 1e-6
 
 
+@pytest.mark.parametrize("d", [0.5, 0.9, 0.95, 0.99])
+def test_pagerank_damping_range(sage, d):
+    """Pull (fp32 contributions up to d = 0.9, fp64 above) and push forms within 1e-6 of the
+    oracle across the damping range the ABI accepts."""
+    g = sg.rmat(16, 16, seed=13, symmetric=True)
+    ref = oracle.pagerank(g.off, g.col, d, 30)
+    with sage.load_csr(g.off, g.col, symmetric=True) as G:
+        for po in (False, True):
+            x, _ = G.pagerank(d, 30, push_only=po)
+            assert np.max(np.abs(x - ref) / ref) <= 1e-6, (d, po)
+
+
 def test_pagerank_pull_precision_at_scale(sage):
     """Pull form: fp32 contributions, fp64 accumulation (R7) stays well inside 1e-6 on RMAT-18."""
     g = sg.rmat(18, 16, seed=3, symmetric=True)
@@ -359,3 +371,36 @@ def test_deferred_contraction_every_level(sage):
             for s in sg.sources(g, 3, seed=2):
                 assert np.array_equal(G.bfs(int(s), push_only=True)[0], oracle.bfs(g.off, g.col, int(s)))
                 assert np.array_equal(G.sssp(int(s))[0], oracle.sssp(g.off, g.col, w, int(s))[0])
+
+
+@pytest.mark.parametrize("scale,sym", [(14, True), (16, True), (16, False), (18, True)])
+def test_hub_filter_parity(sage, scale, sym):
+    """Push BFS with the shared-memory hub filter forced on (8-bit keys, n <= 2^24) equals the
+    oracle's levels and, with parents, passes the parent rule; with the filter forced off too."""
+    g = sg.rmat(scale, 16, seed=40 + scale, symmetric=sym)
+    for hub in (1, -1):
+        with sage.load_csr(g.off, g.col, symmetric=sym, hub_filter=hub) as G:
+            for s in sg.sources(g, 3, seed=2):
+                ref = oracle.bfs(g.off, g.col, int(s))
+                lv, par, _ = G.bfs(int(s), push_only=True, parents=True)
+                assert np.array_equal(lv, ref), (hub, int(s))
+                _parents_ok(g.off, g.col, lv, par, int(s))
+                lv, _, _ = G.bfs(int(s))
+                assert np.array_equal(lv, ref), (hub, int(s), "do")
+
+
+def test_hub_filter_16bit_keys(sage):
+    """n > 2^24 selects 16-bit hub keys: a sparse random graph over 2^24 + 5000 vertices with a
+    dense core (hubs) gives the oracle's levels."""
+    n = (1 << 24) + 5000
+    rng = np.random.default_rng(7)
+    core = rng.integers(0, n, size=2000)
+    src = rng.integers(0, n, size=3_000_000)
+    dst = core[rng.integers(0, len(core), size=3_000_000)]
+    e = np.stack([src, dst], 1)
+    g = sg.from_edges(n, np.concatenate([e, e[:, ::-1]]), True, "hubby")
+    with sage.load_csr(g.off, g.col, symmetric=True, hub_filter=1) as G:
+        for s in [int(core[0]), int(src[1])]:
+            ref = oracle.bfs(g.off, g.col, s)
+            lv, _, _ = G.bfs(s, push_only=True)
+            assert np.array_equal(lv, ref)

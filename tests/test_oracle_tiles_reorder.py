@@ -160,3 +160,37 @@ def test_reorder_improves_objective_on_scrambled_rmat():
     off2, col2, _, _, info = oracle.reorder(g.off, g.col, None, rounds=2, B=256, M=8, A=4, S=8)
     after = oracle.objective(off2, col2, B=256, M=8, A=4, S=8)
     assert info[0]["swaps"] > 0 and after < before
+
+
+def test_tile_log_quads_with_fragments(golden_dir):
+    """Hand-derived resident tile log quadruples (vertex, offset, size, kind) with aligned head
+    fragments, tail fragments, empty rows and several ladders (tests/golden/tile_log_quads.json)."""
+    fx = json.load(open(os.path.join(golden_dir, "tile_log_quads.json")))
+    off = np.array(fx["off"], dtype=np.int64)
+    vs = np.array(fx["vertices"], dtype=np.int32)
+    for lad in fx["ladders"]:
+        got = oracle.tile_log(off, vs, lad["B"], lad["M"], lad["A"]).tolist()
+        assert got == lad["quads"], (lad["B"], lad["M"], lad["A"])
+
+
+def _tie_csr(fx):
+    n = fx["n"]
+    rows = {int(k): v for k, v in fx["rows"].items()}
+    off = np.zeros(n + 1, dtype=np.int64)
+    for u in range(n):
+        off[u + 1] = off[u] + len(rows.get(u, []))
+    col = np.array([c for u in range(n) for c in rows.get(u, [])], dtype=np.int32)
+    return off, col
+
+
+def test_stage2_tie_goes_left(golden_dir):
+    """Reading R21's tie rule (L == R -> left half) on a hand-built sample whose first stage-2
+    step ties (tests/golden/stage2_tie.json)."""
+    fx = json.load(open(os.path.join(golden_dir, "stage2_tie.json")))
+    off, col = _tie_csr(fx)
+    tp, mem = oracle.sample_tiles(off, col, fx["B"], fx["M"], fx["A"])
+    st = oracle.reorder_stages(fx["n"], tp, mem, fx["S"], trace_v=1)
+    assert [list(t) for t in st["trace"]] == fx["trace_v1"]
+    assert st["target"][1] == fx["target_v1"]
+    assert st["loc1"][1] == fx["loc1_v1"] and st["loc3"][1] == fx["loc3_v1"]
+    assert st["mover"][1] == fx["mover_v1"]

@@ -68,7 +68,7 @@ enum {
 
 /* Multi-GPU description (1D vertex partition).  NULL in sage_csr = single GPU.
  * Non-NULL selects the NCCL path (also with world == 1: a 1-rank communicator).  On that path
- * sage_bfs (no parents), sage_sssp and sage_pagerank are collective (every rank calls them with
+ * sage_bfs (parents included), sage_sssp and sage_pagerank are collective (every rank calls them with
  * the same arguments; outputs hold the rank's own rows); sage_reorder / sage_bc return
  * SAGE_E_UNSUPPORTED.  Multi-GPU SSSP exchanges candidate distances of
  * remote targets with one ncclReduceScatter(min) per Bellman-Ford iteration.                   */
@@ -100,7 +100,8 @@ typedef struct {
 typedef struct {
   int64_t n;                     /* GLOBAL vertex count, 0 < n < 2^31                              */
   int64_t m;                     /* LOCAL arc count; must equal row_offsets[n_local]                */
-  const int64_t *row_offsets;    /* n_local + 1 entries, row_offsets[0] = 0, non-decreasing.
+  const int64_t *row_offsets;    /* n_local + 1 entries, row_offsets[0] = 0, non-decreasing, every
+                                    row shorter than 2^31 arcs.
                                     n_local = v_end - v_begin (multi-GPU) or n                     */
   const int32_t *col_indices;    /* m entries, GLOBAL ids in [0, n); rows need not be sorted       */
   const uint32_t *weights;       /* m entries >= 1, or NULL (SSSP then returns SAGE_E_INVALID)     */
@@ -248,6 +249,15 @@ sage_status sage_debug_reorder_stages(sage_graph *g, int32_t sector_width, const
  * Writes min(levels, cap) records to host memory; *n_out = number of levels (<= 4096 kept).     */
 sage_status sage_debug_level_records(const sage_graph *g, int64_t *rec_out, int32_t cap,
                                      int32_t *n_out);
+
+/* Test entry point (not part of the release ABI): a 128-byte id that, passed as
+ * sage_dist.nccl_unique_id by `world` graphs loaded in ONE process on ONE GPU (one host thread
+ * per rank, every rank loaded before any collective call), replaces NCCL by a loopback transport
+ * (stream-ordered device copies / reductions between the ranks' buffers; xport.h).  It exists so
+ * the multi-GPU path's remote-owner code (r > 0, padded indexing, the apply kernels, the sparse
+ * and dense exchanges) is checked against the oracle on a single-GPU test pool.  The group lives
+ * until its last graph is freed.                                                               */
+sage_status sage_debug_loopback_id(int32_t world, void *out128);
 
 /* Thread-local message of the last failing call on this thread ("" if none).                   */
 const char *sage_last_error(void);

@@ -27,7 +27,7 @@ STATUS_NAMES = {0: "SAGE_OK", 1: "SAGE_E_INVALID", 2: "SAGE_E_NOMEM", 3: "SAGE_E
 EXPORTED = ["sage_load_csr", "sage_free", "sage_bfs", "sage_bfs_ex", "sage_sssp", "sage_pagerank",
             "sage_pagerank_ex", "sage_bc", "sage_online_reorder", "sage_online_reorder_info",
             "sage_reorder", "sage_reorder_objective", "sage_get_permutation", "sage_get_csr", "sage_graph_info",
-            "sage_debug_export_tiles", "sage_debug_reorder_stages", "sage_nccl_unique_id", "sage_debug_level_records", "sage_last_error", "sage_version"]
+            "sage_debug_export_tiles", "sage_debug_reorder_stages", "sage_nccl_unique_id", "sage_debug_level_records", "sage_debug_loopback_id", "sage_last_error", "sage_version"]
 
 
 class SageError(RuntimeError):
@@ -100,6 +100,7 @@ def lib():
         L.sage_debug_export_tiles.argtypes = [p, p, i64, p, i64, p]
         L.sage_debug_level_records.argtypes = [p, p, i32, p]
         L.sage_nccl_unique_id.argtypes = [p]
+        L.sage_debug_loopback_id.argtypes = [i32, p]
         L.sage_last_error.restype = ctypes.c_char_p
         L.sage_version.restype = ctypes.c_char_p
         for f in EXPORTED:
@@ -308,6 +309,13 @@ def nccl_unique_id() -> bytes:
     """sage_nccl_unique_id: 128 bytes to broadcast from rank 0 to every rank."""
     buf = ctypes.create_string_buffer(128)
     _check(lib().sage_nccl_unique_id(buf))
+    return buf.raw
+
+
+def debug_loopback_id(world: int) -> bytes:
+    """sage_debug_loopback_id (tests only): an id for ``world`` logical ranks on this one GPU."""
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().sage_debug_loopback_id(int(world), buf))
     return buf.raw
 
 

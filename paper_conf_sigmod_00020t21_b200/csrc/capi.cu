@@ -103,7 +103,7 @@ __global__ void k_validate_rows(const long long *__restrict__ off, long long n_l
   unsigned long long bad = 0, iso = 0, mx = 0;
   for (; i < n_local; i += stride) {
     long long b = off[i], e = off[i + 1];
-    if (e < b || b < 0 || e > m) { bad++; continue; }
+    if (e < b || b < 0 || e > m || e - b > 0x7fffffffll) { bad++; continue; }
     if (e == b) iso++;
     else if (rowstart) atomicOr(rowstart + (b >> 5), 1u << (b & 31));
     unsigned long long d = (unsigned long long)(e - b);

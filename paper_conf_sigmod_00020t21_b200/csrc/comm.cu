@@ -5,8 +5,11 @@
 // contiguous vertex block [vb[r], vb[r+1]) and its out-rows (global column ids); one process per
 // GPU; the communicator is created from a unique id the caller broadcasts.  Per BFS level:
 //   push : the local stealing consumer expands the local log; owned neighbours are claimed
-//          locally, remote ones are marked in an outgoing bitmap -> NCCL alltoall of the owners'
-//          slices (dense next-frontier exchange, C1b) -> owners apply the received candidates.
+//          locally, remote ones go to their owner in one of two forms, chosen per level from the
+//          global arcs(F) every rank already knows (so all ranks agree without a counts round):
+//          sparse (C1a) when arcs(F) < Wp - int32 ids in per-destination lists of capacity
+//          arcs(F), which no sender can exceed - else dense (C1b) - the owners' bitmap slices;
+//          an all-to-all(v) moves them and the owners apply the received candidates.
 //   pull : allgather of the frontier slices (C1c), then every rank scans its own unvisited rows.
 //   stats: allreduce of (|F|, arcs(F)) gives termination and the Beamer direction (C1d).
 // PageRank: push into a full-length partial y, ncclReduceScatter(sum) to the owners (C1e), plus
@@ -14,7 +17,12 @@
 // Global-indexed bitmaps / vectors use a PADDED layout: vertex v of owner r sits at
 // r * P + (v - vb[r]) with P = 32 * Wp >= max rows per rank, so every rank's slice is a contiguous
 // word range and the exchanges are plain equal-count collectives.
-// With dist != NULL and world == 1 the same path runs on a 1-rank communicator (tested on 1 GPU).
+// With dist != NULL and world == 1 the same path runs on a 1-rank communicator (tested on 1 GPU);
+// the collectives go through an Xport (xport.h): NCCL, or the test-only loopback transport that
+// runs p logical ranks on one GPU so the r > 0 paths are checked against the oracle.
+// BFS parents (any valid BFS-tree parent, sage.h): after the traversal every rank allgathers the
+// levels, proposes for each target v of its rows the smallest u with level(u) = level(v) - 1, and
+// a reduce-scatter(min) hands each owner its answer.
 #include <cuda_runtime.h>
 #include <nccl.h>
 #include <string.h>
@@ -25,6 +33,7 @@
 #include "common.cuh"
 #include "graph.h"
 #include "internal.h"
+#include "xport.h"
 
 namespace sage {
 
@@ -48,7 +57,7 @@ __device__ __forceinline__ long long pidx(const PartMap &pm, long long v, bool *
 }
 
 struct Comm {
-  ncclComm_t nc = nullptr;
+  Xport *x = nullptr;
   int rank = 0, world = 1;
   std::vector<long long> vb;
   long long Wp = 0;                  // padded words per rank
@@ -60,18 +69,17 @@ struct Comm {
   unsigned long long *stats = nullptr;  // 8 u64
   double *y = nullptr, *yown = nullptr, *dsum = nullptr;
   uint32_t *cand = nullptr, *cown = nullptr;   // SSSP min-exchange buffers (p*P and P)
+  uint32_t *sp_send = nullptr, *sp_recv = nullptr;   // sparse exchange: p blocks of (cap + 2) words
+  long long sp_words = 0;                            // allocated words of each
+  int32_t *glevel = nullptr;         // parents: allgathered levels (p*P, padded layout)
+  uint32_t *pcand = nullptr, *pown = nullptr;        // parents: p*P proposals, own P after min
   PartMap pm;
 };
 
-static sage_status nccl_fail(sage_graph *g, ncclResult_t r, const char *what) {
-  set_error("%s: %s", what, ncclGetErrorString(r));
-  if (g) g->sticky = SAGE_E_NCCL;
-  return SAGE_E_NCCL;
-}
-#define NCCL_CHECK(g, call, what)                     \
-  do {                                                \
-    ncclResult_t r_ = (call);                         \
-    if (r_ != ncclSuccess) return nccl_fail(g, r_, what); \
+#define XCHECK(call)                \
+  do {                              \
+    sage_status s_ = (call);        \
+    if (s_ != SAGE_OK) return s_;   \
   } while (0)
 
 // ============================================================================ filters / kernels
@@ -91,6 +99,9 @@ struct MultiArgs {
   int vec_ok;
   int lvl;                         // current level L
   PartMap pm;
+  uint32_t *sp_send;               // sparse form: p blocks of (sp_cap + 2) words [count, 0, ids...]
+  const uint32_t *sp_recv;
+  long long sp_cap;                // 0 = dense form this level
   int *flist;                      // deferred contraction: frontier list
   // SSSP (frontier Bellman-Ford across ranks)
   const uint32_t *w;
@@ -136,8 +147,13 @@ struct BfsPushMulti {
         if (fb_next) atomicOr(fb_next + (p >> 5), bit);
         v[j] = lv;                   // enqueue the LOCAL row id
         in[j] = true;
+      } else if (a->sp_cap) {       // candidate for its owner: sparse form (global id)
+        const int q = (int)(p / a->pm.P);
+        uint32_t *blk = a->sp_send + (long long)q * (a->sp_cap + 2);
+        const uint32_t pos = atomicAdd(blk, 1u);
+        blk[2 + pos] = (uint32_t)v[j];
       } else {
-        atomicOr(a->out + (p >> 5), bit);   // candidate for its owner (dense exchange)
+        atomicOr(a->out + (p >> 5), bit);   // dense form: the owner's bitmap slice
       }
     }
   }
@@ -212,6 +228,66 @@ __global__ void __launch_bounds__(kBlock) k_mapply(const __grid_constant__ Multi
     }
   }
   if (bcnt) buffer_flush(&wsm[warp], bcnt, a.off, a.L, Qn, csn);
+}
+
+// Sparse form: owners apply the ids received from every other rank.
+__global__ void __launch_bounds__(kBlock) k_mapply_sparse(const __grid_constant__ MultiArgs a) {
+  __shared__ WarpScratch wsm[kWarps];
+  const int warp = threadIdx.x >> 5;
+  const int L = a.lvl;
+  const long long gt = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long nt = (long long)gridDim.x * blockDim.x;
+  uint32_t *fbn = a.do_enabled ? a.fb[(L + 1) % 3] : nullptr;
+  const Queues &Qn = a.q[(L + 1) & 1];
+  CounterSet *csn = &a.ctl->set[(L + 1) % 3];
+  const long long blk = a.sp_cap + 2;
+  const long long total = (long long)a.pm.p * a.sp_cap;
+  int bcnt = 0;
+  for (long long base = gt - (gt & 31); base < total; base += nt) {
+    const long long i = base + (gt & 31);
+    bool in = false;
+    int lv = 0;
+    if (i < total) {
+      const int q = (int)(i / a.sp_cap);
+      const long long k = i - (long long)q * a.sp_cap;
+      if (q != a.pm.rank && k < (long long)a.sp_recv[(long long)q * blk]) {
+        lv = (int)((long long)a.sp_recv[(long long)q * blk + 2 + k] - a.v_begin);
+        const long long gp = (long long)a.pm.rank * a.pm.P + lv;
+        const uint32_t bit = 1u << (gp & 31);
+        if (!(atomicOr(a.visited + (gp >> 5), bit) & bit)) {
+          in = true;
+          a.level[lv] = L + 1;
+          if (fbn) atomicOr(fbn + (gp >> 5), bit);
+        }
+      }
+    }
+    buffer_push(in, lv, &wsm[warp], bcnt, a.off, a.L, Qn, csn);
+  }
+  if (bcnt) buffer_flush(&wsm[warp], bcnt, a.off, a.L, Qn, csn);
+}
+
+// Parents after the traversal: for every own row u and arc u->v with level(v) = level(u) + 1,
+// propose u (global id) for v in the padded proposal array (smallest wins: atomicMin).
+__global__ void k_mparent_propose(const MultiArgs a, const int32_t *glevel, uint32_t *pcand) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long u = (long long)blockIdx.x * blockDim.x + threadIdx.x; u < a.n_local; u += stride) {
+    const int lu = a.level[u];
+    if (lu < 0) continue;
+    for (long long k = a.off[u]; k < a.off[u + 1]; ++k) {
+      bool own;
+      const long long p = pidx(a.pm, a.col[k], &own);
+      if (glevel[p] == lu + 1) atomicMin(pcand + p, (uint32_t)(u + a.v_begin));
+    }
+  }
+}
+__global__ void k_mparent_final(const int *level, const uint32_t *pown, long long n, int *parent) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+    parent[v] = level[v] > 0 ? (int)pown[v] : -1;
+}
+__global__ void k_fill_u32(uint32_t *p, long long n, uint32_t v) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) p[i] = v;
 }
 
 // Pull level over the own rows; the frontier bitmap holds the allgathered global frontier.
@@ -525,16 +601,16 @@ sage_status init_comm(sage_graph *g, const sage_dist *ds) {
     set_error("at most %d ranks", kMaxRanks);
     return SAGE_E_INVALID;
   }
-  ncclUniqueId id;
-  memcpy(&id, ds->nccl_unique_id, sizeof(id));
-  NCCL_CHECK(g, ncclCommInitRank(&c->nc, c->world, id, c->rank), "ncclCommInitRank");
+  sage_status s;
+  c->x = make_loopback_xport(g, ds->nccl_unique_id, c->rank, c->world, &s);
+  if (!c->x && s == SAGE_OK) c->x = make_nccl_xport(g, ds->nccl_unique_id, c->rank, c->world, &s);
+  if (!c->x) return s;
   // every rank's block and arc count
   long long *d = nullptr;
-  sage_status s;
   if ((s = dalloc(g, (void **)&d, sizeof(long long) * 4 * (size_t)(c->world + 1))) != SAGE_OK) return s;
   long long mine[3] = {(long long)g->v_begin, (long long)g->v_end, (long long)g->m};
   cudaMemcpyAsync(d + 3 * c->rank, mine, sizeof(mine), cudaMemcpyHostToDevice, g->stream);
-  NCCL_CHECK(g, ncclAllGather(d + 3 * c->rank, d, 3, ncclInt64, c->nc, g->stream), "allgather blocks");
+  XCHECK(c->x->allgather(g, d + 3 * c->rank, d, 3 * sizeof(long long)));
   std::vector<long long> all(3 * (size_t)c->world);
   cudaMemcpyAsync(all.data(), d, sizeof(long long) * all.size(), cudaMemcpyDeviceToHost, g->stream);
   cudaError_t e = cudaStreamSynchronize(g->stream);
@@ -586,8 +662,13 @@ void free_comm(sage_graph *g) {
   dfree(g, c->dsum);
   dfree(g, c->cand);
   dfree(g, c->cown);
+  dfree(g, c->sp_send);
+  dfree(g, c->sp_recv);
+  dfree(g, c->glevel);
+  dfree(g, c->pcand);
+  dfree(g, c->pown);
   cudaStreamSynchronize(g->stream);
-  if (c->nc) ncclCommDestroy(c->nc);
+  delete c->x;
   delete c;
   g->comm = nullptr;
 }
@@ -595,8 +676,7 @@ void free_comm(sage_graph *g) {
 static sage_status allreduce_stats(sage_graph *g, int L, unsigned long long *h6) {
   Comm *c = g->comm;
   k_mstats<<<1, 32, 0, g->stream>>>(g->ts.ctl, L % 3, (L + 1) % 3, c->stats);
-  NCCL_CHECK(g, ncclAllReduce(c->stats, c->stats + 8, 6, ncclUint64, ncclSum, c->nc, g->stream),
-             "stats allreduce");
+  XCHECK(c->x->allreduce_sum_u64(g, c->stats, c->stats + 8, 6));
   cudaMemcpyAsync(h6, c->stats + 8, sizeof(unsigned long long) * 6, cudaMemcpyDeviceToHost, g->stream);
   cudaError_t e = cudaStreamSynchronize(g->stream);
   if (e != cudaSuccess) return cuda_fail(g, e, "stats");
@@ -606,10 +686,6 @@ static sage_status allreduce_stats(sage_graph *g, int L, unsigned long long *h6)
 sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int32_t *parent_out,
                           uint32_t call_flags, sage_stats *st) {
   Comm *c = g->comm;
-  if (parent_out) {
-    set_error("BFS parents are not produced by the multi-GPU path");
-    return SAGE_E_UNSUPPORTED;
-  }
   sage_status s;
   if ((s = ensure_traversal_state(g)) != SAGE_OK) return s;
   TraversalState &t = g->ts;
@@ -650,14 +726,14 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
   unsigned long long h6[6];
   {
     k_mstats<<<1, 32, 0, g->stream>>>(t.ctl, 2, 0, c->stats);   // set[0] = the seed's log
-    NCCL_CHECK(g, ncclAllReduce(c->stats, c->stats + 8, 6, ncclUint64, ncclSum, c->nc, g->stream),
-               "stats allreduce");
+    XCHECK(c->x->allreduce_sum_u64(g, c->stats, c->stats + 8, 6));
     cudaMemcpyAsync(h6, c->stats + 8, sizeof(h6), cudaMemcpyDeviceToHost, g->stream);
     cudaError_t e = cudaStreamSynchronize(g->stream);
     if (e != cudaSuccess) return cuda_fail(g, e, "seed");
   }
   double mU = (double)c->m_total - (double)h6[1];
   unsigned long long reached_arcs = h6[1];
+  unsigned long long aF_cur = h6[1];   // global arcs(F) of the level about to run
   const int grid_push = g->num_sms * 4;
   int dir = 0;
   unsigned long long prev_nF = 1;
@@ -668,21 +744,42 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
     if (do_enabled) cudaMemsetAsync(c->fb[(L + 2) % 3], 0, 4 * words, g->stream);
     a.lvl = L;
     if (dir == 0) {
+      // exchange form of this level (every rank knows the global arcs(F)): sparse lists of
+      // capacity arcs(F) when that is smaller than a dense slice, else the dense slices
+      const long long cap = (c->world > 1 && (long long)aF_cur < c->Wp) ? (long long)aF_cur : 0;
+      a.sp_cap = cap;
+      if (cap) {
+        const long long need = (cap + 2) * c->world;
+        if (need > c->sp_words) {
+          dfree(g, c->sp_send);
+          dfree(g, c->sp_recv);
+          c->sp_send = c->sp_recv = nullptr;
+          const long long alloc = std::max<long long>(need, 4096);
+          if ((s = dalloc(g, (void **)&c->sp_send, 4 * (size_t)alloc)) != SAGE_OK ||
+              (s = dalloc(g, (void **)&c->sp_recv, 4 * (size_t)alloc)) != SAGE_OK)
+            return s;
+          c->sp_words = alloc;
+        }
+        cudaMemsetAsync(c->sp_send, 0, 4 * (size_t)need, g->stream);
+        a.sp_send = c->sp_send;
+        a.sp_recv = c->sp_recv;
+      }
       if (g->vec == 4) k_mpush<4><<<grid_push, kBlock, 0, g->stream>>>(a);
       else k_mpush<1><<<grid_push, kBlock, 0, g->stream>>>(a);
       k_mclassify<<<grid_push, kBlock, 0, g->stream>>>(a);
-      // dense alltoall of the owners' candidate slices
-      NCCL_CHECK(g, ncclGroupStart(), "group");
-      for (int r = 0; r < c->world; ++r) {
-        if (r == c->rank) continue;
-        NCCL_CHECK(g, ncclSend(c->out + (size_t)r * c->Wp, (size_t)c->Wp, ncclUint32, r, c->nc, g->stream),
-                   "send");
-        NCCL_CHECK(g, ncclRecv(c->recv + (size_t)r * c->Wp, (size_t)c->Wp, ncclUint32, r, c->nc, g->stream),
-                   "recv");
+      if (c->world > 1) {
+        std::vector<size_t> off((size_t)c->world + 1);
+        const size_t blk = cap ? 4 * (size_t)(cap + 2) : 4 * (size_t)c->Wp;
+        for (int r = 0; r <= c->world; ++r) off[(size_t)r] = blk * (size_t)r;
+        if (cap) {
+          XCHECK(c->x->alltoallv(g, c->sp_send, off.data(), c->sp_recv, off.data()));
+          k_mapply_sparse<<<grid_push, kBlock, 0, g->stream>>>(a);
+        } else {
+          XCHECK(c->x->alltoallv(g, c->out, off.data(), c->recv, off.data()));
+          cudaMemsetAsync(c->out, 0, 4 * words, g->stream);
+          k_mapply<<<grid_push, kBlock, 0, g->stream>>>(a);
+        }
       }
-      NCCL_CHECK(g, ncclGroupEnd(), "group");
-      cudaMemsetAsync(c->out, 0, 4 * words, g->stream);
-      if (c->world > 1) k_mapply<<<grid_push, kBlock, 0, g->stream>>>(a);
     } else {
       k_mpull<<<grid_push, kBlock, 0, g->stream>>>(a);
     }
@@ -703,6 +800,7 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
       pull_disc += (long long)nF;
     }
     reached_arcs += aF;
+    aF_cur = aF;
     if (nF == 0) break;
     if (L + 1 > g->n) {
       set_error("level cap exceeded");
@@ -720,9 +818,7 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
     if (ndir == 1) {
       // pull needs the global frontier: allgather of every owner's slice of fb[L+1]
       uint32_t *fbn = c->fb[(L + 1) % 3];
-      NCCL_CHECK(g, ncclAllGather(fbn + (size_t)c->rank * c->Wp, fbn, (size_t)c->Wp, ncclUint32, c->nc,
-                                  g->stream),
-                 "frontier allgather");
+      XCHECK(c->x->allgather(g, fbn + (size_t)c->rank * c->Wp, fbn, 4 * (size_t)c->Wp));
     }
     dir = ndir;
     prev_nF = nF;
@@ -748,6 +844,28 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
     const double n = (double)g->n;
     st->model_bytes = 4.0 * n + 20.0 * push_exp + 8.0 * push_arcs + 8.0 * push_disc + 16.0 * pull_sc +
                       (n / 8.0) * pullL + 4.125 * pull_insp + 4.125 * pull_disc;
+  }
+  if (parent_out) {
+    // any valid parent: allgather the levels (padded layout), propose the smallest u with
+    // level(u) = level(v) - 1 for every target v of the own rows, min reduce-scatter to the owners
+    const long long P = c->pm.P;
+    if (!c->glevel) {
+      if ((s = dalloc(g, (void **)&c->glevel, sizeof(int32_t) * (size_t)P * c->world)) != SAGE_OK ||
+          (s = dalloc(g, (void **)&c->pcand, sizeof(uint32_t) * (size_t)P * c->world)) != SAGE_OK ||
+          (s = dalloc(g, (void **)&c->pown, sizeof(uint32_t) * (size_t)P)) != SAGE_OK)
+        return s;
+    }
+    if (!t.parent && (s = dalloc(g, (void **)&t.parent, sizeof(int32_t) * (size_t)g->n_local)) != SAGE_OK)
+      return s;
+    int32_t *mine = c->glevel + (size_t)c->rank * P;
+    cudaMemsetAsync(mine, 0xff, sizeof(int32_t) * (size_t)P, g->stream);
+    cudaMemcpyAsync(mine, t.level, sizeof(int32_t) * (size_t)g->n_local, cudaMemcpyDeviceToDevice, g->stream);
+    XCHECK(c->x->allgather(g, mine, c->glevel, sizeof(int32_t) * (size_t)P));
+    k_fill_u32<<<grid_push, 256, 0, g->stream>>>(c->pcand, P * c->world, 0xffffffffu);
+    k_mparent_propose<<<grid_push, 256, 0, g->stream>>>(a, c->glevel, c->pcand);
+    XCHECK(c->x->reduce_scatter_min_u32(g, c->pcand, c->pown, (size_t)P));
+    k_mparent_final<<<grid_push, 256, 0, g->stream>>>(t.level, c->pown, g->n_local, t.parent);
+    if ((s = copy_out(g, parent_out, t.parent, sizeof(int32_t) * (size_t)g->n_local)) != SAGE_OK) return s;
   }
   if ((s = copy_out(g, level_out, t.level, sizeof(int32_t) * (size_t)g->n_local)) != SAGE_OK) return s;
   e = cudaStreamSynchronize(g->stream);
@@ -813,8 +931,7 @@ sage_status run_sssp_multi(sage_graph *g, int32_t source, uint32_t *dist_out, sa
     a.inq_next = t.fb[(L + 1) % 3];
     if (g->vec == 4) k_msssp_push<4><<<grid, kBlock, 0, g->stream>>>(a);
     else k_msssp_push<1><<<grid, kBlock, 0, g->stream>>>(a);
-    NCCL_CHECK(g, ncclReduceScatter(c->cand, c->cown, (size_t)P, ncclUint32, ncclMin, c->nc, g->stream),
-               "SSSP min reduce-scatter");
+    XCHECK(c->x->reduce_scatter_min_u32(g, c->cand, c->cown, (size_t)P));
     cudaMemsetAsync(c->cand, 0xff, sizeof(uint32_t) * (size_t)P * c->world, g->stream);
     if (c->world > 1) k_msssp_apply<<<grid, kBlock, 0, g->stream>>>(a);
     cudaError_t e = cudaGetLastError();
@@ -844,21 +961,20 @@ sage_status run_sssp_multi(sage_graph *g, int32_t source, uint32_t *dist_out, sa
   cudaStreamSynchronize(g->stream);
   unsigned long long fl[2] = {(unsigned long long)hflag, 0ull};
   cudaMemcpyAsync(red, fl, sizeof(unsigned long long), cudaMemcpyHostToDevice, g->stream);
-  NCCL_CHECK(g, ncclAllReduce(red, red + 8, 1, ncclUint64, ncclSum, c->nc, g->stream), "overflow flag");
+  XCHECK(c->x->allreduce_sum_u64(g, red, red + 8, 1));
   cudaMemcpyAsync(&fl[1], red + 8, sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream);
   cudaStreamSynchronize(g->stream);
   if (fl[1]) {
     uint32_t *bits = c->visited;   // p*Wp words, padded layout
     k_mreached_bits<<<grid, 256, 0, g->stream>>>(t.dist, g->n_local, bits + (size_t)c->rank * c->Wp);
-    NCCL_CHECK(g, ncclAllGather(bits + (size_t)c->rank * c->Wp, bits, (size_t)c->Wp, ncclUint32, c->nc,
-                                g->stream), "reached allgather");
+    XCHECK(c->x->allgather(g, bits + (size_t)c->rank * c->Wp, bits, 4 * (size_t)c->Wp));
     k_moverflow_check<<<grid, 256, 0, g->stream>>>(a, bits, ovf + 1);
     int hf = 0;
     cudaMemcpyAsync(&hf, ovf + 1, sizeof(int), cudaMemcpyDeviceToHost, g->stream);
     cudaStreamSynchronize(g->stream);
     fl[0] = (unsigned long long)hf;
     cudaMemcpyAsync(red, fl, sizeof(unsigned long long), cudaMemcpyHostToDevice, g->stream);
-    NCCL_CHECK(g, ncclAllReduce(red, red + 8, 1, ncclUint64, ncclSum, c->nc, g->stream), "overflow found");
+    XCHECK(c->x->allreduce_sum_u64(g, red, red + 8, 1));
     cudaMemcpyAsync(&fl[1], red + 8, sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream);
     cudaStreamSynchronize(g->stream);
     if (fl[1]) {
@@ -881,7 +997,7 @@ sage_status run_sssp_multi(sage_graph *g, int32_t source, uint32_t *dist_out, sa
     unsigned long long *ra = c->stats;
     cudaMemsetAsync(ra, 0, sizeof(unsigned long long), g->stream);
     k_mreached_arcs<<<grid, 256, 0, g->stream>>>((const long long *)g->off, t.dist, g->n_local, ra);
-    NCCL_CHECK(g, ncclAllReduce(ra, ra + 8, 1, ncclUint64, ncclSum, c->nc, g->stream), "reached arcs");
+    XCHECK(c->x->allreduce_sum_u64(g, ra, ra + 8, 1));
     cudaMemcpyAsync(&hra, ra + 8, sizeof(hra), cudaMemcpyDeviceToHost, g->stream);
     cudaStreamSynchronize(g->stream);
   }
@@ -942,10 +1058,8 @@ sage_status run_pagerank_multi(sage_graph *g, double damping, int32_t iterations
     cudaMemsetAsync(&p.cs[0].tk, 0, sizeof(p.cs[0].tk), g->stream);
     if (g->vec == 4) k_mpr_push<4><<<grid, kBlock, 0, g->stream>>>(a);
     else k_mpr_push<1><<<grid, kBlock, 0, g->stream>>>(a);
-    NCCL_CHECK(g, ncclReduceScatter(c->y, c->yown, (size_t)P, ncclFloat64, ncclSum, c->nc, g->stream),
-               "reduce-scatter");
-    NCCL_CHECK(g, ncclAllReduce(c->dsum, c->dsum + 1, 1, ncclFloat64, ncclSum, c->nc, g->stream),
-               "dangling allreduce");
+    XCHECK(c->x->reduce_scatter_sum_f64(g, c->y, c->yown, (size_t)P));
+    XCHECK(c->x->allreduce_sum_f64(g, c->dsum, c->dsum + 1, 1));
     k_mpr_finalize<<<grid, 256, 0, g->stream>>>(p.x, c->yown, g->n_local, (1.0 - damping) / N, damping,
                                                 c->dsum + 1, N);
   }

@@ -488,7 +488,7 @@ struct WarpScratch {
   int pre[32];
   int hl[32];
   long long hb[32];
-  long long tb[32];
+  int tb[32];          // fragment gather: tail start - head start (a row's length fits 31 bits)
   int buf[64];
   long long cpos, cend;   // deferred contraction: the warp's open chunk of the frontier list
 };
@@ -957,7 +957,7 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
     ws->pre[lane] = inc - fl;
     ws->hl[lane] = hl;
     ws->hb[lane] = hb;
-    ws->tb[lane] = tb;
+    ws->tb[lane] = (int)(tb - hb);
     fsrc[lane] = sc;
     __syncwarp();
     for (int k0 = 0; k0 < total; k0 += 32) {
@@ -978,7 +978,7 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
       const typename F::Src so = fsrc[o];
       if (kv) {
         const int idx = k - ws->pre[o];
-        const long long pos = idx < ws->hl[o] ? ws->hb[o] + idx : ws->tb[o] + (idx - ws->hl[o]);
+        const long long pos = ws->hb[o] + (idx < ws->hl[o] ? idx : ws->tb[o] + (idx - ws->hl[o]));
         vv[0] = ld_col(col + pos, pol);
         if (F::kWeights) w1[0] = ld_colu(w + pos, pol);
       }

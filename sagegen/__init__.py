@@ -164,3 +164,54 @@ def config(name: str) -> Graph:
     if name == "C4":
         return uk_like()
     raise KeyError(name)
+
+
+# ---------------------------------------------------------------- per-rank device generation
+_DEV = None
+
+
+def _dev_lib():
+    global _DEV
+    if _DEV is None:
+        import sys
+        sys.path.insert(0, os.path.dirname(_HERE))
+        from tools.build import build_sagegen_dev
+        lib = ctypes.CDLL(build_sagegen_dev())
+        i64, u64, p, dbl, c_int = ctypes.c_longlong, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_double, ctypes.c_int
+        lib.sgd_rmat_build.argtypes = [c_int, c_int, u64, dbl, dbl, dbl, c_int, i64, i64, p,
+                                       ctypes.POINTER(p), ctypes.POINTER(i64)]
+        lib.sgd_rmat_take.argtypes = [p, p, p, p]
+        lib.sgd_weights.argtypes = [i64, i64, p, p, u64, ctypes.c_uint32, p, p]
+        lib.sgd_free.argtypes = [p]
+        _DEV = lib
+    return _DEV
+
+
+def rmat_device(scale: int, edgefactor: int = 16, seed: int = 1, symmetric: bool = True,
+                v_begin: int = 0, v_end: int | None = None, weights_seed: int | None = None,
+                abc=(0.57, 0.19, 0.19), stream=None):
+    """Rows [v_begin, v_end) of ``rmat(scale, edgefactor, seed, symmetric)`` generated on the current
+    CUDA device (every tuple is regenerated; arcs whose source is outside the block are dropped).
+    Returns torch tensors (off int64[n_local+1] rebased to 0, col int32[m_local], w uint32 or None)."""
+    import torch
+    n = 1 << scale
+    v_end = n if v_end is None else v_end
+    st = torch.cuda.current_stream().cuda_stream if stream is None else stream
+    h, m = ctypes.c_void_p(), ctypes.c_longlong(0)
+    rc = _dev_lib().sgd_rmat_build(scale, edgefactor, seed, abc[0], abc[1], abc[2], int(symmetric), v_begin, v_end,
+                                   st, ctypes.byref(h), ctypes.byref(m))
+    if rc != 0:
+        raise RuntimeError(f"sgd_rmat_build failed ({rc})")
+    off = torch.empty(v_end - v_begin + 1, dtype=torch.int64, device="cuda")
+    col = torch.empty(max(m.value, 1), dtype=torch.int32, device="cuda")
+    if _dev_lib().sgd_rmat_take(h, off.data_ptr(), col.data_ptr(), st) != 0:
+        raise RuntimeError("sgd_rmat_take failed")
+    col = col[:m.value]
+    w = None
+    if weights_seed is not None:
+        w = torch.empty(max(m.value, 1), dtype=torch.int32, device="cuda").view(torch.uint32)
+        if _dev_lib().sgd_weights(v_end - v_begin, v_begin, off.data_ptr(), col.data_ptr(), weights_seed, 255,
+                                  w.data_ptr(), st) != 0:
+            raise RuntimeError("sgd_weights failed")
+        w = w[:m.value]
+    return off, col, w

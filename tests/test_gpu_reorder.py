@@ -209,3 +209,48 @@ def test_online_reorder_errors(sage):
         info = G.online_info()
         assert info["rounds"] == 0 and info["pending"] > 0
         assert np.array_equal(G.permutation(), np.arange(g.n))
+
+
+def _digest(a):
+    import hashlib
+    return hashlib.sha256(np.ascontiguousarray(a).tobytes()).hexdigest()
+
+
+def test_reorder_rmat16_equals_oracle(sage):
+    """SURVEY §8(c) c5 sizes: one round on RMAT-16 (symmetric, weighted), sigma and the relabelled
+    CSR (with weights) equal to the oracle's, computed live."""
+    g = sg.rmat(16, 16, seed=7, symmetric=True)
+    w = sg.weights(g, 2)
+    off2, col2, w2, sigma, info = oracle.reorder(g.off, g.col, w, rounds=1)
+    with sage.load_csr(g.off, g.col, w, symmetric=True) as G:
+        st = G.reorder(1)
+        assert st["vertices_discovered"] == info[0]["swaps"]
+        assert np.array_equal(G.permutation(), sigma)
+        o, c, ww = G.csr()
+        assert np.array_equal(o, off2) and np.array_equal(c, col2) and np.array_equal(ww, w2)
+
+
+@pytest.mark.parametrize("name", ["rmat20", "twitter1m"])
+def test_reorder_large_equals_oracle_golden(sage, golden_dir, name):
+    """SURVEY §8(c) c5 sizes too slow to recompute here (the serial oracle takes 3-6 min): the
+    oracle's sigma and relabelled CSR are stored as SHA-256 digests by
+    tools/golden/make_reorder_golden.py (which calls only oracle/); the GPU round must match them."""
+    fx = json.load(open(os.path.join(golden_dir, f"reorder_{name}.json")))
+    c = fx["case"]
+    if c["gen"] == "rmat":
+        g = sg.rmat(c["scale"], c["ef"], c["seed"], c["symmetric"])
+    else:
+        g = sg.twitter_like(n=c["n"], tuples=c["tuples"], seed=c["seed"])
+    w = sg.weights(g, c["weights_seed"]) if c.get("weights_seed") else None
+    assert (g.n, g.m) == (fx["n"], fx["m"])
+    with sage.load_csr(g.off, g.col, w, symmetric=g.symmetric, tile_cta=c["B"], tile_min=c["M"],
+                       align=c["A"]) as G:
+        st = G.reorder(c["rounds"], sector_width=c["S"])
+        assert st["vertices_discovered"] == fx["info"][0]["swaps"]
+        sig = G.permutation()
+        assert int(np.sum(sig != np.arange(g.n))) == fx["n_moved"]
+        assert _digest(sig.astype(np.int32)) == fx["sha256_sigma"]
+        o, cc, ww = G.csr()
+        assert _digest(o) == fx["sha256_off"] and _digest(cc) == fx["sha256_col"]
+        if fx["sha256_w"] is not None:
+            assert _digest(ww) == fx["sha256_w"]

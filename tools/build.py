@@ -4,6 +4,8 @@
   the C ABI declared in ``include/sage.h`` (nvcc, ``-gencode arch=compute_100a,code=sm_100a``).
 * ``oracle/liboracle.so`` — the serial CPU oracle (plain C, gcc).  Test infrastructure.
 * ``sagegen/libsagegen.so`` — seeded input generators (C++/OpenMP).  Test infrastructure.
+* ``sagegen/libsagegen_dev.so`` — the same RMAT/Kronecker generator per rank on the device
+  (CUDA; multi-GPU bench inputs such as C5).  Test / bench infrastructure.
 
 The three share no source file and no header.  Builds are incremental (mtime based) and
 in-tree so the ``.so`` files travel to the GPU box with the repo snapshot.
@@ -55,6 +57,15 @@ def build_sagegen(force=False):
     out = os.path.join(ROOT, "sagegen", "libsagegen.so")
     if force or _stale(out, [src]):
         _run(["g++", "-O3", "-march=x86-64-v2", "-std=c++17", "-fopenmp", "-shared", "-fPIC", src, "-o", out])
+    return out
+
+
+def build_sagegen_dev(force=False):
+    """Per-rank device generator of the RMAT / Kronecker inputs (bench + tests infrastructure)."""
+    src = os.path.join(ROOT, "sagegen", "sagegen_dev.cu")
+    out = os.path.join(ROOT, "sagegen", "libsagegen_dev.so")
+    if force or _stale(out, [src]):
+        _run([NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC", "-shared", src, "-o", out])
     return out
 
 
@@ -110,7 +121,7 @@ def build_sage(force=False, verbose=False):
 
 
 def build_all(force=False, verbose=False):
-    return [build_sagegen(force), build_oracle(force), build_sage(force, verbose)]
+    return [build_sagegen(force), build_sagegen_dev(force), build_oracle(force), build_sage(force, verbose)]
 
 
 if __name__ == "__main__":

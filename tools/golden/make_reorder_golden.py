@@ -2,9 +2,9 @@
 too large to recompute inside the GPU test run (RMAT-20, a 1M-vertex twitter-like graph).
 
 Calls only oracle/ (plus the seeded input generator sagegen/, which holds no SAGE arithmetic).
-Stored per case: the generator parameters, the ladder / sector width / rounds, the permutation as
-its non-identity pairs (v, sigma[v]), SHA-256 digests of the relabelled off / col / weights
-arrays, and the per-round info.  tests/test_gpu_reorder.py regenerates the graph, runs the GPU
+Stored per case: the generator parameters, the ladder / sector width / rounds, the number of
+relabelled vertices, SHA-256 digests of the permutation (int32 sigma[v], original id -> label) and
+of the relabelled off / col / weights arrays, and the per-round info.  tests/test_gpu_reorder.py regenerates the graph, runs the GPU
 reorder and compares.
 
     python tools/golden/make_reorder_golden.py [case ...]
@@ -56,13 +56,13 @@ def main(names):
                            "matching R23, sorted relabel R24) on a seeded sagegen input; written by "
                            "tools/golden/make_reorder_golden.py, which calls only oracle/",
                "case": c, "n": int(g.n), "m": int(g.m), "oracle_seconds": round(dt, 1),
-               "moved": [[int(v), int(sigma[v])] for v in moved],
+               "n_moved": int(len(moved)), "sha256_sigma": digest(sigma.astype(np.int32)),
                "sha256_off": digest(off2), "sha256_col": digest(col2),
                "sha256_w": digest(w2) if w2 is not None else None,
                "info": [{k: int(v) for k, v in r.items()} for r in info]}
         p = os.path.join(ROOT, "tests", "golden", f"reorder_{name}.json")
         with open(p, "w") as f:
-            json.dump(out, f)
+            json.dump(out, f, indent=1)
         print(name, g.n, g.m, f"{dt:.1f}s", len(moved), "moved", info, flush=True)
 
 

@@ -119,6 +119,32 @@ def _traffic():
         return None
 
 
+def _pin_one_core():
+    """SURVEY §8(d) oracle timing: the serial oracle runs pinned to one host core; returns a
+    description of the host (CPU model, cores) for the cpu_baseline object."""
+    try:
+        cpus = sorted(os.sched_getaffinity(0))
+        os.sched_setaffinity(0, {cpus[-1]})
+    except Exception:
+        pass
+    model = "unknown CPU"
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return model, os.cpu_count()
+
+
+def _unpin():
+    try:
+        os.sched_setaffinity(0, set(range(os.cpu_count())))
+    except Exception:
+        pass
+
+
 def _dist():
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -136,6 +162,7 @@ def run_reference(a):
     g, gname = _graph(a.config, a.scale)
     srcs = sg.sources(g, a.warmup + a.steps, seed=2)
     deg = np.diff(g.off)
+    model, ncpu = _pin_one_core()
     times, edges = [], []
     for i, s in enumerate(srcs):
         t0 = time.perf_counter()
@@ -152,9 +179,57 @@ def run_reference(a):
             "impl": "reference",
             "config": {"workload": gname, "n": g.n, "arcs": g.m, "mode": "serial FIFO BFS (oracle/oracle.c)"},
             "cpu_baseline": {"value": hm, "unit": "GTEPS", "cores": 1, "kind": "oracle",
-                             "sample": f"{a.steps} timed oracle BFS sources of {gname} after {a.warmup} warm-up"},
+                             "sample": f"{a.steps} timed oracle BFS sources of {gname} after {a.warmup} warm-up",
+                             "host": f"serial oracle, 1 core of {model}, host has {ncpu} cores"},
             "e2e": {"value": hm, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def _spawn_if_needed(a):
+    """`python bench.py --gpus N` with N > 1 outside torchrun: re-launch as N ranks (one process
+    per GPU) through torch.distributed.run on 127.0.0.1; returns the child's exit code, or None
+    when this process is already a rank (or N == 1)."""
+    if a.gpus <= 1 or "WORLD_SIZE" in os.environ:
+        return None
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
+def multi_workload(config: str, world: int):
+    """Kronecker scale of the multi-GPU runs (weak scaling: per-GPU work fixed as N grows).
+    Default: 24 + log2(N) (N = 1 is C2's scale); --config C5: 27 + log2(N) (Kron-30 at N = 8,
+    SURVEY §8(d) C5).  N must be a power of two."""
+    lg = world.bit_length() - 1
+    if 1 << lg != world:
+        raise ValueError("the multi-GPU bench needs a power-of-two number of ranks")
+    base = 27 if config == "C5" else 24
+    return base + lg
+
+
+def _nonempty_sources(torch, off_d, n, world, k, seed=2):
+    """sagegen.sources' rule (uniform over vertices with out-degree > 0, seeded hash tries) on a
+    1D-partitioned graph: the per-rank 'row non-empty' flags are allgathered."""
+    import sagegen as sg
+    ne = (off_d[1:] > off_d[:-1]).to(torch.uint8)
+    if world > 1:
+        parts = [torch.empty_like(ne) for _ in range(world)]
+        torch.distributed.all_gather(parts, ne)
+        ne = torch.cat(parts)
+    out = []
+    for i in range(k):
+        for j0 in range(0, 1 << 20, 64):
+            cand = torch.tensor([sg.hash3(seed, i, j) % n for j in range(j0, j0 + 64)], dtype=torch.int64,
+                                device=ne.device)
+            hit = torch.nonzero(ne[cand]).flatten()
+            if len(hit):
+                out.append(int(cand[int(hit[0])]))
+                break
+    return np.array(out, dtype=np.int32)
 
 
 def main():
@@ -162,6 +237,9 @@ def main():
     if a.impl == "reference":
         run_reference(a)
         return
+    rc = _spawn_if_needed(a)
+    if rc is not None:
+        sys.exit(rc)
     import torch
 
     import paper_conf_sigmod_00020t21_b200 as sage
@@ -174,7 +252,8 @@ def main():
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     build()
-    stream = torch.cuda.current_stream()
+    stream = torch.cuda.Stream()   # one dedicated stream: the library's work, the L2 flush and the
+    torch.cuda.set_stream(stream)  # timing events are all ordered on it
     multi = world > 1 or a.nccl
     if not multi:
         g, gname = _graph(a.config, a.scale)
@@ -185,43 +264,32 @@ def main():
         n = g.n
         n_rows = n
     else:
-        # rank 0 generates the workload and broadcasts it; every rank keeps its 1D block
-        g, gname = _graph(a.config, a.scale) if rank == 0 else (None, None)
-        hdr = torch.tensor([g.n, g.m] if rank == 0 else [0, 0], dtype=torch.int64, device="cuda")
+        # every rank generates its own 1D block of the Kronecker graph on its GPU (all tuples
+        # regenerated, arcs of other owners dropped: sagegen/sagegen_dev.cu), no host graph
+        scale = a.scale if a.scale is not None else multi_workload(a.config, world)
+        n = 1 << scale
+        vb, ve = n * rank // world, n * (rank + 1) // world
+        off_d, col_d, w_d = sg.rmat_device(scale, 16, 1, True, vb, ve, weights_seed=1)
         if world > 1:
-            torch.distributed.broadcast(hdr, 0)
-        n, m = int(hdr[0]), int(hdr[1])
-        off_full = torch.from_numpy(g.off).cuda() if rank == 0 else torch.empty(n + 1, dtype=torch.int64, device="cuda")
-        col_full = torch.from_numpy(g.col).cuda() if rank == 0 else torch.empty(m, dtype=torch.int32, device="cuda")
-        w_full = (torch.from_numpy(g.w.view(np.int32)).cuda() if rank == 0 else
-                  torch.empty(m, dtype=torch.int32, device="cuda"))
-        if world > 1:
-            torch.distributed.broadcast(off_full, 0)
-            torch.distributed.broadcast(col_full, 0)
-            torch.distributed.broadcast(w_full, 0)
-            obj = [gname, sage.nccl_unique_id() if rank == 0 else None]
+            obj = [sage.nccl_unique_id() if rank == 0 else None]
             torch.distributed.broadcast_object_list(obj, 0)
-            gname, uid = obj
+            uid = obj[0]
         else:
             uid = sage.nccl_unique_id()
-        vb, ve = n * rank // world, n * (rank + 1) // world
-        b0 = int(off_full[vb])
-        off_d = (off_full[vb:ve + 1] - b0).contiguous()
-        col_d = col_full[b0:int(off_full[ve])].contiguous()
-        w_d = w_full[b0:int(off_full[ve])].contiguous().view(torch.uint32)
+        m_all = torch.tensor([col_d.numel()], dtype=torch.int64, device="cuda")
+        if world > 1:
+            torch.distributed.all_reduce(m_all)
+        gname = f"kron{scale}_sym_ef16_seed1_w255" + ("_C5" if a.config == "C5" else "")
         G = sage.load_csr(off_d, col_d, w_d, n=n, symmetric=True, borrow=True, stream=stream.cuda_stream,
                           rank=rank, world=world, nccl_unique_id=uid, v_begin=vb, v_end=ve)
         n_rows = ve - vb
-        if rank != 0:
-            class _G:  # sources only need the degree array
-                pass
-            g = _G()
-            g.n = n
-            g.off = off_full.cpu().numpy()
-            g.m = m
-            g.w = None
-        del off_full, col_full, w_full
-    srcs = sg.sources(g, a.warmup + a.steps, seed=2)
+
+        class _G:   # what the rest of main needs of the workload
+            pass
+        g = _G()
+        g.n, g.m, g.w = n, int(m_all.item()), None
+        g.srcs = _nonempty_sources(torch, off_d, n, world, a.warmup + a.steps)
+    srcs = g.srcs if multi else sg.sources(g, a.warmup + a.steps, seed=2)
     level = torch.empty(n_rows, dtype=torch.int32, device="cuda")
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
 
@@ -270,8 +338,19 @@ def main():
     peaks, peak_src = _peaks()
     achieved = kbytes / (kms * 1e-3) / 1e9
     tr = _traffic()
+    st_last = stats[-1]
+    # SURVEY §8(d) compulsory floor: 4 B per inspected arc + 16 B per expanded vertex + 4n B
+    floor = 4.0 * st_last["arcs_inspected"] + 16.0 * st_last["vertices_expanded"] + 4.0 * n
+    traffic = (tr or {}).get("bfs_push_bytes_per_launch")
     roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-            "frac": achieved / peaks["hbm_gbs"], "traffic": (tr or {}).get("bfs_push_bytes_per_launch"),
+            "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
+            "traffic_source": (tr or {}).get("source", "none") + " — an ncu --set full capture of this kernel on "
+                              "this workload, committed under profiles/; not measured inside this run",
+            "frac_nominal_8TBps": achieved / 8000.0,
+            "amplification": (traffic / kbytes) if traffic else None,
+            "l2_hit_rate_pct": (tr or {}).get("lts_hit_rate_pct"),
+            "compulsory_floor_bytes": floor,
+            "floor_frac": floor / (kms * 1e-3) / 1e9 / peaks["hbm_gbs"],
             "kernel": ("k_bfs<4> (persistent TP+RTS consumer)" if not multi else
                        "host-sequenced NCCL levels (k_mpush + alltoall + k_mapply), time incl. exchange"),
             "peak_source": peak_src,
@@ -279,10 +358,13 @@ def main():
             "kernel_ms": kms, "model_bytes_per_launch": kbytes}
     line = {"metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": world, "steps": a.steps,
             "warmup": a.warmup, "ms_per_step": t_max / a.steps, "higher_is_better": True,
-            "scaling": "strong" if multi else "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": gname, "n": n, "arcs": g.m, "mode": "push-only (SAGE_F_PUSH_ONLY)",
                        "tile_ladder": "B=256 M=8 A=4", "l2": "flushed between steps (256 MB write)",
-                       "parallelism": f"1D-partition x{world} (NCCL)" if multi else "single"},
+                       "parallelism": f"1D-partition x{world} (NCCL)" if multi else "single",
+                       **({"generated": ("per rank on device (sagegen_dev); weak scaling, Kronecker scale "
+                                         + ("27" if a.config == "C5" else "24") + " + log2(N)")}
+                          if multi else {})},
             "gpu_launches": (2 * a.steps if not multi else
                              sum(2 + s["levels"] * (3 if world > 1 else 2) for s in stats)),
             "clocks": clocks, "roofline": roof,
@@ -495,21 +577,42 @@ def _extras(a, G, g, srcs, level, flush, stream, sage):
                  "ms_per_step": float(np.mean([t for t, _ in e2e])) * 1e3, "warmup": 1, "steps": len(e2e),
                  "h2d_bytes_per_step": int(g.off.nbytes + g.col.nbytes), "d2h_bytes_per_step": int(4 * g.n),
                  "includes": "sage_load_csr from pinned host CSR (copy + validation) + sage_bfs + level D2H"}
-    # timed CPU oracle on a bounded sample of the same workload (also the full-size parity check)
-    G.bfs(int(srcs[0]), out=level, push_only=True)
-    gpu_lv = level.cpu().numpy()
-    t0 = time.perf_counter()
-    lv = oracle.bfs(g.off, g.col, int(srcs[0]))
-    dt = time.perf_counter() - t0
-    e = int(np.diff(g.off)[lv >= 0].sum()) // 2
-    ex["cpu_baseline"] = {"value": e / dt / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
-                          "sample": "1 serial oracle BFS (oracle/oracle.c FIFO queue) from the first warm-up source",
-                          "seconds": dt, "host_cpus": os.cpu_count()}
-    G.sssp(int(srcs[0]), out=dist)
-    ex["parity"] = {"bfs_levels_equal_oracle": bool(np.array_equal(lv, gpu_lv)),
-                    "sssp_certificate_ok": oracle.check_sssp(g.off, g.col, g.w, int(srcs[0]),
-                                                              dist.cpu().numpy().view(np.uint32)) == 0,
-                    "source": int(srcs[0])}
+    # timed CPU oracle on a bounded sample of the same workload (serial, pinned to one
+    # core, 8 BFS and 4 SSSP sources at C2), also the full-size parity check of those sources
+    import sagegen as sg
+    osrc = sg.sources(g, 8, seed=2)    # the first 8 bench sources (same seeded rule)
+    gpu_lv, gpu_d = [], []
+    for i in range(8):
+        G.bfs(int(osrc[i]), out=level, push_only=True)
+        gpu_lv.append(level.cpu().numpy().copy())
+    for i in range(4):
+        G.sssp(int(osrc[i]), out=dist)
+        gpu_d.append(dist.cpu().numpy().view(np.uint32).copy())
+    model, ncpu = _pin_one_core()
+    deg = np.diff(g.off)
+    bt, be, st_, se = [], [], [], []
+    bfs_ok = sssp_ok = True
+    for i in range(8):
+        t0 = time.perf_counter()
+        lv = oracle.bfs(g.off, g.col, int(osrc[i]))
+        bt.append(time.perf_counter() - t0)
+        be.append(int(deg[lv >= 0].sum()) // 2)
+        bfs_ok &= bool(np.array_equal(lv, gpu_lv[i]))
+    for i in range(4):
+        t0 = time.perf_counter()
+        dd, _ = oracle.sssp(g.off, g.col, g.w, int(osrc[i]))
+        st_.append(time.perf_counter() - t0)
+        se.append(int(deg[dd != 0xFFFFFFFF].sum()) // 2)
+        sssp_ok &= bool(np.array_equal(dd, gpu_d[i]))
+    _unpin()
+    hb = len(bt) / sum(t * 1e9 / e for t, e in zip(bt, be))
+    hs = len(st_) / sum(t * 1e9 / e for t, e in zip(st_, se))
+    ex["cpu_baseline"] = {"value": hb, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                          "sample": "8 serial oracle BFS (oracle/oracle.c FIFO queue) of the bench sources, "
+                                    "harmonic mean; 4 Dijkstra SSSP beside it",
+                          "seconds": sum(bt), "sssp_gteps": hs, "sssp_seconds": sum(st_),
+                          "host": f"serial oracle, 1 core of {model}, host has {ncpu} cores"}
+    ex["parity"] = {"bfs_levels_equal_oracle_8_sources": bfs_ok, "sssp_equal_oracle_4_sources": sssp_ok}
     # one Sampling-based Reordering round on a copy of the graph (C3-style reorder on/off)
     with sage.load_csr(torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda(), symmetric=True,
                        stream=stream.cuda_stream) as H:

@@ -119,7 +119,10 @@ __global__ void __launch_bounds__(kBlock, 4) k_bc_fwd(const __grid_constant__ Bc
   __shared__ BcFwd::Src fsrc[kWarps][32];
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
-  if ((threadIdx.x & 31) == 0) wsm[warp].cpos = wsm[warp].cend = 0;
+  if ((threadIdx.x & 31) == 0) {
+    wsm[warp].cpos = wsm[warp].cend = 0;
+    wsm[warp].ndisc = 0;
+  }
   for (int L = 0;; ++L) {
     CounterSet *cur = &ctl->set[L % 3];
     CounterSet *nxt = &ctl->set[(L + 1) % 3];

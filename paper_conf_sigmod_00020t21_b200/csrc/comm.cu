@@ -165,7 +165,10 @@ __global__ void __launch_bounds__(kBlock, 4) k_mpush(const __grid_constant__ Mul
   __shared__ BfsPushMulti::Src fsrc[kWarps][32];
   const int warp = threadIdx.x >> 5;
   const int L = a.lvl;
-  if ((threadIdx.x & 31) == 0) wsm[warp].cpos = wsm[warp].cend = 0;
+  if ((threadIdx.x & 31) == 0) {
+    wsm[warp].cpos = wsm[warp].cend = 0;
+    wsm[warp].ndisc = 0;
+  }
   __syncwarp();
   BfsPushMulti f;
   f.a = &a;

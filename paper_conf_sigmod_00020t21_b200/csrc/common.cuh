@@ -64,6 +64,7 @@ struct CounterSet {                      // counters of one log (rotated over 3 
   PaddedCounter inspected;               // pull: arcs inspected while consuming this level
   PaddedCounter scanned;                 // pull: unvisited non-isolated vertices scanned
   PaddedCounter flc;                     // deferred contraction: frontier-list slots reserved
+  PaddedCounter ftk;                     // fused tiling: frontier-list chunk tickets
 };
 
 struct LevelRec {                        // per-level record (first kMaxRec levels)
@@ -491,6 +492,7 @@ struct WarpScratch {
   int tb[32];          // fragment gather: tail start - head start (a row's length fits 31 bits)
   int buf[64];
   long long cpos, cend;   // deferred contraction: the warp's open chunk of the frontier list
+  unsigned long long ndisc;   // deferred contraction: vertices appended since the last close
 };
 
 #ifdef SAGE_PROF
@@ -535,6 +537,7 @@ __device__ __forceinline__ void defer_push(bool in, int v, WarpScratch *ws, int 
   const unsigned lane = lane_id();
   if (in) ws->buf[cnt + __popc(m & lanemask_lt())] = v;
   cnt += __popc(m);
+  if (lane == 0) ws->ndisc += (unsigned long long)__popc(m);
   if (cnt >= 32) {
     __syncwarp();
     const int x = ws->buf[lane];
@@ -546,8 +549,10 @@ __device__ __forceinline__ void defer_push(bool in, int v, WarpScratch *ws, int 
     defer_group(x, ws, list, lc);
   }
 }
-// last partial group, then -1 over the rest of the open chunk; leaves the chunk state reset
-__device__ __forceinline__ void defer_close(WarpScratch *ws, int &cnt, int *list, unsigned long long *lc) {
+// last partial group, then -1 over the rest of the open chunk; leaves the chunk state reset.
+// nfc (optional): the vertices appended since the last close are added to it (|F| of the list).
+__device__ __forceinline__ void defer_close(WarpScratch *ws, int &cnt, int *list, unsigned long long *lc,
+                                            unsigned long long *nfc = nullptr) {
   __syncwarp();
   const unsigned lane = lane_id();
   if (cnt) {
@@ -560,7 +565,11 @@ __device__ __forceinline__ void defer_close(WarpScratch *ws, int &cnt, int *list
   const long long p0 = ws->cpos, p1 = ws->cend;
   for (long long i = p0 + lane; i < p1; i += 32) list[i] = -1;
   __syncwarp();
-  if (lane == 0) ws->cpos = ws->cend = 0;
+  if (lane == 0) {
+    if (nfc && ws->ndisc) atomicAdd(nfc, ws->ndisc);
+    ws->ndisc = 0;
+    ws->cpos = ws->cend = 0;
+  }
   __syncwarp();
 }
 
@@ -726,12 +735,20 @@ __device__ __forceinline__ void push_filtered(const F &f, bool in, int v, WarpSc
   }
   buffer_push(in, v, ws, cnt, off, L, *f.next_q, f.next_cs);
 }
+// Filters may carry `nfc`: where the deferred contraction counts |F| of the list it appends to
+// (the fused runtime tiling of push BFS, traversal.cu); others count in the K2' phase.
+template <class F, class = void> struct NfcOf {
+  __device__ __forceinline__ static unsigned long long *get(const F &) { return nullptr; }
+};
+template <class F> struct NfcOf<F, std::void_t<decltype(F::nfc)>> {
+  __device__ __forceinline__ static unsigned long long *get(const F &f) { return f.nfc; }
+};
 template <class F>
 __device__ __forceinline__ void close_filtered(const F &f, WarpScratch *ws, int &cnt,
                                                const long long *__restrict__ off, const Ladder &L) {
   if constexpr (DeferTrait<F>::value) {
     if (!SAGE_DEFER_RUNTIME || f.flist) {
-      defer_close(ws, cnt, f.flist, f.flc);
+      defer_close(ws, cnt, f.flist, f.flc, NfcOf<F>::get(f));
       return;
     }
   }

@@ -41,7 +41,9 @@ struct SampleArgs {
   unsigned long long cnt[kQueues];
   int lgS;
   int sort_tiles;              // rows not known to be sorted -> sort every tile in smem
-  unsigned long long *loc1, *loc3, *cl, *cr;
+  unsigned long long *loc1, *loc3;
+  void *cd;                    // stage 2: L - R per vertex (int32 when it cannot overflow, else int64)
+  int cd32;
   const int2 *lohi;
   const int *target;
   unsigned long long *objective;
@@ -145,8 +147,12 @@ __global__ void __launch_bounds__(256) k_sample(const __grid_constant__ SampleAr
             const int ihi = lower_bound_s(seg, t, hi << a.lgS);
             const int Lc = imid - ilo - ((sx >= lo && sx < mid) ? 1 : 0);
             const int Rc = ihi - imid - ((sx >= mid && sx < hi) ? 1 : 0);
-            if (Lc > 0) atomicAdd(a.cl + x, (unsigned long long)Lc * wt);
-            if (Rc > 0) atomicAdd(a.cr + x, (unsigned long long)Rc * wt);
+            // only the sign of L - R decides the step (L >= R -> left): one signed counter
+            const long long d = (long long)(Lc - Rc) * (long long)wt;
+            if (d != 0) {
+              if (a.cd32) atomicAdd(static_cast<int *>(a.cd) + x, (int)d);
+              else atomicAdd(static_cast<unsigned long long *>(a.cd) + x, (unsigned long long)d);
+            }
           }
         } else if (MODE == 2) {
           const long long tg = a.target[x];
@@ -172,18 +178,35 @@ __global__ void k_s2_init(int2 *lohi, long long n, int nsec) {
     lohi[v] = make_int2(0, nsec);
 }
 // stage-2 decision: L >= R -> hi = mid, else lo = mid (R21), then reset the counts
-__global__ void k_s2_update(int2 *lohi, unsigned long long *cl, unsigned long long *cr, long long n) {
+__global__ void k_s2_update(int2 *lohi, void *cd, int cd32, long long n) {
   const long long stride = (long long)gridDim.x * blockDim.x;
   for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
     int2 lh = lohi[v];
+    const long long d = cd32 ? (long long)static_cast<int *>(cd)[v] : static_cast<long long *>(cd)[v];
     if (lh.y - lh.x > 1) {
       const int mid = lh.x + (lh.y - lh.x) / 2;
-      if (cl[v] >= cr[v]) lh.y = mid; else lh.x = mid;
+      if (d >= 0) lh.y = mid; else lh.x = mid;   // L >= R -> left half (R21)
       lohi[v] = lh;
     }
-    cl[v] = 0;
-    cr[v] = 0;
+    if (cd32) static_cast<int *>(cd)[v] = 0;
+    else static_cast<long long *>(cd)[v] = 0;
   }
+}
+// in-degree (label-invariant; bounds the stage-2 counters: |L - R| <= in-degree * (B - 1))
+__global__ void k_indeg(const int *__restrict__ col, long long m, unsigned *deg) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long k = (long long)blockIdx.x * blockDim.x + threadIdx.x; k < m; k += stride) atomicAdd(deg + col[k], 1u);
+}
+__global__ void k_max_u32(const unsigned *x, long long n, unsigned *out) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  unsigned mx = 0;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) mx = x[i] > mx ? x[i] : mx;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned y = __shfl_xor_sync(FULL, mx, o);
+    mx = y > mx ? y : mx;
+  }
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
 }
 __global__ void k_s2_final(const int2 *lohi, int *target, long long n) {
   const long long stride = (long long)gridDim.x * blockDim.x;
@@ -338,7 +361,7 @@ static sage_status objective(sage_graph *g, int lgS, unsigned long long *out) {
 }
 
 struct RoundBufs {
-  unsigned long long *loc1 = nullptr, *loc3 = nullptr, *cl = nullptr, *cr = nullptr;
+  unsigned long long *loc1 = nullptr, *loc3 = nullptr, *cl = nullptr;   // cl: stage-2 L - R
   int2 *lohi = nullptr;
   int *target = nullptr, *ids = nullptr, *mids = nullptr, *mids2 = nullptr, *sr = nullptr;
   uint8_t *mover = nullptr, *cand = nullptr;
@@ -350,7 +373,7 @@ struct RoundBufs {
 };
 
 static void free_round(sage_graph *g, RoundBufs &b) {
-  void *ps[] = {b.loc1, b.loc3, b.cl, b.cr, b.lohi, b.target, b.ids, b.mids, b.mids2, b.sr,
+  void *ps[] = {b.loc1, b.loc3, b.cl, b.lohi, b.target, b.ids, b.mids, b.mids2, b.sr,
                 b.mover, b.cand, b.gkeys, b.gkeys2, b.tkeys, b.tkeys2, b.scal, b.tmp};
   for (void *p : ps) dfree(g, p);
   b = RoundBufs();
@@ -370,14 +393,15 @@ static sage_status one_round(sage_graph *g, RoundBufs &b, int lgS, const uint8_t
   a.vw = vw;
   a.loc1 = b.loc1;
   a.loc3 = b.loc3;
-  a.cl = b.cl;
-  a.cr = b.cr;
+  a.cd = b.cl;
+  a.cd32 = (vw == nullptr && g->max_indeg >= 0 &&
+            (unsigned long long)g->max_indeg * (unsigned long long)(g->ladder.B > 1 ? g->ladder.B - 1 : 1) <
+                0x7fffffffull) ? 1 : 0;
   a.lohi = b.lohi;
   a.target = b.target;
   cudaMemsetAsync(b.loc1, 0, sizeof(unsigned long long) * n, g->stream);
   cudaMemsetAsync(b.loc3, 0, sizeof(unsigned long long) * n, g->stream);
   cudaMemsetAsync(b.cl, 0, sizeof(unsigned long long) * n, g->stream);
-  cudaMemsetAsync(b.cr, 0, sizeof(unsigned long long) * n, g->stream);
   // stage 1
   if ((s = launch_sample<0>(g, a)) != SAGE_OK) return s;
   // stage 2: ceil(log2(nsec)) halving sweeps
@@ -385,7 +409,7 @@ static sage_status one_round(sage_graph *g, RoundBufs &b, int lgS, const uint8_t
   const int steps = ceil_log2(nsec);
   for (int it = 0; it < steps; ++it) {
     if ((s = launch_sample<1>(g, a)) != SAGE_OK) return s;
-    k_s2_update<<<grid, 256, 0, g->stream>>>(b.lohi, b.cl, b.cr, n);
+    k_s2_update<<<grid, 256, 0, g->stream>>>(b.lohi, a.cd, a.cd32, n);
   }
   k_s2_final<<<grid, 256, 0, g->stream>>>(b.lohi, b.target, n);
   // stage 3
@@ -488,7 +512,20 @@ static sage_status one_round(sage_graph *g, RoundBufs &b, int lgS, const uint8_t
 static sage_status alloc_round(sage_graph *g, RoundBufs &b, bool with_cand) {
   const long long n = g->n;
   sage_status s;
-  void **ps[] = {(void **)&b.loc1, (void **)&b.loc3, (void **)&b.cl, (void **)&b.cr};
+  if (g->max_indeg < 0) {   // once per graph (label-invariant)
+    unsigned *deg = nullptr;
+    if ((s = dalloc(g, (void **)&deg, sizeof(unsigned) * (size_t)(n + 1))) != SAGE_OK) return s;
+    cudaMemsetAsync(deg, 0, sizeof(unsigned) * (size_t)(n + 1), g->stream);
+    k_indeg<<<g->num_sms * 8, 256, 0, g->stream>>>(g->col, g->m, deg);
+    k_max_u32<<<g->num_sms * 8, 256, 0, g->stream>>>(deg, n, deg + n);
+    unsigned hmax = 0;
+    cudaMemcpyAsync(&hmax, deg + n, sizeof(hmax), cudaMemcpyDeviceToHost, g->stream);
+    cudaError_t e = cudaStreamSynchronize(g->stream);
+    dfree(g, deg);
+    if (e != cudaSuccess) return cuda_fail(g, e, "in-degree");
+    g->max_indeg = (long long)hmax;
+  }
+  void **ps[] = {(void **)&b.loc1, (void **)&b.loc3, (void **)&b.cl};
   for (auto p : ps)
     if ((s = dalloc(g, p, sizeof(unsigned long long) * (size_t)n)) != SAGE_OK) return s;
   if ((s = dalloc(g, (void **)&b.lohi, sizeof(int2) * (size_t)n)) != SAGE_OK) return s;

@@ -76,6 +76,7 @@ struct BfsPushT {
   const Queues *next_q;
   CounterSet *next_cs;
   uint32_t ht = 0;     // shared-memory address of the hub table (HT > 0)
+  unsigned long long *nfc = nullptr;   // fused tiling: |F| of the next list, counted at discovery
 
   __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
 
@@ -190,6 +191,8 @@ struct TravArgs {
   struct TailSmem *tailmem;   // tail mode state (global scratch: only block 0 uses it)
   int steal;            // 0 = ablation: static tile assignment instead of stealing
   int *flist;           // deferred contraction: frontier list (n + slack entries)
+  int *fl[2];           // fused runtime tiling: the frontier list of level L is fl[L & 1]
+  int src;              // fused path: the source (query init runs inside the kernel)
   HubIns hub;           // hub filter: global table + insert rule (hub.g null = off)
   unsigned long long hub_min_arcs;   // reload the CTA's table before levels with arcs(F) >= this
 };
@@ -341,10 +344,34 @@ __device__ __forceinline__ int block_scan_excl(int x, int *out_excl, int *wsum) 
 // lives in a small global scratch block (L1-cached for this CTA) rather than in shared memory, so
 // the persistent kernel's static shared memory — and with it the L1 left for the status words of
 // the main path — is unchanged.
+template <bool FUSED>
 __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
   Ctl *ctl = a.ctl;
   const int tid = threadIdx.x, lane = (int)lane_id(), warp = tid >> 5;
   int nf = 0;
+  if constexpr (FUSED) {
+    // ---- the frontier of level Lstart is its list (each vertex once; -1 = empty slot)
+    const CounterSet *cs = &ctl->set[Lstart % 3];
+    const int *fl = a.fl[Lstart & 1];
+    const long long fc = (long long)ldcg(&cs->flc.v);
+    if (tid == 0) ts.nnext = 0;
+    __syncthreads();
+    for (long long i = tid; i < fc; i += blockDim.x) {   // order is free: compact with a counter
+      const int u = ldcg(fl + i);
+      if (u >= 0) {
+        const int pos = atomicAdd(&ts.nnext, 1);
+        if (pos < kTailV) {
+          const long long rb = a.off[u];
+          ts.f[0][pos] = u;
+          ts.b[0][pos] = rb;
+          ts.d[0][pos] = (int)(a.off[u + 1] - rb);
+        }
+      }
+    }
+    __syncthreads();
+    nf = ts.nnext < kTailV ? ts.nnext : kTailV;
+    __syncthreads();
+  } else {
   // ---- gather the frontier of level Lstart from its log and deduplicate
   {
     const CounterSet *cs = &ctl->set[Lstart % 3];
@@ -390,6 +417,7 @@ __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
     }
     __syncthreads();
   }
+  }
   // statistics kept in registers of thread 0, written once
   unsigned long long s_exp = 0, s_arcs = 0, s_disc = 0, s_reach = 0;
   int cur = 0;
@@ -398,6 +426,15 @@ __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
     // exclusive scan of the frontier's degrees (nf <= kTailV = blockDim: one row per thread)
     int p1;
     const int A = block_scan_excl(tid < nf ? ts.d[cur][tid] : 0, &p1, ts.wsum);
+    if constexpr (FUSED) {
+      if (L == Lstart && A > kTailE) {   // the entering frontier is too heavy: the grid runs it
+        if (tid == 0) {
+          ctl->tail_state = 2;
+          ctl->tail_resume = Lstart;
+        }
+        return;
+      }
+    }
     if (tid < nf) ts.pre[tid] = p1;
     if (tid == 0) {
       ts.pre[nf] = A;
@@ -436,7 +473,7 @@ __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
       s_exp += nf;
       s_arcs += A;
       s_disc += nn;
-      s_reach += an;
+      s_reach += FUSED ? (unsigned long long)A : an;
       if (L < kMaxRec) {
         LevelRec &r = ctl->rec[L];
         r.dir = 0;
@@ -472,7 +509,7 @@ __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
     }
   }
   if (nn == 0 || L + 1 >= a.max_levels) return;
-  // the frontier grew: classify it into level L+1's log and hand back to the grid
+  // the frontier grew: hand level L+1's frontier back to the grid (its list, or its tile log)
   constexpr int nctr = sizeof(CounterSet) / sizeof(PaddedCounter);
   if (tid < nctr) {
     reinterpret_cast<PaddedCounter *>(&ctl->set[(L + 1) % 3])[tid].v = 0ull;
@@ -480,10 +517,19 @@ __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
   }
   __threadfence_block();
   __syncthreads();
-  for (int base = warp * 32; base < nn; base += blockDim.x) {
-    const int i = base + lane;
-    const bool act = i < nn;
-    enqueue_ids(act, act ? ldcg(a.tail + i) : 0, a.off, a.L, a.q[(L + 1) & 1], &ctl->set[(L + 1) % 3]);
+  if constexpr (FUSED) {
+    int *fl = a.fl[(L + 1) & 1];
+    for (int i = tid; i < nn; i += blockDim.x) fl[i] = ldcg(a.tail + i);
+    if (tid == 0) {
+      ctl->set[(L + 1) % 3].flc.v = (unsigned long long)nn;
+      ctl->set[(L + 1) % 3].nF.v = (unsigned long long)nn;
+    }
+  } else {
+    for (int base = warp * 32; base < nn; base += blockDim.x) {
+      const int i = base + lane;
+      const bool act = i < nn;
+      enqueue_ids(act, act ? ldcg(a.tail + i) : 0, a.off, a.L, a.q[(L + 1) & 1], &ctl->set[(L + 1) % 3]);
+    }
   }
   if (tid == 0) {
     ctl->tail_state = 2;
@@ -521,7 +567,10 @@ __device__ __forceinline__ void bfs_body(const TravArgs &a, WarpScratch *wsm, ty
   int dir = 0;
   unsigned long long prev_nF = 1;
   const long long nwords = (a.n + 31) >> 5;
-  if ((threadIdx.x & 31) == 0) wsm[warp].cpos = wsm[warp].cend = 0;
+  if ((threadIdx.x & 31) == 0) {
+    wsm[warp].cpos = wsm[warp].cend = 0;
+    wsm[warp].ndisc = 0;
+  }
   if constexpr (HT > 0) {   // empty table
     for (int i = threadIdx.x; i < HubGeom<HT>::bytes / 4; i += blockDim.x) reinterpret_cast<uint32_t *>(ht)[i] = 0u;
   }
@@ -578,7 +627,7 @@ __device__ __forceinline__ void bfs_body(const TravArgs &a, WarpScratch *wsm, ty
           __syncthreads();
           if (threadIdx.x == 0) ctl->tail_state = 0;
           __syncthreads();
-          tail_run(a, L + 1, *a.tailmem);
+          tail_run<false>(a, L + 1, *a.tailmem);
         }
         grid_barrier(&ctl->bar);
         if (ldcg(&ctl->tail_state) == 1) break;
@@ -596,6 +645,471 @@ __device__ __forceinline__ void bfs_body(const TravArgs &a, WarpScratch *wsm, ty
     }
     prev_nF = nF;
   }
+}
+
+// ============================================================================ fused runtime tiling
+#ifndef SAGE_FUSED_PACK
+#define SAGE_FUSED_PACK 0
+#endif
+// Push-only BFS (the configuration of the headline): Tiled Partitioning runs INSIDE the consumer,
+// as Alg. 2's runtime tiling does (the expand kernel splits each frontier vertex's
+// adjacency list into tiles when it reaches it), instead of as a separate K2' grid phase with its
+// own barrier that re-reads every discovered vertex's row offsets twice.  Per level L:
+//   phase A: every warp takes 32-entry chunks of the level's frontier list (ticket cur->ftk),
+//            loads the rows once, and splits each row (split_row): CTA tiles (>= B) go to the
+//            level's CTA-tile log (device-visible, consumed with stealing in phase B); the
+//            sub-CTA class tiles t = B/2 .. M are consumed right away by lane groups of t/VEC
+//            lanes (tps tiles per warp step, like consume_log); the fragments (< M) by the warp
+//            scan-gather.  Filtered-in vertices are appended to level L+1's list.
+//   grid barrier;
+//   phase B: the CTA tiles (hub rows, the load imbalance Resident Tile Stealing exists for) are
+//            consumed by the stealing consumer (consume_log on class 0 only); one more barrier.
+// |F| of the next list is counted at discovery; arcs(F) of the level in phase A.  The tile log
+// (a3/a4) stays the same decomposition (tests: sage_debug_export_tiles vs the oracle).
+// Hub table refresh while a level runs: the frontier's hubs are inserted into the global table as
+// phase A reaches them, and every warp copies its 1/(warps per CTA) share of the table into the
+// CTA's shared copy every kRefreshChunks chunks.  Entries are single bytes / aligned shorts and
+// only ever change from one visited vertex to another (or from empty), so readers need no sync.
+constexpr int kRefreshChunks = 16;
+template <int HT>
+__device__ __forceinline__ void hub_refresh_share(const TravArgs &a, uint32_t ht_s) {
+  constexpr int nvec = (1 << HubGeom<HT>::lgT) >> 2;   // 4 slots per uint4 of the global table
+  constexpr uint32_t km = (1u << HubGeom<HT>::kbits) - 1u;
+  const int nw = blockDim.x >> 5, w = threadIdx.x >> 5;
+  const int per = (nvec + nw - 1) / nw;
+  const uint4 *g4 = reinterpret_cast<const uint4 *>(a.hub.g);
+  for (int i = w * per + (int)lane_id(); i < (w + 1) * per && i < nvec; i += 32) {
+    const uint4 p = __ldcg(g4 + i);
+    const uint32_t k0 = p.x & km, k1 = p.y & km, k2 = p.z & km, k3 = p.w & km;
+    if constexpr (HubGeom<HT>::kbits == 8) {
+      asm volatile("st.shared.u32 [%0], %1;" ::"r"(ht_s + 4u * i), "r"(k0 | (k1 << 8) | (k2 << 16) | (k3 << 24)));
+    } else {
+      asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(ht_s + 8u * i), "r"(k0 | (k1 << 16)), "r"(k2 | (k3 << 16)));
+    }
+  }
+}
+template <class F> struct HtOf { static constexpr int value = 0; };
+template <int HT> struct HtOf<BfsPushT<HT>> { static constexpr int value = HT; };
+
+template <int VEC, class F>
+__device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, CounterSet *cur, const int *fl_in,
+                                              const Queues &Q, WarpScratch *ws, typename F::Src *fsrc,
+                                              int &bcnt) {
+  const unsigned lane = lane_id();
+  int chunks = 0;
+  const unsigned lt = lanemask_lt();
+  const Ladder &L = a.L;
+  const unsigned long long pol = policy_evict_first();
+  const long long fcount = (long long)ldcg(&cur->flc.v);
+  const bool contig_ok = a.vec_ok && (VEC % 4) == 0;
+  unsigned long long arcs = 0;
+  for (;;) {
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(&cur->ftk.v, 32ull);
+    base = shfl64(base, 0);
+    if ((long long)base >= fcount) break;
+    if constexpr (HtOf<F>::value > 0) {
+      if (++chunks % kRefreshChunks == 0) hub_refresh_share<HtOf<F>::value>(a, f.ht);
+    }
+    const long long i = (long long)base + lane;
+    const int v = i < fcount ? ldcg(fl_in + i) : -1;
+    long long b = 0, e = 0;
+    if (v >= 0) ld_row_pair(a.off, v, &b, &e);
+    const bool act = v >= 0;
+    arcs += act ? (unsigned long long)(e - b) : 0ull;
+    hub_insert(a.hub, v, e - b);
+    RowSplit s{0, 0, 0, 0};
+    if (act) s = split_row(b, e, L);
+    // (1) CTA tiles -> the level's CTA-tile log (one reservation atomic per chunk)
+    {
+      unsigned long long q = act ? (unsigned long long)s.q : 0ull;
+      unsigned long long incq = q;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long y = __shfl_up_sync(FULL, incq, o);
+        if ((int)lane >= o) incq += y;
+      }
+      const unsigned long long totq = shfl64(incq, 31);
+      if (totq) {
+        unsigned long long base0 = 0;
+        if (lane == 0) base0 = atomicAdd(&cur->cnt[0].v, totq);
+        base0 = shfl64(base0, 0);
+        if (q > 0 && q <= SAGE_ENQ_LANEQ) {
+          const unsigned long long bs = base0 + incq - q;
+          for (unsigned long long j = 0; j < q; ++j) st_tile(Q.cta + bs + j, s.b2 + (long long)j * L.B, v, L.B);
+        }
+        unsigned hm = __ballot_sync(FULL, q > SAGE_ENQ_LANEQ);
+        while (hm) {
+          const int src = __ffs(hm) - 1;
+          hm &= hm - 1;
+          const unsigned long long qs = shfl64(q, src);
+          const unsigned long long bs = base0 + shfl64(incq, src) - qs;
+          const long long b2 = (long long)shfl64((unsigned long long)s.b2, src);
+          const int vv = __shfl_sync(FULL, v, src);
+          for (unsigned long long j = lane; j < qs; j += 32) st_tile(Q.cta + bs + j, b2 + (long long)j * L.B, vv, L.B);
+        }
+      }
+    }
+#if SAGE_FUSED_PACK
+    // (2) sub-CTA class tiles, consumed here, all classes of the chunk packed into warp steps: tile
+    //     k of class c (t = B >> c elements, lpt = t / VEC lanes) takes lanes [base_c + k * lpt, ..)
+    //     of the chunk's lane sequence; classes in descending size keep every group aligned.  A
+    //     lane finds its class, tile and owner vertex (nth set bit of the class ballot) and reads
+    //     the owner's row end / residual by shuffle; each lane loads VEC consecutive elements.
+    if (VEC == 4 && contig_ok && (L.B >> 1) <= 32 * VEC) {
+      int cbase[kMaxCls + 1];
+      unsigned cms[kMaxCls];
+      int tl = 0;
+#pragma unroll
+      for (int c = 1; c < kMaxCls; ++c) {
+        cms[c] = 0;
+        cbase[c] = tl;
+        if (c < L.ncls) {
+          const int t = L.B >> c;
+          cms[c] = __ballot_sync(FULL, act && (s.r & t));
+          tl += __popc(cms[c]) * (t / VEC);
+        }
+      }
+      cbase[kMaxCls] = tl;
+      const int nst = (tl + 31) >> 5;
+      auto load_step = [&](int st, int (&vv)[VEC], int &u_out, bool &valid, int &lg) {
+        const int g = st * 32 + (int)lane;
+        valid = g < tl;
+        int c = 1, cb = cbase[1];
+        unsigned m = cms[1];
+#pragma unroll
+        for (int cc = 2; cc < kMaxCls; ++cc)   // unrolled: the arrays stay in registers
+          if (cc < L.ncls && g >= cbase[cc]) {
+            c = cc;
+            cb = cbase[cc];
+            m = cms[cc];
+          }
+        const int t = L.B >> c;
+        const int lgl = L.lgB - c - 2;                 // log2(lanes per tile) = log2(t / 4)
+        const int rel = g - cb;
+        const int k = rel >> lgl, sl = rel & ((1 << lgl) - 1);
+        int owner = 0, kk = k;
+#pragma unroll
+        for (int sh = 16; sh > 0; sh >>= 1) {
+          const int cnt = __popc(m & ((1u << sh) - 1u));
+          if (kk >= cnt) {
+            kk -= cnt;
+            m >>= sh;
+            owner += sh;
+          }
+        }
+        owner &= 31;
+        const long long eo = (long long)shfl64((unsigned long long)e, owner);
+        const int ro = __shfl_sync(FULL, s.r, owner);
+        u_out = __shfl_sync(FULL, v, owner);
+        const long long start = eo - (long long)(ro & (2 * t - 1));
+        int4 c4 = make_int4(0, 0, 0, 0);
+        if (valid) c4 = ld_col4(a.col + start + 4ll * sl, pol);
+        vv[0] = c4.x; vv[1 % VEC] = c4.y; vv[2 % VEC] = c4.z; vv[3 % VEC] = c4.w;
+        lg = 1 << lgl;
+      };
+      int vn[VEC], un = 0, lgn = 1;
+      bool vdn = false;
+      if (nst) load_step(0, vn, un, vdn, lgn);
+      for (int st = 0; st < nst; ++st) {
+        int vv[VEC];
+        uint32_t ww[VEC];
+#pragma unroll
+        for (int j = 0; j < VEC; ++j) {
+          vv[j] = vn[j];
+          ww[j] = 0u;
+        }
+        const int u = un, lg = lgn;
+        const bool valid = vdn;
+        if (st + 1 < nst) load_step(st + 1, vn, un, vdn, lgn);
+        typename F::Src sc = f.src(valid, u, 0, 0);
+        bool in[VEC];
+        f.template visit<VEC>(valid, sc, vv, ww, in, lg);
+#pragma unroll
+        for (int j = 0; j < VEC; ++j) push_filtered(f, in[j], vv[j], ws, bcnt, a.off, L);
+      }
+    } else
+#endif
+    {
+    // (2) sub-CTA class tiles, consumed here: the class members' tile starts and sources are
+    //     staged in shared memory, then lane groups of t/VEC lanes take one tile each per step
+    for (int c = 1; c < L.ncls; ++c) {
+      const int t = L.B >> c;
+      const unsigned cm = __ballot_sync(FULL, act && (s.r & t));
+      if (!cm) continue;
+      const int nt = __popc(cm);
+      __syncwarp();
+      if (cm & (1u << lane)) {
+        const int r = __popc(cm & lt);
+        ws->hb[r] = class_tile_start(e, s.r, t);
+        fsrc[r] = f.src(true, v, b, e);
+      }
+      __syncwarp();
+      const int lpt = (t / VEC) < 32 ? (t / VEC) : 32;
+      const int tps = 32 / lpt;
+      const int spt = (t / VEC) > 32 ? (t / (32 * VEC)) : 1;
+      const int lg_spt = __ffs(spt) - 1;
+      const int sub = lane / lpt, sl = lane % lpt;
+      const bool contiguous = lpt < 32 && contig_ok;
+      const int nst = ((nt + tps - 1) / tps) << lg_spt;
+      int vn[VEC];
+      uint32_t wn[VEC];
+      auto load_step = [&](int st, int (&vv)[VEC], uint32_t (&ww)[VEC]) {
+        const int k = ((st >> lg_spt) * tps) + sub;
+        const bool valid = k < nt;
+        const long long start = ws->hb[valid ? k : 0];
+        if (contiguous) {
+          const long long p0 = start + (long long)sl * VEC;
+#pragma unroll
+          for (int qq = 0; qq < (VEC + 3) / 4; ++qq) {
+            int4 c4 = make_int4(0, 0, 0, 0);
+            if (valid) c4 = ld_col4(a.col + p0 + 4 * qq, pol);
+            vv[(4 * qq) % VEC] = c4.x; vv[(4 * qq + 1) % VEC] = c4.y;
+            vv[(4 * qq + 2) % VEC] = c4.z; vv[(4 * qq + 3) % VEC] = c4.w;
+          }
+        } else {
+          const long long p0 = start + (long long)(st & (spt - 1)) * (lpt * VEC) + sl;
+#pragma unroll
+          for (int j = 0; j < VEC; ++j) vv[j] = valid ? ld_col(a.col + p0 + j * lpt, pol) : 0;
+        }
+#pragma unroll
+        for (int j = 0; j < VEC; ++j) ww[j] = 0u;
+      };
+      load_step(0, vn, wn);
+      for (int st = 0; st < nst; ++st) {
+        int vv[VEC];
+        uint32_t ww[VEC];
+#pragma unroll
+        for (int j = 0; j < VEC; ++j) {
+          vv[j] = vn[j];
+          ww[j] = wn[j];
+        }
+        if (st + 1 < nst) load_step(st + 1, vn, wn);
+        const int k = ((st >> lg_spt) * tps) + sub;
+        const bool valid = k < nt;
+        const typename F::Src sc = fsrc[valid ? k : 0];
+        bool in[VEC];
+        f.template visit<VEC>(valid, sc, vv, ww, in, lpt);
+#pragma unroll
+        for (int j = 0; j < VEC; ++j) push_filtered(f, in[j], vv[j], ws, bcnt, a.off, L);
+      }
+      __syncwarp();
+    }
+    }
+    // (3) fragments (< M, and the aligned head): warp scan-based gather over the chunk's rows
+    {
+      int hl = 0, tl = 0;
+      long long tb = 0;
+      if (act) {
+        hl = s.h;
+        tl = s.r & (L.M - 1);
+        tb = e - tl;
+      }
+      const int fl = hl + tl;
+      int inc = fl;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(FULL, inc, o);
+        if ((int)lane >= o) inc += y;
+      }
+      const int total = __shfl_sync(FULL, inc, 31);
+      if (total) {
+        __syncwarp();
+        ws->pre[lane] = inc - fl;
+        ws->hl[lane] = hl;
+        ws->hb[lane] = b;
+        ws->tb[lane] = (int)(tb - b);
+        fsrc[lane] = f.src(act, v, b, e);
+        __syncwarp();
+        for (int k0 = 0; k0 < total; k0 += 32) {
+          const int k = k0 + (int)lane;
+          const bool kv = k < total;
+          int o = 0;
+          if (kv) {   // largest o with pre[o] <= k
+            int lo = 0, hi = 31;
+#pragma unroll
+            for (int it = 0; it < 5; ++it) {
+              const int mid = (lo + hi + 1) >> 1;
+              if (ws->pre[mid] <= k) lo = mid; else hi = mid - 1;
+            }
+            o = lo;
+          }
+          int vv[1] = {0};
+          uint32_t w1[1] = {0u};
+          const typename F::Src so = fsrc[o];
+          if (kv) {
+            const int idx = k - ws->pre[o];
+            const long long pos = ws->hb[o] + (idx < ws->hl[o] ? idx : ws->tb[o] + (idx - ws->hl[o]));
+            vv[0] = ld_col(a.col + pos, pol);
+          }
+          bool in[1];
+          f.template visit<1>(kv, so, vv, w1, in, 1);
+          push_filtered(f, in[0], vv[0], ws, bcnt, a.off, L);
+        }
+        __syncwarp();
+      }
+    }
+  }
+  arcs = warp_sum64(arcs);
+  if (lane == 0 && arcs) atomicAdd(&cur->arcsF.v, arcs);
+}
+
+// level L's record in the fused path: |F| and arcs(F) of the level itself, discoveries = |F_{L+1}|
+__device__ __forceinline__ void record_level_fused(Ctl *ctl, int L, const CounterSet *cur, const CounterSet *nxt) {
+  const unsigned long long nF = ldcg(&cur->nF.v), aF = ldcg(&cur->arcsF.v), disc = ldcg(&nxt->nF.v);
+  ctl->tot_push_expanded += nF;
+  ctl->tot_push_arcs += aF;
+  ctl->tot_push_disc += disc;
+  ctl->push_levels++;
+  ctl->tot_arcs_reached += aF;
+  ctl->tot_improved += disc;
+  if (L < kMaxRec) {
+    LevelRec &r = ctl->rec[L];
+    r.dir = 0;
+    r.nF = nF;
+    r.arcsF = aF;
+    r.inspected = aF;
+    r.scanned = 0;
+    r.discovered = disc;
+    r.t_ns = globaltimer();
+  }
+  ctl->levels = L + 1;
+}
+
+// Push-only BFS level loop with the fused runtime tiling.
+constexpr unsigned long long kHubReloadMinF = 4096;   // reload the CTA's hub table before such levels
+template <int VEC, int HT>
+__device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *wsm,
+                                               typename BfsPushT<HT>::Src (*fsrc)[32], uint8_t *ht) {
+  const int warp = threadIdx.x >> 5;
+  Ctl *ctl = a.ctl;
+  if ((threadIdx.x & 31) == 0) {
+    wsm[warp].cpos = wsm[warp].cend = 0;
+    wsm[warp].ndisc = 0;
+  }
+  if constexpr (HT > 0) {
+    for (int i = threadIdx.x; i < HubGeom<HT>::bytes / 4; i += blockDim.x) reinterpret_cast<uint32_t *>(ht)[i] = 0u;
+  }
+  // ---- query init (a2, Alg. 1 l.2) inside the kernel: level = -1 (the source 0), visited = 0 (the
+  //      source's bit set), parent = -1, the global hub table and the counters cleared, the source
+  //      seeded as level 0's list; one grid barrier instead of six memsets and a seed launch
+  {
+    const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const long long nth = (long long)gridDim.x * blockDim.x;
+    const int src = a.src;
+    const long long n4 = a.n >> 2;
+    for (long long i = tid; i < n4; i += nth) {
+      int4 x = make_int4(-1, -1, -1, -1);
+      if ((src >> 2) == i) reinterpret_cast<int *>(&x)[src & 3] = 0;
+      reinterpret_cast<int4 *>(a.level)[i] = x;
+      if (a.parent) reinterpret_cast<int4 *>(a.parent)[i] = make_int4(-1, -1, -1, -1);
+    }
+    for (long long i = 4 * n4 + tid; i < a.n; i += nth) {
+      a.level[i] = i == src ? 0 : -1;
+      if (a.parent) a.parent[i] = -1;
+    }
+    const long long words = ((a.n + 31) >> 5) + 8;
+    for (long long i = tid; i < words; i += nth) a.visited[i] = i == (src >> 5) ? 1u << (src & 31) : 0u;
+    if (a.hub.g)
+      for (long long i = tid; i <= (long long)a.hub.mask; i += nth) a.hub.g[i] = 0u;
+    if (blockIdx.x == 0) {
+      constexpr int nctr = sizeof(CounterSet) / sizeof(PaddedCounter);
+      for (int i = threadIdx.x; i < 3 * nctr; i += blockDim.x) reinterpret_cast<PaddedCounter *>(ctl->set)[i].v = 0ull;
+      if (threadIdx.x == 0) {
+        ctl->tot_push_expanded = ctl->tot_push_arcs = ctl->tot_push_disc = 0;
+        ctl->tot_pull_scanned = ctl->tot_pull_inspected = ctl->tot_pull_disc = 0;
+        ctl->tot_arcs_reached = ctl->tot_improved = ctl->tail_levels = 0;
+        ctl->levels = ctl->push_levels = ctl->pull_levels = ctl->status = 0;
+        ctl->tail_state = ctl->tail_resume = 0;
+        ctl->rec[0].t_work = ctl->rec[0].t_mid = 0;
+        ctl->t0_ns = globaltimer();
+      }
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        a.fl[0][0] = src;
+        ctl->set[0].flc.v = 1ull;
+        ctl->set[0].nF.v = 1ull;
+      }
+    }
+    grid_barrier(&ctl->bar);
+  }
+  for (int L = 0;; ++L) {
+    CounterSet *cur = &ctl->set[L % 3];
+    CounterSet *nxt = &ctl->set[(L + 1) % 3];
+    __syncthreads();   // block 0: record of L-1 finished before set (L+2)%3 is zeroed
+    if (L > 0) zero_counterset(&ctl->set[(L + 2) % 3]);
+    if (blockIdx.x == 0 && threadIdx.x == 0 && L + 1 < kMaxRec) ctl->rec[L + 1].t_work = ctl->rec[L + 1].t_mid = 0;
+    if constexpr (HT > 0) {
+      if (ldcg(&cur->nF.v) >= kHubReloadMinF) {
+        hub_load<HT>(a, ht);
+        __syncthreads();
+      }
+    }
+    BfsPushT<HT> f;
+    f.visited = a.visited;
+    f.level = a.level;
+    f.parent = a.parent;
+    f.fb_next = nullptr;
+    f.next_level = L + 1;
+    f.v_base = 0;
+    f.next_q = &a.q[(L + 1) & 1];
+    f.next_cs = nxt;
+    f.flist = a.fl[(L + 1) & 1];
+    f.flc = &nxt->flc.v;
+    f.nfc = &nxt->nF.v;
+    if constexpr (HT > 0) f.ht = (uint32_t)__cvta_generic_to_shared(ht);
+    int bcnt = 0;
+    fused_phase_a<VEC>(a, f, cur, a.fl[L & 1], a.q[L & 1], &wsm[warp], fsrc[warp], bcnt);
+    defer_close(&wsm[warp], bcnt, f.flist, f.flc, f.nfc);
+    if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
+    grid_barrier(&ctl->bar);
+    if (blockIdx.x == 0 && threadIdx.x == 0 && L < kMaxRec) ctl->rec[L].t_mid = globaltimer();
+    if (ldcg(&cur->cnt[0].v) > 0) {   // phase B: the CTA tiles, with Resident Tile Stealing
+      if constexpr (HT > 0) {   // with the hubs phase A inserted
+        if (ldcg(&cur->nF.v) >= kHubReloadMinF) {
+          hub_load<HT>(a, ht);
+          __syncthreads();
+        }
+      }
+      consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok,
+                       a.steal != 0);
+      grid_barrier(&ctl->bar);
+    }
+    const unsigned long long nF = ldcg(&nxt->nF.v);
+    if (blockIdx.x == 0 && threadIdx.x == 0) record_level_fused(ctl, L, cur, nxt);
+    if (nF == 0) break;
+    if (L + 1 >= a.max_levels) {
+      if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = 1;
+      break;
+    }
+    // small frontier: block 0 runs the next levels alone (it hands back when arcs(F) is large)
+    if (nF <= kTailV) {
+      if (blockIdx.x == 0) {
+        __syncthreads();
+        if (threadIdx.x == 0) ctl->tail_state = 0;
+        __syncthreads();
+        tail_run<true>(a, L + 1, *a.tailmem);
+      }
+      grid_barrier(&ctl->bar);
+      if (ldcg(&ctl->tail_state) == 1) break;
+      L = ldcg(&ctl->tail_resume) - 1;   // ++L resumes the grid at the returned level
+      continue;
+    }
+  }
+}
+
+template <int VEC>
+__global__ void __launch_bounds__(kBlock, 4) k_bfs_fused(const __grid_constant__ TravArgs a) {
+  __shared__ WarpScratch wsm[kWarps];
+  __shared__ BfsPush::Src fsrc[kWarps][32];
+  bfs_body_fused<VEC, 0>(a, wsm, fsrc, nullptr);
+}
+template <int VEC, int HT>
+__global__ void __launch_bounds__(1024, 1) k_bfs_fused_hub(const __grid_constant__ TravArgs a) {
+  __shared__ WarpScratch wsm[32];
+  __shared__ typename BfsPushT<HT>::Src fsrc[32][32];
+  extern __shared__ __align__(16) uint8_t hub_smem[];
+  bfs_body_fused<VEC, HT>(a, wsm, fsrc, hub_smem);
 }
 
 template <int VEC>
@@ -623,7 +1137,10 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
   const long long nwords = (a.n + 31) >> 5;
-  if ((threadIdx.x & 31) == 0) wsm[warp].cpos = wsm[warp].cend = 0;
+  if ((threadIdx.x & 31) == 0) {
+    wsm[warp].cpos = wsm[warp].cend = 0;
+    wsm[warp].ndisc = 0;
+  }
   if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t0_ns = globaltimer();
   for (int L = 0;; ++L) {
     CounterSet *cur = &ctl->set[L % 3];
@@ -655,8 +1172,18 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
 }
 
 // Seed the level-0 log with the source (one warp).
-__global__ void k_seed(TravArgs a, int src, int mode /*0 bfs, 1 sssp*/) {
+__global__ void k_seed(TravArgs a, int src, int mode /*0 bfs, 1 sssp, 2 bfs with fused tiling*/) {
   const bool act = threadIdx.x == 0;
+  if (mode == 2) {   // level 0's frontier list = {src}
+    if (act) {
+      a.visited[src >> 5] |= 1u << (src & 31);
+      a.level[src] = 0;
+      a.fl[0][0] = src;
+      a.ctl->set[0].flc.v = 1ull;
+      a.ctl->set[0].nF.v = 1ull;
+    }
+    return;
+  }
   long long b = 0, e = 0;
   if (act) {
     b = a.off[src];
@@ -823,6 +1350,13 @@ void free_traversal_state(sage_graph *g) {
   dfree(g, t.tailmem);
   dfree(g, t.flist);
   dfree(g, t.hub_g);
+  dfree(g, t.flist2);
+  for (int i = 0; i < 3; ++i)
+    if (t.ev[i]) cudaEventDestroy(t.ev[i]);
+  if (t.hctl) {
+    cudaStreamSynchronize(g->stream);
+    cudaFreeHost(t.hctl);
+  }
   t = TraversalState();
 }
 
@@ -859,6 +1393,14 @@ sage_status ensure_traversal_state(sage_graph *g) {
       free_traversal_state(g);
       return st;
     }
+  cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);   // the grid barrier starts consistent
+  for (int i = 0; i < 3; ++i) cudaEventCreate(&t.ev[i]);
+  if (cudaMallocHost((void **)&t.hctl, sizeof(Ctl)) != cudaSuccess) {
+    cudaGetLastError();
+    free_traversal_state(g);
+    set_error("pinned host allocation failed");
+    return SAGE_E_NOMEM;
+  }
   t.ready = true;
   return SAGE_OK;
 }
@@ -1048,25 +1590,31 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   const int32_t src = to_internal_id(g, source);
   const bool symmetric = g->flags & SAGE_F_SYMMETRIC;
   const bool push_only = (g->flags | call_flags) & SAGE_F_PUSH_ONLY;
-  cudaEvent_t e0, e1, e2;
-  cudaEventCreate(&e0);
-  cudaEventCreate(&e1);
-  cudaEventCreate(&e2);
+  const bool do_enabled = symmetric && !push_only;
+#ifdef SAGE_NO_FUSED
+  const bool fused = false;
+#else
+  const bool fused = !do_enabled;   // push-only: Tiled Partitioning fused into the consumer
+#endif
+  cudaEvent_t e0 = t.ev[0], e1 = t.ev[1], e2 = t.ev[2];
   cudaEventRecord(e0, g->stream);
   const size_t words = (size_t)((g->n + 31) / 32 + 8);
-  cudaMemsetAsync(t.level, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
-  if (parent_out) cudaMemsetAsync(t.parent, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
-  cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
-  for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
-  cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);
+  if (!fused) {   // (the fused kernel initialises its query state itself)
+    cudaMemsetAsync(t.level, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
+    if (parent_out) cudaMemsetAsync(t.parent, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
+    cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
+    for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
+    cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);
+  }
   TravArgs a = make_args(g);
   a.parent = parent_out ? t.parent : nullptr;
-  a.do_enabled = (symmetric && !push_only) ? 1 : 0;
+  a.do_enabled = do_enabled ? 1 : 0;
   a.steal = (call_flags & SAGE_F_NO_STEALING) ? 0 : 1;
+  a.src = src;
   if (const int ht = hub_mode(g)) {
     const int lgT = hub_lgT(ht);
     if (!t.hub_g && (s = dalloc(g, (void **)&t.hub_g, sizeof(uint32_t) << 17)) != SAGE_OK) return s;
-    cudaMemsetAsync(t.hub_g, 0, sizeof(uint32_t) << lgT, g->stream);
+    if (!fused) cudaMemsetAsync(t.hub_g, 0, sizeof(uint32_t) << lgT, g->stream);
     a.hub.g = t.hub_g;
     a.hub.lgT = lgT;
     a.hub.mask = (1u << lgT) - 1u;
@@ -1074,9 +1622,28 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
     a.hub.thr = std::max<long long>(2, 2 * ((g->m + g->n_local - 1) / std::max<long long>(1, g->n_local)));
     a.hub_min_arcs = kHubMinLevelArcs;
   }
-  k_seed<<<1, 32, 0, g->stream>>>(a, src, 0);
+  if (fused) {
+    if (!t.flist2 && (s = dalloc(g, (void **)&t.flist2,
+                                 sizeof(int) * (size_t)(g->n_local + (long long)g->num_sms * 64 * kDeferChunk + 64))) != SAGE_OK)
+      return s;
+    a.fl[0] = t.flist;
+    a.fl[1] = t.flist2;
+  }
+  if (!fused) k_seed<<<1, 32, 0, g->stream>>>(a, src, 0);
   cudaEventRecord(e1, g->stream);
-  {
+  if (fused) {
+    const int ht = hub_mode(g);
+    const void *fn = ht == 1 ? (const void *)k_bfs_fused_hub<4, 1>
+                   : ht == 2 ? (const void *)k_bfs_fused_hub<4, 2>
+                   : ht == 3 ? (const void *)k_bfs_fused_hub<4, 3>
+                   : ht == 4 ? (const void *)k_bfs_fused_hub<4, 4>
+                   : g->vec == 4 ? (const void *)k_bfs_fused<4> : (const void *)k_bfs_fused<1>;
+    const int block = ht ? kHubBlock : kBlock;
+    const size_t dyn = ht ? hub_bytes(ht) : 0;
+    const int grid = coop_grid(g, fn, ht ? &g->grid_bfs_fused_hub : &g->grid_bfs_fused, block, dyn);
+    void *args[] = {&a};
+    if ((s = launch_coop(g, fn, grid, args, "BFS kernel", block, dyn)) != SAGE_OK) return s;
+  } else {
     const int ht = hub_mode(g);
     const void *fn = ht == 1 ? (const void *)k_bfs_hub<4, 1>
                    : ht == 2 ? (const void *)k_bfs_hub<4, 2>
@@ -1097,26 +1664,22 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
     (void)block;
   }
   cudaEventRecord(e2, g->stream);
-  Ctl h;
+  // counters and outputs in one stream round trip (one synchronisation per call)
+  Ctl &h = *t.hctl;
   cudaMemcpyAsync(&h, t.ctl, offsetof(Ctl, rec), cudaMemcpyDeviceToHost, g->stream);
+  if ((s = translate_out_i32(g, t.level, level_out, false)) != SAGE_OK) return s;
+  if (parent_out && (s = translate_out_i32(g, t.parent, parent_out, true)) != SAGE_OK) return s;
   cudaError_t e = cudaStreamSynchronize(g->stream);
   if (e != cudaSuccess) return cuda_fail(g, e, "BFS");
   float ms = 0, kms = 0;
   cudaEventElapsedTime(&ms, e0, e2);
   cudaEventElapsedTime(&kms, e1, e2);
-  cudaEventDestroy(e0);
-  cudaEventDestroy(e1);
-  cudaEventDestroy(e2);
   if (h.status == 1) {
     set_error("BFS exceeded the level cap (internal error)");
     g->sticky = SAGE_E_CUDA;
     return SAGE_E_CUDA;
   }
   fill_stats(g, h, true, symmetric, ms, kms, st);
-  if ((s = translate_out_i32(g, t.level, level_out, false)) != SAGE_OK) return s;
-  if (parent_out && (s = translate_out_i32(g, t.parent, parent_out, true)) != SAGE_OK) return s;
-  e = cudaStreamSynchronize(g->stream);
-  if (e != cudaSuccess) return cuda_fail(g, e, "BFS output");
   // online sampling: record the rows this query expanded (after the answer has been delivered)
   return online_after_query(g, t.level, 0);
 }

@@ -162,6 +162,7 @@ struct LoopXport : Xport {
     cudaEventRecord(me.done, g->stream);
     grp->barrier();
     for (int q = 0; q < world; ++q) cudaStreamWaitEvent(g->stream, grp->slot[q].done, 0);
+    grp->barrier();   // no rank may destroy its events (sage_free) while another still waits on them
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(g, e, "loopback collective");
     return SAGE_OK;
@@ -216,6 +217,7 @@ struct LoopXport : Xport {
 
 Xport *make_loopback_xport(sage_graph *g, const void *id128, int rank, int world, sage_status *st) {
   const char *id = static_cast<const char *>(id128);
+  *st = SAGE_OK;
   if (memcmp(id, kLoopMagic, sizeof(kLoopMagic)) != 0) return nullptr;
   LoopGroup *grp = nullptr;
   memcpy(&grp, id + 16, sizeof(grp));

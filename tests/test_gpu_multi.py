@@ -1,9 +1,10 @@
 """The NCCL multi-GPU path (1D partition) on a 1-rank communicator.
 
-gpurun and the round-end runs expose one GPU, so world > 1 cannot run here; with dist != NULL and
-world == 1 the library takes exactly the host-sequenced NCCL path (padded layout, per-level stats
-allreduce, frontier allgather before pull levels, dense alltoall loop, PR reduce-scatter).  The
-protocol itself with two ranks is checked on CPU by tests/test_partition_model.py (gloo).
+gpurun and the round-end runs expose one GPU, so world > 1 cannot run on NCCL here; with
+dist != NULL and world == 1 the library takes exactly the host-sequenced NCCL path (padded layout,
+per-level stats allreduce, frontier allgather before pull levels, PR reduce-scatter).  World 2-4
+runs on one GPU through the loopback transport in tests/test_gpu_multi_loopback.py, and the
+protocol is modelled on CPU with gloo in tests/test_partition_model.py.
 """
 import numpy as np
 import pytest
@@ -41,9 +42,12 @@ def test_nccl_path_bfs_pagerank(sage, sym):
         x, _ = G.pagerank(0.85, 20)
         xr = oracle.pagerank(g.off, g.col, 0.85, 20)
         assert np.max(np.abs(x - xr) / xr) <= 1e-6
-        with pytest.raises(sage.SageError) as ei:
-            G.bfs(0, parents=True)
-        assert ei.value.status == sage.E_UNSUPPORTED
+        s = int(sg.sources(g, 1, seed=4)[0])
+        lv, par, _ = G.bfs(s, parents=True)       # parents on the multi-GPU path (post-pass)
+        ref = oracle.bfs(g.off, g.col, s)
+        assert par[s] == -1 and np.all(par[ref < 0] == -1)
+        ok = ref > 0
+        assert np.all(ref[par[ok]] == ref[ok] - 1)
 
 
 @pytest.mark.parametrize("sym", [True, False])

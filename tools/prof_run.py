@@ -26,7 +26,8 @@ elif a.graph == "uk":
 else:
     g = sg.twitter_like(n=a.n or 4_000_000, tuples=(a.n or 4_000_000) * 36, seed=1)
 w = sg.weights(g, 1)
-s = stream = torch.cuda.current_stream()
+s = stream = torch.cuda.Stream()   # the library's work and the events on one stream
+torch.cuda.set_stream(stream)
 G = sage.load_csr(torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda(), torch.from_numpy(w).cuda(),
                   symmetric=g.symmetric, borrow=True, stream=stream.cuda_stream, tile_cta=a.tile_cta, align=a.align)
 src = sg.sources(g, a.reps, seed=2)

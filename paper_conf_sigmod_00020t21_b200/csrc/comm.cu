@@ -72,6 +72,8 @@ struct Comm {
   uint32_t *sp_send = nullptr, *sp_recv = nullptr;   // sparse exchange: p blocks of (cap + 2) words
   long long sp_words = 0;                            // allocated words of each
   int32_t *glevel = nullptr;         // parents: allgathered levels (p*P, padded layout)
+  unsigned long long *hmap = nullptr, *dmap = nullptr;   // mapped pinned stats (16 u64) + device alias
+  unsigned long long pub_seq = 0;
   uint32_t *pcand = nullptr, *pown = nullptr;        // parents: p*P proposals, own P after min
   PartMap pm;
 };
@@ -649,6 +651,13 @@ sage_status init_comm(sage_graph *g, const sage_dist *ds) {
     return s;
   for (int i = 0; i < 3; ++i)
     if ((s = dalloc(g, (void **)&c->fb[i], 4 * words)) != SAGE_OK) return s;
+  if (cudaHostAlloc((void **)&c->hmap, 16 * sizeof(unsigned long long), cudaHostAllocMapped) != cudaSuccess ||
+      cudaHostGetDevicePointer((void **)&c->dmap, c->hmap, 0) != cudaSuccess) {
+    cudaGetLastError();
+    set_error("mapped pinned host memory unavailable");
+    return SAGE_E_NOMEM;
+  }
+  memset(c->hmap, 0, 16 * sizeof(unsigned long long));
   return SAGE_OK;
 }
 
@@ -671,19 +680,42 @@ void free_comm(sage_graph *g) {
   dfree(g, c->pcand);
   dfree(g, c->pown);
   cudaStreamSynchronize(g->stream);
+  if (c->hmap) cudaFreeHost(c->hmap);
   delete c->x;
   delete c;
   g->comm = nullptr;
+}
+
+// The per-level stats reach the host through mapped pinned memory: a one-warp kernel copies the
+// allreduced counters and then a sequence number (after a system-scope fence), and the host spins
+// on that number instead of synchronising the stream (no driver round trip per level).
+__global__ void k_publish(const unsigned long long *src, int n, volatile unsigned long long *dst,
+                          unsigned long long seq) {
+  if (threadIdx.x < (unsigned)n) dst[threadIdx.x] = src[threadIdx.x];
+  __threadfence_system();
+  __syncwarp();
+  if (threadIdx.x == 0) dst[15] = seq;
+}
+static sage_status wait_published(sage_graph *g, unsigned long long *h6, int n) {
+  Comm *c = g->comm;
+  const unsigned long long seq = ++c->pub_seq;
+  k_publish<<<1, 32, 0, g->stream>>>(c->stats + 8, n, c->dmap, seq);
+  volatile unsigned long long *hm = c->hmap;
+  for (unsigned long long spins = 0; hm[15] != seq; ++spins) {
+    if ((spins & 4095) == 4095) {   // the stream failed or is slow: look at it
+      const cudaError_t q = cudaStreamQuery(g->stream);
+      if (q != cudaSuccess && q != cudaErrorNotReady) return cuda_fail(g, q, "stats");
+    }
+  }
+  for (int i = 0; i < n; ++i) h6[i] = hm[i];
+  return SAGE_OK;
 }
 
 static sage_status allreduce_stats(sage_graph *g, int L, unsigned long long *h6) {
   Comm *c = g->comm;
   k_mstats<<<1, 32, 0, g->stream>>>(g->ts.ctl, L % 3, (L + 1) % 3, c->stats);
   XCHECK(c->x->allreduce_sum_u64(g, c->stats, c->stats + 8, 6));
-  cudaMemcpyAsync(h6, c->stats + 8, sizeof(unsigned long long) * 6, cudaMemcpyDeviceToHost, g->stream);
-  cudaError_t e = cudaStreamSynchronize(g->stream);
-  if (e != cudaSuccess) return cuda_fail(g, e, "stats");
-  return SAGE_OK;
+  return wait_published(g, h6, 6);
 }
 
 sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int32_t *parent_out,
@@ -730,9 +762,7 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
   {
     k_mstats<<<1, 32, 0, g->stream>>>(t.ctl, 2, 0, c->stats);   // set[0] = the seed's log
     XCHECK(c->x->allreduce_sum_u64(g, c->stats, c->stats + 8, 6));
-    cudaMemcpyAsync(h6, c->stats + 8, sizeof(h6), cudaMemcpyDeviceToHost, g->stream);
-    cudaError_t e = cudaStreamSynchronize(g->stream);
-    if (e != cudaSuccess) return cuda_fail(g, e, "seed");
+    XCHECK(wait_published(g, h6, 6));
   }
   double mU = (double)c->m_total - (double)h6[1];
   unsigned long long reached_arcs = h6[1];

@@ -65,6 +65,7 @@ struct CounterSet {                      // counters of one log (rotated over 3 
   PaddedCounter scanned;                 // pull: unvisited non-isolated vertices scanned
   PaddedCounter flc;                     // deferred contraction: frontier-list slots reserved
   PaddedCounter ftk;                     // fused tiling: frontier-list chunk tickets
+  PaddedCounter hubc;                    // fused tiling: hub-table slots changed in this level
 };
 
 struct LevelRec {                        // per-level record (first kMaxRec levels)
@@ -313,7 +314,8 @@ __device__ __forceinline__ long long class_tile_start(long long e, int r, int t)
 // All queue reservations of one call are issued in ONE parallel round of atomics (lane c reserves
 // for queue c), so a call costs a single atomic latency whatever the number of classes.
 __device__ __forceinline__ void enqueue_warp(bool active, int v, long long b, long long e,
-                                             const Ladder &L, const Queues &Q, CounterSet *cs) {
+                                             const Ladder &L, const Queues &Q, CounterSet *cs,
+                                             bool count_f = true) {
   const unsigned am = __ballot_sync(FULL, active);
   if (!am) return;
   const unsigned lane = lane_id();
@@ -350,9 +352,9 @@ __device__ __forceinline__ void enqueue_warp(bool active, int v, long long b, lo
   } else if (lane == 29) {
     if (Q.order) mybase = atomicAdd(Q.order_cnt, (unsigned long long)__popc(am));
   } else if (lane == 30) {
-    atomicAdd(&cs->nF.v, (unsigned long long)__popc(am));
+    if (count_f) atomicAdd(&cs->nF.v, (unsigned long long)__popc(am));
   } else if (lane == 31) {
-    if (deg) atomicAdd(&cs->arcsF.v, deg);
+    if (deg && count_f) atomicAdd(&cs->arcsF.v, deg);
   }
   if (Q.order) {
     const unsigned long long ob = shfl64(mybase, 29);
@@ -589,14 +591,17 @@ struct HubIns {
   int kbits = 0;           // key field bits (8 or 16); degree in the upper 32 - kbits bits
   long long thr = 0;       // minimum degree of an inserted vertex
 };
-__device__ __forceinline__ void hub_insert(const HubIns &h, int v, long long deg) {
+// returns 1 when the slot changed (the caller counts changes to decide when to reload)
+__device__ __forceinline__ int hub_insert(const HubIns &h, int v, long long deg) {
   if (h.g && v >= 0 && deg >= h.thr) {
     const uint32_t k1 = ((uint32_t)v >> h.lgT) + 1u;
-    if (k1 >> h.kbits) return;
+    if (k1 >> h.kbits) return 0;
     const unsigned long long dmax = (1ull << (32 - h.kbits)) - 1;
     const uint32_t d = (uint32_t)((unsigned long long)deg < dmax ? (unsigned long long)deg : dmax);
-    atomicMax(h.g + ((uint32_t)v & h.mask), (d << h.kbits) | k1);
+    const uint32_t nv = (d << h.kbits) | k1;
+    return atomicMax(h.g + ((uint32_t)v & h.mask), nv) < nv ? 1 : 0;
   }
+  return 0;
 }
 
 __device__ __forceinline__ bool classify_deferred(const long long *__restrict__ off, const int *flist,

@@ -48,6 +48,7 @@ struct SampleArgs {
   const int *target;
   unsigned long long *objective;
   const uint32_t *vw;          // online sampling: occurrences of each vertex's tiles (null = 1)
+  int xlo, xhi;                // this sweep updates the counters of members x in [xlo, xhi) only
 };
 
 // first index i in seg[0, len) with seg[i] >= key (seg sorted ascending)
@@ -134,6 +135,7 @@ __global__ void __launch_bounds__(256) k_sample(const __grid_constant__ SampleAr
         const int pos = t < 32 ? lane % G : i;
         if (!tv || (MODE != 3 && wt == 0)) continue;
         const int x = seg[pos];
+        if (MODE != 3 && (x < a.xlo || x >= a.xhi)) continue;
         const long long sx = (long long)x >> a.lgS;
         if (MODE == 0) {
           const int cnt = lower_bound_s(seg, t, (sx + 1) << a.lgS) - lower_bound_s(seg, t, sx << a.lgS) - 1;
@@ -331,13 +333,24 @@ static sage_status sample_args(sage_graph *g, SampleArgs *a, int lgS) {
   return SAGE_OK;
 }
 
+// A sweep's counter updates are random over the n members; when the counters do not fit L2 the
+// sweep runs in passes over member ranges of at most kPassBytes of counters each (every pass reads
+// the sample again, ~1 ms of column stream at C3, but its atomics stay L2-resident).
+constexpr size_t kPassBytes = 48ull << 20;
 template <int MODE>
-static sage_status launch_sample(sage_graph *g, const SampleArgs &a) {
+static sage_status launch_sample(sage_graph *g, const SampleArgs &a0, size_t counter_bytes = 8) {
   const int bufn = g->ladder.B > 32 ? g->ladder.B : 32;
   const size_t smem = sizeof(int) * (size_t)bufn * 8;
   if (smem > 48 * 1024)
     cudaFuncSetAttribute(k_sample<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  k_sample<MODE><<<g->num_sms * 8, 256, smem, g->stream>>>(a);
+  const long long n = g->n;
+  const int passes = MODE == 3 ? 1 : (int)std::max<long long>(1, ((long long)counter_bytes * n + kPassBytes - 1) / (long long)kPassBytes);
+  for (int p = 0; p < passes; ++p) {
+    SampleArgs a = a0;
+    a.xlo = (int)(n * p / passes);
+    a.xhi = (int)(n * (p + 1) / passes);
+    k_sample<MODE><<<g->num_sms * 8, 256, smem, g->stream>>>(a);
+  }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(g, e, "reorder sample sweep");
   return SAGE_OK;
@@ -408,7 +421,7 @@ static sage_status one_round(sage_graph *g, RoundBufs &b, int lgS, const uint8_t
   k_s2_init<<<grid, 256, 0, g->stream>>>(b.lohi, n, (int)nsec);
   const int steps = ceil_log2(nsec);
   for (int it = 0; it < steps; ++it) {
-    if ((s = launch_sample<1>(g, a)) != SAGE_OK) return s;
+    if ((s = launch_sample<1>(g, a, a.cd32 ? 4 : 8)) != SAGE_OK) return s;
     k_s2_update<<<grid, 256, 0, g->stream>>>(b.lohi, a.cd, a.cd32, n);
   }
   k_s2_final<<<grid, 256, 0, g->stream>>>(b.lohi, b.target, n);

@@ -691,10 +691,15 @@ __device__ __forceinline__ void hub_refresh_share(const TravArgs &a, uint32_t ht
 template <class F> struct HtOf { static constexpr int value = 0; };
 template <int HT> struct HtOf<BfsPushT<HT>> { static constexpr int value = HT; };
 
+// Small frontiers (|F| < kFusedLogAll): one warp per chunk would expand its rows' sub-CTA tiles
+// serially; instead phase A only classifies (Tiled Partitioning into the level's log, every class)
+// and phase B consumes the whole log with stealing — the latency of a small level is then one
+// classification round plus one parallel consume, as with the separate K2' phase.
+constexpr unsigned long long kFusedLogAll = 8192;
 template <int VEC, class F>
 __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, CounterSet *cur, const int *fl_in,
                                               const Queues &Q, WarpScratch *ws, typename F::Src *fsrc,
-                                              int &bcnt) {
+                                              int &bcnt, bool log_all) {
   const unsigned lane = lane_id();
   int chunks = 0;
   const unsigned lt = lanemask_lt();
@@ -703,6 +708,7 @@ __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, Cou
   const long long fcount = (long long)ldcg(&cur->flc.v);
   const bool contig_ok = a.vec_ok && (VEC % 4) == 0;
   unsigned long long arcs = 0;
+  unsigned hubc = 0;
   for (;;) {
     unsigned long long base = 0;
     if (lane == 0) base = atomicAdd(&cur->ftk.v, 32ull);
@@ -717,7 +723,11 @@ __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, Cou
     if (v >= 0) ld_row_pair(a.off, v, &b, &e);
     const bool act = v >= 0;
     arcs += act ? (unsigned long long)(e - b) : 0ull;
-    hub_insert(a.hub, v, e - b);
+    hubc += (unsigned)hub_insert(a.hub, v, e - b);
+    if (log_all) {   // small frontier: classify every tile into the log; phase B consumes it
+      enqueue_warp(act, v, b, e, L, Q, cur, false);
+      continue;
+    }
     RowSplit s{0, 0, 0, 0};
     if (act) s = split_row(b, e, L);
     // (1) CTA tiles -> the level's CTA-tile log (one reservation atomic per chunk)
@@ -952,6 +962,8 @@ __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, Cou
   }
   arcs = warp_sum64(arcs);
   if (lane == 0 && arcs) atomicAdd(&cur->arcsF.v, arcs);
+  const unsigned long long hc = warp_sum64((unsigned long long)hubc);
+  if (lane == 0 && hc) atomicAdd(&cur->hubc.v, hc);
 }
 
 // level L's record in the fused path: |F| and arcs(F) of the level itself, discoveries = |F_{L+1}|
@@ -977,7 +989,7 @@ __device__ __forceinline__ void record_level_fused(Ctl *ctl, int L, const Counte
 }
 
 // Push-only BFS level loop with the fused runtime tiling.
-constexpr unsigned long long kHubReloadMinF = 4096;   // reload the CTA's hub table before such levels
+constexpr unsigned long long kHubReloadMinChanges = 256;   // reload the CTA's hub table after such levels
 template <int VEC, int HT>
 __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *wsm,
                                                typename BfsPushT<HT>::Src (*fsrc)[32], uint8_t *ht) {
@@ -999,8 +1011,9 @@ __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *w
     const int src = a.src;
     const long long n4 = a.n >> 2;
     for (long long i = tid; i < n4; i += nth) {
-      int4 x = make_int4(-1, -1, -1, -1);
-      if ((src >> 2) == i) reinterpret_cast<int *>(&x)[src & 3] = 0;
+      const bool here = (src >> 2) == i;
+      const int4 x = make_int4(here && (src & 3) == 0 ? 0 : -1, here && (src & 3) == 1 ? 0 : -1,
+                               here && (src & 3) == 2 ? 0 : -1, here && (src & 3) == 3 ? 0 : -1);
       reinterpret_cast<int4 *>(a.level)[i] = x;
       if (a.parent) reinterpret_cast<int4 *>(a.parent)[i] = make_int4(-1, -1, -1, -1);
     }
@@ -1039,12 +1052,6 @@ __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *w
     __syncthreads();   // block 0: record of L-1 finished before set (L+2)%3 is zeroed
     if (L > 0) zero_counterset(&ctl->set[(L + 2) % 3]);
     if (blockIdx.x == 0 && threadIdx.x == 0 && L + 1 < kMaxRec) ctl->rec[L + 1].t_work = ctl->rec[L + 1].t_mid = 0;
-    if constexpr (HT > 0) {
-      if (ldcg(&cur->nF.v) >= kHubReloadMinF) {
-        hub_load<HT>(a, ht);
-        __syncthreads();
-      }
-    }
     BfsPushT<HT> f;
     f.visited = a.visited;
     f.level = a.level;
@@ -1059,18 +1066,23 @@ __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *w
     f.nfc = &nxt->nF.v;
     if constexpr (HT > 0) f.ht = (uint32_t)__cvta_generic_to_shared(ht);
     int bcnt = 0;
-    fused_phase_a<VEC>(a, f, cur, a.fl[L & 1], a.q[L & 1], &wsm[warp], fsrc[warp], bcnt);
+    const bool log_all = ldcg(&cur->nF.v) < kFusedLogAll;
+    fused_phase_a<VEC>(a, f, cur, a.fl[L & 1], a.q[L & 1], &wsm[warp], fsrc[warp], bcnt, log_all);
     defer_close(&wsm[warp], bcnt, f.flist, f.flc, f.nfc);
     if ((threadIdx.x & 31) == 0 && L < kMaxRec) atomicMax(&ctl->rec[L].t_work, globaltimer());
     grid_barrier(&ctl->bar);
     if (blockIdx.x == 0 && threadIdx.x == 0 && L < kMaxRec) ctl->rec[L].t_mid = globaltimer();
-    if (ldcg(&cur->cnt[0].v) > 0) {   // phase B: the CTA tiles, with Resident Tile Stealing
-      if constexpr (HT > 0) {   // with the hubs phase A inserted
-        if (ldcg(&cur->nF.v) >= kHubReloadMinF) {
-          hub_load<HT>(a, ht);
-          __syncthreads();
-        }
+    // phase B: the logged tiles (CTA tiles; every class on a small level), Resident Tile Stealing
+    bool logged = ldcg(&cur->cnt[0].v) > 0;
+    if (log_all)
+      for (int c = 1; c <= a.L.ncls; ++c) logged |= ldcg(&cur->cnt[c].v) > 0;
+    if constexpr (HT > 0) {   // the CTA's copy of the table with the hubs phase A inserted
+      if (ldcg(&cur->hubc.v) >= kHubReloadMinChanges) {
+        hub_load<HT>(a, ht);
+        __syncthreads();
       }
+    }
+    if (logged) {
       consume_log<VEC>(f, a.L, a.q[L & 1], cur, a.off, a.col, a.w, &wsm[warp], fsrc[warp], a.vec_ok,
                        a.steal != 0);
       grid_barrier(&ctl->bar);

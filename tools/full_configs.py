@@ -24,7 +24,8 @@ def run(cfg):
     res = {"config": cfg, "graph": g.name, "n": g.n, "arcs": g.m, "gen_s": round(time.time() - t0, 1),
            "max_out_degree": int(np.diff(g.off).max())}
     srcs = [int(s) for s in sg.sources(g, 4, seed=2)]
-    stream = torch.cuda.current_stream()
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
     off_d, col_d = torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda()
     G = sage.load_csr(off_d, col_d, borrow=True, stream=stream.cuda_stream)
     lv = torch.empty(g.n, dtype=torch.int32, device="cuda")
@@ -51,7 +52,17 @@ def run(cfg):
             _, st = G.pagerank(0.85, 20, out=x)
             pr.append(st["ms"])
         res["pagerank_20_ms"] = pr
+        res["pagerank_form"] = "push, propagation blocking (automatic: y > 64 MB)"
+        res["pagerank_ms_per_iteration"] = min(pr) / 20
         res["pagerank_GBps_model"] = 20 * (40.0 * g.n + 12.0 * g.m) / (min(pr) * 1e-3) / 1e9
+        # the unblocked push form (round 1's) on the same graph, for the A/B
+        G2 = sage.load_csr(off_d, col_d, borrow=True, stream=stream.cuda_stream, pr_blocked=-1)
+        x2 = torch.empty(g.n, dtype=torch.float64, device="cuda")
+        G2.pagerank(0.85, 2, out=x2)
+        _, st2 = G2.pagerank(0.85, 20, out=x2)
+        res["pagerank_unblocked_ms_per_iteration"] = st2["ms"] / 20
+        G2.free()
+        del x2
         t1 = time.time()
         xr = oracle.pagerank(g.off, g.col, 0.85, 20)
         res["pagerank_oracle_s"] = round(time.time() - t1, 1)

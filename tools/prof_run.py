@@ -14,10 +14,11 @@ p = argparse.ArgumentParser()
 p.add_argument("--scale", type=int, default=24)
 p.add_argument("--graph", default="rmat", choices=["rmat", "uk", "twitter"])
 p.add_argument("--n", type=int, default=0, help="vertices for uk / twitter shapes")
-p.add_argument("--op", default="bfs_push", choices=["bfs_push", "bfs_do", "sssp", "pr", "reorder", "bc"])
+p.add_argument("--op", default="bfs_push", choices=["bfs_push", "bfs_do", "sssp", "pr", "pr_push", "reorder", "bc"])
 p.add_argument("--reps", type=int, default=3)
 p.add_argument("--tile-cta", type=int, default=256)
 p.add_argument("--align", type=int, default=4)
+p.add_argument("--pr-blocked", type=int, default=0)
 a = p.parse_args()
 if a.graph == "rmat":
     g = sg.rmat(a.scale, 16, 1, True)
@@ -29,7 +30,8 @@ w = sg.weights(g, 1)
 s = stream = torch.cuda.Stream()   # the library's work and the events on one stream
 torch.cuda.set_stream(stream)
 G = sage.load_csr(torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda(), torch.from_numpy(w).cuda(),
-                  symmetric=g.symmetric, borrow=True, stream=stream.cuda_stream, tile_cta=a.tile_cta, align=a.align)
+                  symmetric=g.symmetric, borrow=True, stream=stream.cuda_stream, tile_cta=a.tile_cta, align=a.align,
+                  pr_blocked=a.pr_blocked)
 src = sg.sources(g, a.reps, seed=2)
 lv = torch.empty(g.n, dtype=torch.int32, device="cuda")
 for i in range(a.reps):
@@ -45,14 +47,14 @@ for i in range(a.reps):
         _, st = G.bc([int(src[i])])
     else:
         x = torch.empty(g.n, dtype=torch.float64, device="cuda")
-        _, st = G.pagerank(0.85, 5, out=x)
+        _, st = G.pagerank(0.85, 5, out=x, push_only=(a.op == "pr_push"))
     print(a.op, i, {k: st[k] for k in ("levels", "kernel_ms", "ms", "edges_traversed", "model_bytes")}, flush=True)
-    if a.op not in ("pr", "reorder", "bc") and os.environ.get("LEVELS", "1") == "0":
+    if a.op not in ("pr", "pr_push", "reorder", "bc") and os.environ.get("LEVELS", "1") == "0":
         rec = G.level_records()
         dt = np.diff(np.concatenate([[0], rec[:, 6]])) / 1e3
         small = dt[rec[:, 2] < 10000]
         print("   levels=%d  median small-level us=%.1f  total small-level ms=%.2f" % (len(rec), np.median(small) if len(small) else 0, small.sum() / 1e3))
-    if a.op not in ("pr", "reorder", "bc") and os.environ.get("LEVELS", "1") == "1":
+    if a.op not in ("pr", "pr_push", "reorder", "bc") and os.environ.get("LEVELS", "1") == "1":
         prev = 0
         for r in G.level_records():
             print("   L dir=%d |F|=%9d arcsF=%11d insp=%11d disc=%9d  %8.1f us (work done at +%8.1f, phase1 +%8.1f)" % (

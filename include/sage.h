@@ -94,10 +94,6 @@ typedef struct {
   int32_t hub_filter;  /* push BFS hub filter (a shared-memory table of visited
                         high-degree vertices skips their status reads; results identical):
                         0 = automatic (graphs with >= 32M arcs), 1 = always, -1 = never        */
-  int32_t pr_blocked;  /* push PageRank with propagation blocking (contributions to
-                        other blocks of y staged per target block, applied while the block is
-                        L2-resident; same arithmetic): 0 = automatic (y > 64 MB), 1 = always,
-                        -1 = never                                                                */
 } sage_options;
 
 /* CSR input of sage_load_csr (Fig. 1: u_offset / v arrays).                         */

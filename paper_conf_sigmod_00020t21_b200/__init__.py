@@ -39,7 +39,7 @@ class SageError(RuntimeError):
 class Options(ctypes.Structure):
     _fields_ = [("tile_cta", ctypes.c_int32), ("tile_min", ctypes.c_int32), ("align", ctypes.c_int32),
                 ("alpha", ctypes.c_double), ("beta", ctypes.c_double), ("ctas_per_sm", ctypes.c_int32),
-                ("hub_filter", ctypes.c_int32), ("pr_blocked", ctypes.c_int32)]
+                ("hub_filter", ctypes.c_int32)]
 
 
 class Dist(ctypes.Structure):
@@ -322,7 +322,7 @@ def debug_loopback_id(world: int) -> bytes:
 def load_csr(off, col, w=None, n: int | None = None, symmetric: bool = False, push_only: bool = False,
              borrow: bool = False, validate: bool = True, tile_cta: int = 256, tile_min: int = 8,
              align: int = 4, alpha: float = 15.0, beta: float = 18.0, stream=None, ctas_per_sm: int = 0,
-             hub_filter: int = 0, pr_blocked: int = 0,
+             hub_filter: int = 0,
              rank: int = 0, world: int = 1, nccl_unique_id: bytes | None = None,
              v_begin: int = 0, v_end: int | None = None, host_columns: bool = False) -> Graph:
     """sage_load_csr.  ``off``/``col``/``w`` are host arrays or tensors, or CUDA tensors."""
@@ -353,7 +353,7 @@ def load_csr(off, col, w=None, n: int | None = None, symmetric: bool = False, pu
         import torch
         stream = torch.cuda.current_stream().cuda_stream
     csr.cuda_stream = stream
-    opts = Options(tile_cta, tile_min, align, alpha, beta, ctas_per_sm, hub_filter, pr_blocked)
+    opts = Options(tile_cta, tile_min, align, alpha, beta, ctas_per_sm, hub_filter)
     csr.opts = ctypes.pointer(opts)
     dist = None
     if nccl_unique_id is not None:

@@ -79,7 +79,7 @@ struct BcFwd {
           l = next_level;
         }
       }
-      if (l == next_level) atomicAdd(sigma + v[j], s.su);     // Alg. 1 l.13-15
+      if (l == next_level) red_add_f64(sigma + v[j], s.su);   // Alg. 1 l.13-15
     }
   }
 };
@@ -109,7 +109,7 @@ struct BcBwd {
         acc += (1.0 + ldcg(delta + v[j])) / ldcg(sigma + v[j]);   // Alg. 1 l.21-23
     }
     for (int o = lpt >> 1; o > 0; o >>= 1) acc += __shfl_xor_sync(FULL, acc, o);
-    if (valid && (lane_id() & (lpt - 1)) == 0 && acc != 0.0) atomicAdd(delta + s.u, ldcg(sigma + s.u) * acc);
+    if (valid && (lane_id() & (lpt - 1)) == 0 && acc != 0.0) red_add_f64(delta + s.u, ldcg(sigma + s.u) * acc);
   }
 };
 

@@ -166,7 +166,7 @@ static int ilog2(long long x) {
 static bool is_pow2(long long x) { return x > 0 && (x & (x - 1)) == 0; }
 
 static sage_status make_ladder(const sage_options *o, sage_graph *g) {
-  int B = 256, M = 8, A = 4, cps = 0, hub = 0, prb = 0;
+  int B = 256, M = 8, A = 4, cps = 0, hub = 0;
   double alpha = 15.0, beta = 18.0;
   if (o) {
     B = o->tile_cta;
@@ -176,11 +176,6 @@ static sage_status make_ladder(const sage_options *o, sage_graph *g) {
     beta = o->beta;
     cps = o->ctas_per_sm;
     hub = o->hub_filter;
-    prb = o->pr_blocked;
-  }
-  if (prb < -1 || prb > 1) {
-    set_error("pr_blocked must be -1, 0 or 1");
-    return SAGE_E_INVALID;
   }
   if (hub < -1 || hub > 1) {
     set_error("hub_filter must be -1, 0 or 1");
@@ -215,7 +210,6 @@ static sage_status make_ladder(const sage_options *o, sage_graph *g) {
   g->beta = beta;
   g->ctas_per_sm = cps;
   g->hub_filter = hub;
-  g->pr_blocked = prb;
   return SAGE_OK;
 }
 

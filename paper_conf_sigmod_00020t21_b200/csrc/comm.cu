@@ -542,7 +542,7 @@ struct PrPushMulti {
       in[j] = false;
       if (!valid) continue;
       bool own;
-      atomicAdd(y + pidx(*pm, v[j], &own), s.c);
+      red_add_f64(y + pidx(*pm, v[j], &own), s.c);
     }
   }
 };

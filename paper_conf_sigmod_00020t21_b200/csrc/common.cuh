@@ -205,6 +205,11 @@ __device__ __forceinline__ uint32_t atom_or_if(bool pred, uint32_t *p, uint32_t 
                : "+r"(r) : "l"(p), "r"(bits), "r"((uint32_t)pred));
   return r;
 }
+// fp64 add without a return value.  atomicAdd(double *) whose result is unused can still come out
+// as a returning ATOMG (it did in the PageRank push filter); red.global.add.f64 is the REDG form.
+__device__ __forceinline__ void red_add_f64(double *p, double v) {
+  asm volatile("red.global.add.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
+}
 template <class T> __device__ __forceinline__ T ldcg(const T *p) { return __ldcg(p); }
 __device__ __forceinline__ CtaTile ldcg_tile(const CtaTile *p) {
   longlong2 v = __ldcg(reinterpret_cast<const longlong2 *>(p));
@@ -811,6 +816,19 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
       }
       if (base >= count) break;
       const unsigned long long end = (base + batch < count) ? base + batch : count;
+      // log entries of the batch's next 32-tile group, loaded while the current group's steps run
+      // (the metadata chain of a group is then offsets -> start only)
+      int pf_u = 0;
+      long long pf_start = 0;
+      if ((unsigned long long)lane < end - base) {
+        if (c == 0) {
+          const CtaTile T = ldcg_tile(Q.cta + base + lane);
+          pf_u = T.u;
+          pf_start = T.start;
+        } else {
+          pf_u = ldcg(Q.cls[c] + base + lane);
+        }
+      }
       for (unsigned long long r0 = base; r0 < end; r0 += 32) {
         // ---- metadata round: lane k resolves tile r0 + k (log entry -> row -> tile start and
         //      the filter's per-source context) in ONE round of loads for up to 32 tiles; the
@@ -821,21 +839,28 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
           long long start = 0, rb = 0, re = 0;
           int u = 0;
           if (mv) {
-            const unsigned long long ti = r0 + lane;
+            u = pf_u;
             if (c == 0) {
-              CtaTile T = ldcg_tile(Q.cta + ti);
-              start = T.start;
-              u = T.u;
+              start = pf_start;
               if (F::kNeedRow) {
                 rb = ld_off(off + u);
                 re = ld_off(off + u + 1);
               }
             } else {
-              u = ldcg(Q.cls[c] + ti);
               rb = ld_off(off + u);
               re = ld_off(off + u + 1);
               RowSplit s = split_row(rb, re, L);
               start = class_tile_start(re, s.r, t);
+            }
+          }
+          const unsigned long long r1 = r0 + 32;
+          if (r1 + lane < end) {
+            if (c == 0) {
+              const CtaTile T = ldcg_tile(Q.cta + r1 + lane);
+              pf_u = T.u;
+              pf_start = T.start;
+            } else {
+              pf_u = ldcg(Q.cls[c] + r1 + lane);
             }
           }
           const typename F::Src sc = f.src(mv, u, rb, re);
@@ -931,9 +956,14 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
           PROF_ADD(2, tv1 - tv0);
           PROF_ADD(4, 1);
           if constexpr (F::kEnqueue) {
+            bool anyin = false;
 #pragma unroll
-            for (int j = 0; j < VEC; ++j)
-              push_filtered(f, in[j], v[j], ws, bcnt, off, L);
+            for (int j = 0; j < VEC; ++j) anyin |= in[j];
+            if (__any_sync(FULL, anyin)) {   // most steps of a heavy level find nothing new
+#pragma unroll
+              for (int j = 0; j < VEC; ++j)
+                push_filtered(f, in[j], v[j], ws, bcnt, off, L);
+            }
           }
         }
         __syncwarp();

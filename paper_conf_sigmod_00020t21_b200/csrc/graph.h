@@ -48,13 +48,6 @@ struct PageRankState {      // the all-V resident tile log (built once, reused; 
   long long n_dangling = 0;
   double *x = nullptr, *y = nullptr;
   void *c = nullptr;              // pull form: x_u / out(u) (fp32, or fp64 when damping > 0.9)
-  // blocked push form (pagerank.cu, PrPushBlocked); bin_lg == 0 = not set up
-  int bin_lg = 0, nbin = 0;
-  long long bin_warps = 0;
-  long long *bstart = nullptr;
-  unsigned long long *bfill = nullptr;
-  int *ev = nullptr;
-  double *ec = nullptr;
   size_t c_bytes = 0;
   CounterSet *cs = nullptr;       // device copy of the log's counters (+ rotating tickets)
 };
@@ -86,7 +79,6 @@ struct sage_graph {
   double alpha = 15.0, beta = 18.0;
   int ctas_per_sm = 0;        // sage_options.ctas_per_sm (0 = automatic)
   int hub_filter = 0;         // sage_options.hub_filter (0 auto, 1 on, -1 off)
-  int pr_blocked = 0;         // sage_options.pr_blocked (0 auto, 1 on, -1 off)
   int vec = 4;                // neighbours per lane per step (4; 1 when tile_min < 4)
   bool vec_ok = true;         // sub-warp tiles use 16-B loads (align % 4 == 0, aligned arrays)
   // reordering: sigma[v_orig] = current label; sigma_inv[label] = v_orig (null = identity)
@@ -103,5 +95,5 @@ struct sage_graph {
   long long online_thr = 0, online_pending = 0, online_rounds = 0, online_movers = 0, online_swaps = 0;
   uint32_t *samp_w = nullptr;
   unsigned long long *samp_acc = nullptr;
-  int grid_bfs = 0, grid_bfs_hub = 0, grid_bfs_fused = 0, grid_bfs_fused_hub = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0, grid_pr_pull64 = 0, grid_pr_blk = 0;   // persistent grid sizes
+  int grid_bfs = 0, grid_bfs_hub = 0, grid_bfs_fused = 0, grid_bfs_fused_hub = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0, grid_pr_pull64 = 0;   // persistent grid sizes
 };

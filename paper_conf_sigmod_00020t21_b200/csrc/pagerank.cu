@@ -44,7 +44,7 @@ struct PrPush {
     for (int j = 0; j < N; ++j) in[j] = false;
     if (!valid) return;
 #pragma unroll
-    for (int j = 0; j < N; ++j) atomicAdd(y + v[j], s.c);
+    for (int j = 0; j < N; ++j) red_add_f64(y + v[j], s.c);
   }
 };
 
@@ -79,21 +79,10 @@ struct PrPull {
 #pragma unroll
     for (int j = 0; j < N; ++j) acc += (double)cv[j];
     for (int o = lpt >> 1; o > 0; o >>= 1) acc += __shfl_xor_sync(FULL, acc, o);
-    if (valid && (lane_id() & (lpt - 1)) == 0 && acc != 0.0) atomicAdd(y + s.u, acc);
+    if (valid && (lane_id() & (lpt - 1)) == 0 && acc != 0.0) red_add_f64(y + s.u, acc);
   }
 };
 
-constexpr int kPrChunk = 32;      // entries a warp reserves per bin at a time (one 128-B line of ev)
-constexpr int kPrMaxBins = 16;
-
-// Blocked push form (propagation blocking; B200 addition; the arithmetic is Alg. 1
-// l.26-29's): when y does not fit L2, a push arc u->v whose target lies in another 2^bin_lg-vertex
-// block than u costs a DRAM read-modify-write of a y sector.  Its contribution (v, c_u) is
-// appended to the bin of v's block instead (4 + 8 B written, the same read back later) and the
-// bins are applied block after block while that block of y is L2-resident; arcs inside the
-// source's block (most of a crawl-ordered web graph) are added directly.  Each warp appends
-// through its own open 32-entry chunk per bin (chunk state in shared memory); with <= 16 bins the
-// open chunks of the whole grid fit L2, so every line of the bins is written back whole.
 struct PrArgs {
   const long long *off;
   const int *col;
@@ -108,23 +97,16 @@ struct PrArgs {
   long long n_dangling;
   double *x, *y;
   void *c;            // pull form: x_u / out(u), fp32 or fp64 (see PrPull)
-  // blocked push (PrPushBlocked): far contributions staged per target block of y
-  int bin_lg;                     // target block = v >> bin_lg (2^bin_lg vertices of y per block)
-  int nbin;
-  const long long *bstart;        // bin b's entries live at [bstart[b], bstart[b] + capacity)
-  unsigned long long *bfill;      // reserved entries per bin (multiples of kPrChunk)
-  int *ev;                        // entry target (-1 = padding)
-  double *ec;                     // entry contribution
   Ctl *ctl;
   int vec_ok;
 };
 
 // Build the all-V resident log: one thread per vertex, warp-aggregated classification.
-__global__ void k_build_log(const long long *__restrict__ off, long long n, Ladder L, Queues Q,
+__global__ void k_build_log(const long long *__restrict__ off, long long v0, long long n, Ladder L, Queues Q,
                             CounterSet *cs, int *dangling, unsigned long long *n_dangling) {
   const long long stride = (long long)gridDim.x * blockDim.x;
-  const long long nthr = ((n + 31) / 32) * 32;
-  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nthr; i += stride) {
+  const long long nthr = v0 + ((n - v0 + 31) / 32) * 32;
+  for (long long i = v0 + (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nthr; i += stride) {
     const bool in = i < n;
     long long b = 0, e = 0;
     if (in) {
@@ -145,26 +127,6 @@ __global__ void k_build_log(const long long *__restrict__ off, long long n, Ladd
   }
 }
 
-// Arcs whose target block differs from the source's, per target block (blocked push capacities;
-// one pass over col per resident log).
-__global__ void k_far_count(const long long *__restrict__ off, const int *__restrict__ col, long long n,
-                            int lg, int nbin, unsigned long long *cnt) {
-  __shared__ unsigned long long hc[kPrMaxBins];
-  for (int i = threadIdx.x; i < nbin; i += blockDim.x) hc[i] = 0ull;
-  __syncthreads();
-  const long long stride = (long long)gridDim.x * (blockDim.x / 32);
-  for (long long u = (long long)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); u < n; u += stride) {
-    const int ub = (int)(u >> lg);
-    for (long long k = off[u] + lane_id(); k < off[u + 1]; k += 32) {
-      const int vb = col[k] >> lg;
-      if (vb != ub) atomicAdd(&hc[vb], 1ull);
-    }
-  }
-  __syncthreads();
-  for (int i = threadIdx.x; i < nbin; i += blockDim.x)
-    if (hc[i]) atomicAdd(cnt + i, hc[i]);
-}
-
 __global__ void k_pr_init(double *x, double *y, long long n, double v0) {
   const long long stride = (long long)gridDim.x * blockDim.x;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
@@ -173,73 +135,7 @@ __global__ void k_pr_init(double *x, double *y, long long n, double v0) {
   }
 }
 
-struct PrPushBlocked {
-  struct Src {
-    double c;
-    int ublk;
-  };
-  static constexpr int kPrefetch = SAGE_PR_PREFETCH;
-  static constexpr bool kWeights = false;
-  static constexpr bool kNeedRow = true;
-  static constexpr bool kEnqueue = false;
-  const Queues *next_q = nullptr;
-  CounterSet *next_cs = nullptr;
-  const double *x;
-  double *y;
-  int bin_lg;
-  const long long *bstart;
-  unsigned long long *bfill;
-  int *ev;
-  double *ec;
-  unsigned *wpos, *wend;          // this warp's open chunk per bin (shared memory)
-
-  __device__ __forceinline__ Src src(bool valid, int u, long long b, long long e) const {
-    return Src{(valid && e > b) ? ldcg(x + u) / (double)(e - b) : 0.0, u >> bin_lg};
-  }
-  // warp-collective: lanes with `far` append (v, c) to bin v >> bin_lg (consecutive slots per bin)
-  __device__ __forceinline__ void append(bool far, int v, double c) const {
-    const unsigned fm = __ballot_sync(FULL, far);
-    if (!fm) return;
-    const unsigned lane = lane_id();
-    const int b = far ? (v >> bin_lg) : -1 - (int)lane;
-    const unsigned peers = __match_any_sync(FULL, b);
-    const int leader = __ffs(peers) - 1;
-    const int cnt = __popc(peers), rank = __popc(peers & lanemask_lt());
-    unsigned pos = 0, room = 0, nbase = 0;
-    if (far && (int)lane == leader) {
-      pos = wpos[b];
-      room = wend[b] - pos;
-      if (room >= (unsigned)cnt) {
-        wpos[b] = pos + cnt;
-      } else {   // open a new chunk; the first `room` entries still fill the old one
-        nbase = (unsigned)atomicAdd(bfill + b, (unsigned long long)kPrChunk);
-        wpos[b] = nbase + (cnt - room);
-        wend[b] = nbase + kPrChunk;
-      }
-    }
-    pos = __shfl_sync(FULL, pos, leader);
-    room = __shfl_sync(FULL, room, leader);
-    nbase = __shfl_sync(FULL, nbase, leader);
-    if (far) {
-      const long long i = bstart[b] + (long long)((unsigned)rank < room ? pos + rank : nbase + (rank - room));
-      ev[i] = v;
-      ec[i] = c;
-    }
-  }
-  template <int N>
-  __device__ __forceinline__ void visit(bool valid, const Src &s, int (&v)[N],
-                                        const uint32_t (&)[N], bool (&in)[N], int) const {
-#pragma unroll
-    for (int j = 0; j < N; ++j) {
-      in[j] = false;
-      const bool far = valid && (v[j] >> bin_lg) != s.ublk;
-      if (valid && !far) atomicAdd(y + v[j], s.c);
-      append(far, v[j], s.c);
-    }
-  }
-};
-
-template <int VEC, bool BLK>
+template <int VEC>
 __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ PrArgs a) {
   __shared__ WarpScratch wsm[kWarps];
   __shared__ PrPush::Src fsrc[kWarps][32];
@@ -255,42 +151,10 @@ __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ 
     if (blockIdx.x == 0 && threadIdx.x < kQueues) a.sets[(it + 2) % 3].tk[threadIdx.x].v = 0ull;
     if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->D[(it + 2) % 3] = 0.0;
     // push phase over the resident log
-    if constexpr (BLK) {
-      __shared__ unsigned wpos[kWarps][kPrMaxBins], wend[kWarps][kPrMaxBins];
-      __shared__ PrPushBlocked::Src fsrcb[kWarps][32];
-      if (lane < (unsigned)kPrMaxBins) wpos[warp][lane] = wend[warp][lane] = 0u;
-      __syncwarp();
-      PrPushBlocked f;
-      f.x = a.x;
-      f.y = a.y;
-      f.bin_lg = a.bin_lg;
-      f.bstart = a.bstart;
-      f.bfill = a.bfill;
-      f.ev = a.ev;
-      f.ec = a.ec;
-      f.wpos = wpos[warp];
-      f.wend = wend[warp];
-      consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &wsm[warp], fsrcb[warp], a.vec_ok);
-      __syncwarp();
-      for (int b = 0; b < a.nbin; ++b) {   // pad this warp's open chunks (-1 = no entry)
-        const unsigned p0 = wpos[warp][b], p1 = wend[warp][b];
-        for (unsigned i = p0 + lane; i < p1; i += 32) a.ev[a.bstart[b] + i] = -1;
-      }
-      grid_barrier(&a.ctl->bar);
-      // apply the bins block by block (every warp on the same bin: its block of y stays in L2)
-      for (int b = 0; b < a.nbin; ++b) {
-        const long long s0 = a.bstart[b], cnt = (long long)ldcg(a.bfill + b);
-        for (long long i = tid; i < cnt; i += stride) {
-          const int v = __ldcs(a.ev + s0 + i);
-          if (v >= 0) atomicAdd(a.y + v, __ldcs(a.ec + s0 + i));
-        }
-      }
-    } else {
-      PrPush f;
-      f.x = a.x;
-      f.y = a.y;
-      consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &wsm[warp], fsrc[warp], a.vec_ok);
-    }
+    PrPush f;
+    f.x = a.x;
+    f.y = a.y;
+    consume_log<VEC>(f, a.L, a.q, cs, a.off, a.col, nullptr, &wsm[warp], fsrc[warp], a.vec_ok);
     // dangling mass of this iteration's x
     double dsum = 0.0;
     for (long long i = tid; i < a.n_dangling; i += stride) dsum += ldcg(a.x + a.dangling[i]);
@@ -311,7 +175,6 @@ __global__ void __launch_bounds__(kBlock, 4) k_pagerank(const __grid_constant__ 
       a.x[v] = add + a.d * yv;
       a.y[v] = 0.0;
     }
-    if (tid < a.nbin) a.bfill[tid] = 0ull;   // every bin was applied before the barrier above
     grid_barrier(&a.ctl->bar);
   }
 }
@@ -368,23 +231,8 @@ __global__ void k_pr_init_c(const long long *__restrict__ off, CT *c, long long 
   }
 }
 
-void free_pr_blocks(sage_graph *g) {
-  PageRankState &p = g->pr;
-  dfree(g, p.bstart);
-  dfree(g, p.bfill);
-  dfree(g, p.ev);
-  dfree(g, p.ec);
-  p.bstart = nullptr;
-  p.bfill = nullptr;
-  p.ev = nullptr;
-  p.ec = nullptr;
-  p.bin_lg = p.nbin = 0;
-  p.bin_warps = 0;
-}
-
 void free_pagerank_state(sage_graph *g) {
   PageRankState &p = g->pr;
-  free_pr_blocks(g);
   free_queues(g, &p.q);
   dfree(g, p.dangling);
   dfree(g, p.x);
@@ -407,7 +255,6 @@ sage_status ensure_pagerank_log(sage_graph *g) {
       return s;
     }
   }
-  free_pr_blocks(g);   // capacities follow the labels (rebuilt after sage_reorder)
   if ((s = alloc_queues(g, &p.q, n, g->m)) != SAGE_OK ||
       (s = dalloc(g, (void **)&p.dangling, sizeof(int) * (size_t)(n + 1))) != SAGE_OK) {
     free_pagerank_state(g);
@@ -415,7 +262,7 @@ sage_status ensure_pagerank_log(sage_graph *g) {
   }
   unsigned long long *nd = reinterpret_cast<unsigned long long *>(p.cs + 3);
   cudaMemsetAsync(p.cs, 0, sizeof(CounterSet) * 3 + 64, g->stream);
-  k_build_log<<<g->num_sms * 8, 256, 0, g->stream>>>((const long long *)g->off, n, g->ladder,
+  k_build_log<<<g->num_sms * 8, 256, 0, g->stream>>>((const long long *)g->off, 0, n, g->ladder,
                                                      p.q, p.cs, p.dangling, nd);
   // replicate the counts into the two other rotating sets
   cudaMemcpyAsync(p.cs + 1, p.cs, sizeof(CounterSet), cudaMemcpyDeviceToDevice, g->stream);
@@ -429,50 +276,6 @@ sage_status ensure_pagerank_log(sage_graph *g) {
   for (int i = 0; i < kQueues; ++i) p.cnt[i] = h.cnt[i].v;
   p.n_dangling = (long long)hnd;
   p.valid = true;
-  return SAGE_OK;
-}
-
-// Blocked-push state (PrPushBlocked): used when y (8 B per vertex) would not stay L2-resident;
-// 2^bin_lg-vertex target blocks, 8-16 of them; per-bin capacities from the static far-arc counts.
-constexpr size_t kPrBlockedMinY = 64ull << 20;
-static sage_status ensure_pr_blocks(sage_graph *g, long long nwarps) {
-  PageRankState &p = g->pr;
-  if (p.bin_lg && p.bin_warps == nwarps) return SAGE_OK;
-  free_pr_blocks(g);
-  const long long n = g->n_local;
-  int lg = 10;   // the smallest blocks that keep the bins at <= kPrMaxBins
-  while ((((n - 1) >> lg) + 1) > kPrMaxBins) ++lg;
-  const int nbin = (int)(((n > 0 ? n - 1 : 0) >> lg) + 1);
-  sage_status s;
-  unsigned long long *cnt = nullptr;
-  if ((s = dalloc(g, (void **)&cnt, sizeof(unsigned long long) * (size_t)nbin)) != SAGE_OK) return s;
-  cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * (size_t)nbin, g->stream);
-  k_far_count<<<g->num_sms * 4, 256, 0, g->stream>>>((const long long *)g->off, g->col, n, lg, nbin, cnt);
-  std::vector<unsigned long long> h((size_t)nbin);
-  cudaMemcpyAsync(h.data(), cnt, sizeof(unsigned long long) * (size_t)nbin, cudaMemcpyDeviceToHost, g->stream);
-  cudaError_t e = cudaStreamSynchronize(g->stream);
-  dfree(g, cnt);
-  if (e != cudaSuccess) return cuda_fail(g, e, "PageRank blocks");
-  std::vector<long long> bs((size_t)nbin);
-  long long tot = 0;
-  for (int b = 0; b < nbin; ++b) {
-    bs[(size_t)b] = tot;
-    tot += (long long)h[(size_t)b] + (nwarps + 1) * kPrChunk;   // + one partial chunk per warp
-  }
-  if ((s = dalloc(g, (void **)&p.bstart, sizeof(long long) * (size_t)nbin)) != SAGE_OK ||
-      (s = dalloc(g, (void **)&p.bfill, sizeof(unsigned long long) * (size_t)nbin)) != SAGE_OK ||
-      (s = dalloc(g, (void **)&p.ev, sizeof(int) * (size_t)tot)) != SAGE_OK ||
-      (s = dalloc(g, (void **)&p.ec, sizeof(double) * (size_t)tot)) != SAGE_OK) {
-    free_pr_blocks(g);
-    return s;
-  }
-  cudaMemcpyAsync(p.bstart, bs.data(), sizeof(long long) * (size_t)nbin, cudaMemcpyHostToDevice, g->stream);
-  cudaMemsetAsync(p.bfill, 0, sizeof(unsigned long long) * (size_t)nbin, g->stream);
-  e = cudaStreamSynchronize(g->stream);
-  if (e != cudaSuccess) return cuda_fail(g, e, "PageRank blocks");
-  p.bin_lg = lg;
-  p.nbin = nbin;
-  p.bin_warps = nwarps;
   return SAGE_OK;
 }
 
@@ -553,28 +356,9 @@ extern "C" sage_status sage_pagerank_ex(sage_graph *g, double damping, int32_t i
   if (iterations > 0) {
     const void *fn = pull ? (c64 ? (g->vec == 4 ? (const void *)k_pagerank_pull<4, double> : (const void *)k_pagerank_pull<1, double>)
                                  : (g->vec == 4 ? (const void *)k_pagerank_pull<4, float> : (const void *)k_pagerank_pull<1, float>))
-                          : (g->vec == 4 ? (const void *)k_pagerank<4, false> : (const void *)k_pagerank<1, false>);
+                          : (g->vec == 4 ? (const void *)k_pagerank<4> : (const void *)k_pagerank<1>);
     int *cache = pull ? (c64 ? &g->grid_pr_pull64 : &g->grid_pr_pull) : &g->grid_pr;
-#ifndef SAGE_PR_NO_BLOCKED
-    const bool blocked = !pull && g->pr_blocked >= 0 &&
-                         (g->pr_blocked > 0 || (size_t)g->n_local * sizeof(double) > kPrBlockedMinY);
-#else
-    const bool blocked = false;
-#endif
-    if (blocked) {
-      fn = g->vec == 4 ? (const void *)k_pagerank<4, true> : (const void *)k_pagerank<1, true>;
-      cache = &g->grid_pr_blk;
-    }
     const int grid = coop_grid(g, fn, cache);
-    if (blocked) {
-      if ((s = ensure_pr_blocks(g, (long long)grid * (kBlock / 32))) != SAGE_OK) return s;
-      a.bin_lg = p.bin_lg;
-      a.nbin = p.nbin;
-      a.bstart = p.bstart;
-      a.bfill = p.bfill;
-      a.ev = p.ev;
-      a.ec = p.ec;
-    }
     void *args[] = {&a};
     if ((s = launch_coop(g, fn, grid, args, "PageRank kernel")) != SAGE_OK) return s;
   }

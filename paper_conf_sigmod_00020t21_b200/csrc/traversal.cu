@@ -76,6 +76,7 @@ struct BfsPushT {
   const Queues *next_q;
   CounterSet *next_cs;
   uint32_t ht = 0;     // shared-memory address of the hub table (HT > 0)
+  unsigned long long keep = 0;   // L2 evict_last policy of the status loads (made once per level)
   unsigned long long *nfc = nullptr;   // fused tiling: |F| of the next list, counted at discovery
 
   __device__ __forceinline__ Src src(bool, int u, long long, long long) const { return Src{u}; }
@@ -96,10 +97,17 @@ struct BfsPushT {
       }
     }
     uint32_t wd[N];
-    const unsigned long long keep = policy_evict_last();
 #pragma unroll
     for (int j = 0; j < N; ++j)
       wd[j] = (valid && !hit[j]) ? ld_status(visited + (v[j] >> 5), keep) : 0xffffffffu;
+    bool need = false;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      in[j] = false;
+      need |= !((wd[j] >> (v[j] & 31)) & 1u);
+    }
+    // on the heavy levels almost every target is already visited: one vote skips the claims
+    if (!__any_sync(FULL, need)) return;
     // claims of all N neighbours in flight together (predicated, no branch between them)
     uint32_t old[N];
 #pragma unroll
@@ -114,6 +122,52 @@ struct BfsPushT {
       if (in[j]) {
         level[v[j]] = next_level;
         if (parent) parent[v[j]] = s.u + v_base;
+        if (fb_next) atomicOr(fb_next + (v[j] >> 5), bit);
+      }
+    }
+  }
+  // the same filter for N independent elements per lane, each with its own source and validity
+  // (the fused fragment gather: lane k takes elements k, k + 32, ... of the chunk's fragments)
+  template <int N>
+  __device__ __forceinline__ void visit_each(const bool (&valid)[N], const int (&u)[N], const int (&v)[N],
+                                             bool (&in)[N]) const {
+    bool hit[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      hit[j] = false;
+      if constexpr (HT > 0) {
+        constexpr int lg = HubGeom<HT>::lgT;
+        const uint32_t slot = (uint32_t)v[j] & ((1u << lg) - 1u), k1 = ((uint32_t)v[j] >> lg) + 1u;
+        if (valid[j]) {
+          if constexpr (HubGeom<HT>::kbits == 8) hit[j] = ld_shared_u8(ht + slot) == k1;
+          else hit[j] = ld_shared_u16(ht + 2u * slot) == k1;
+        }
+      }
+    }
+    uint32_t wd[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j)
+      wd[j] = (valid[j] && !hit[j]) ? ld_status(visited + (v[j] >> 5), keep) : 0xffffffffu;
+    bool need = false;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      in[j] = false;
+      need |= !((wd[j] >> (v[j] & 31)) & 1u);
+    }
+    if (!__any_sync(FULL, need)) return;
+    uint32_t old[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const uint32_t bit = 1u << (v[j] & 31);
+      old[j] = atom_or_if(!(wd[j] & bit), visited + (v[j] >> 5), bit, bit);
+    }
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      const uint32_t bit = 1u << (v[j] & 31);
+      in[j] = !(old[j] & bit);
+      if (in[j]) {
+        level[v[j]] = next_level;
+        if (parent) parent[v[j]] = u[j] + v_base;
         if (fb_next) atomicOr(fb_next + (v[j] >> 5), bit);
       }
     }
@@ -589,6 +643,7 @@ __device__ __forceinline__ void bfs_body(const TravArgs &a, WarpScratch *wsm, ty
         }
       }
       BfsPushT<HT> f;
+      f.keep = policy_evict_last();
       f.visited = a.visited;
       f.level = a.level;
       f.parent = a.parent;
@@ -900,8 +955,13 @@ __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, Cou
         const typename F::Src sc = fsrc[valid ? k : 0];
         bool in[VEC];
         f.template visit<VEC>(valid, sc, vv, ww, in, lpt);
+        bool anyin = false;
 #pragma unroll
-        for (int j = 0; j < VEC; ++j) push_filtered(f, in[j], vv[j], ws, bcnt, a.off, L);
+        for (int j = 0; j < VEC; ++j) anyin |= in[j];
+        if (__any_sync(FULL, anyin)) {
+#pragma unroll
+          for (int j = 0; j < VEC; ++j) push_filtered(f, in[j], vv[j], ws, bcnt, a.off, L);
+        }
       }
       __syncwarp();
     }
@@ -931,30 +991,42 @@ __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, Cou
         ws->tb[lane] = (int)(tb - b);
         fsrc[lane] = f.src(act, v, b, e);
         __syncwarp();
-        for (int k0 = 0; k0 < total; k0 += 32) {
-          const int k = k0 + (int)lane;
-          const bool kv = k < total;
-          int o = 0;
-          if (kv) {   // largest o with pre[o] <= k
-            int lo = 0, hi = 31;
+        // FE elements per lane per round (k0 + j * 32 + lane): FE status reads in flight per lane
+        constexpr int FE = 4;
+        for (int k0 = 0; k0 < total; k0 += 32 * FE) {
+          bool kv[FE];
+          int vv[FE], uu[FE];
 #pragma unroll
-            for (int it = 0; it < 5; ++it) {
-              const int mid = (lo + hi + 1) >> 1;
-              if (ws->pre[mid] <= k) lo = mid; else hi = mid - 1;
+          for (int j = 0; j < FE; ++j) {
+            const int k = k0 + j * 32 + (int)lane;
+            kv[j] = k < total;
+            int o = 0;
+            if (kv[j]) {   // largest o with pre[o] <= k
+              int lo = 0, hi = 31;
+#pragma unroll
+              for (int it = 0; it < 5; ++it) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (ws->pre[mid] <= k) lo = mid; else hi = mid - 1;
+              }
+              o = lo;
             }
-            o = lo;
+            vv[j] = 0;
+            uu[j] = fsrc[o].u;
+            if (kv[j]) {
+              const int idx = k - ws->pre[o];
+              const long long pos = ws->hb[o] + (idx < ws->hl[o] ? idx : ws->tb[o] + (idx - ws->hl[o]));
+              vv[j] = ld_col(a.col + pos, pol);
+            }
           }
-          int vv[1] = {0};
-          uint32_t w1[1] = {0u};
-          const typename F::Src so = fsrc[o];
-          if (kv) {
-            const int idx = k - ws->pre[o];
-            const long long pos = ws->hb[o] + (idx < ws->hl[o] ? idx : ws->tb[o] + (idx - ws->hl[o]));
-            vv[0] = ld_col(a.col + pos, pol);
+          bool in[FE];
+          f.template visit_each<FE>(kv, uu, vv, in);
+          bool anyin = false;
+#pragma unroll
+          for (int j = 0; j < FE; ++j) anyin |= in[j];
+          if (__any_sync(FULL, anyin)) {
+#pragma unroll
+            for (int j = 0; j < FE; ++j) push_filtered(f, in[j], vv[j], ws, bcnt, a.off, L);
           }
-          bool in[1];
-          f.template visit<1>(kv, so, vv, w1, in, 1);
-          push_filtered(f, in[0], vv[0], ws, bcnt, a.off, L);
         }
         __syncwarp();
       }
@@ -1053,6 +1125,7 @@ __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *w
     if (L > 0) zero_counterset(&ctl->set[(L + 2) % 3]);
     if (blockIdx.x == 0 && threadIdx.x == 0 && L + 1 < kMaxRec) ctl->rec[L + 1].t_work = ctl->rec[L + 1].t_mid = 0;
     BfsPushT<HT> f;
+    f.keep = policy_evict_last();
     f.visited = a.visited;
     f.level = a.level;
     f.parent = a.parent;
@@ -1495,8 +1568,10 @@ static int hub_mode(const sage_graph *g) {
   return 0;
 #else
   if (g->vec != 4 || g->hub_filter < 0 || (g->hub_filter == 0 && g->m < kHubMinGraphArcs)) return 0;
-  if (SAGE_HUB_KB == 128) return g->n <= 255ll << 17 ? 1 : 2;
-  return g->n <= 255ll << 16 ? 3 : 4;
+  // 8-bit keys hold (v >> lgT) + 1 <= 255, so ids >= 255 << lgT are never inserted (0.4% of the
+  // ids at n = 2^24, which keeps C2 on the 2^16-slot byte table)
+  if (SAGE_HUB_KB == 128) return g->n <= 256ll << 17 ? 1 : 2;
+  return g->n <= 256ll << 16 ? 3 : 4;
 #endif
 }
 static int hub_lgT(int ht) { return ht == 1 ? 17 : ht == 4 ? 15 : 16; }
@@ -1645,10 +1720,14 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   cudaEventRecord(e1, g->stream);
   if (fused) {
     const int ht = hub_mode(g);
-    const void *fn = ht == 1 ? (const void *)k_bfs_fused_hub<4, 1>
-                   : ht == 2 ? (const void *)k_bfs_fused_hub<4, 2>
-                   : ht == 3 ? (const void *)k_bfs_fused_hub<4, 3>
-                   : ht == 4 ? (const void *)k_bfs_fused_hub<4, 4>
+#ifndef SAGE_FUSED_VEC
+#define SAGE_FUSED_VEC 4   // neighbours per lane per step of the fused push BFS (A/B: 8)
+#endif
+    constexpr int FV = SAGE_FUSED_VEC;
+    const void *fn = ht == 1 ? (const void *)k_bfs_fused_hub<FV, 1>
+                   : ht == 2 ? (const void *)k_bfs_fused_hub<FV, 2>
+                   : ht == 3 ? (const void *)k_bfs_fused_hub<FV, 3>
+                   : ht == 4 ? (const void *)k_bfs_fused_hub<FV, 4>
                    : g->vec == 4 ? (const void *)k_bfs_fused<4> : (const void *)k_bfs_fused<1>;
     const int block = ht ? kHubBlock : kBlock;
     const size_t dyn = ht ? hub_bytes(ht) : 0;

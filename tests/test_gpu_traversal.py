@@ -404,24 +404,3 @@ def test_hub_filter_16bit_keys(sage):
             ref = oracle.bfs(g.off, g.col, s)
             lv, _, _ = G.bfs(s, push_only=True)
             assert np.array_equal(lv, ref)
-
-
-@pytest.mark.parametrize("sym,seed", [(False, 3), (True, 4)])
-def test_pagerank_blocked_push_parity(sage, sym, seed):
-    """Push PageRank with propagation blocking (pr_blocked = 1: per-target-block bins, applied block
-    by block) within 1e-6 of the oracle on RMAT and on a UK-like graph (crawl order: most arcs stay
-    in their block), on repeated calls and after a reorder (bins rebuilt for the new labels)."""
-    g = sg.rmat(16, 16, seed=seed, symmetric=sym)
-    xr = oracle.pagerank(g.off, g.col, 0.85, 20)
-    with sage.load_csr(g.off, g.col, symmetric=sym, pr_blocked=1) as G:
-        for _ in range(2):
-            x, _ = G.pagerank(0.85, 20, push_only=True)
-            assert np.max(np.abs(x - xr) / xr) <= 1e-6
-        G.reorder(rounds=1)
-        x, _ = G.pagerank(0.85, 20, push_only=True)
-        assert np.max(np.abs(x - xr) / xr) <= 1e-6
-    uk = sg.uk_like(n=300000, seed=2, n_tendrils=10, tmin=20, tmax=60, hmax=1 << 12)
-    xr = oracle.pagerank(uk.off, uk.col, 0.85, 10)
-    with sage.load_csr(uk.off, uk.col, pr_blocked=1) as G:
-        x, _ = G.pagerank(0.85, 10)
-        assert np.max(np.abs(x - xr) / xr) <= 1e-6

@@ -18,7 +18,6 @@ p.add_argument("--op", default="bfs_push", choices=["bfs_push", "bfs_do", "sssp"
 p.add_argument("--reps", type=int, default=3)
 p.add_argument("--tile-cta", type=int, default=256)
 p.add_argument("--align", type=int, default=4)
-p.add_argument("--pr-blocked", type=int, default=0)
 a = p.parse_args()
 if a.graph == "rmat":
     g = sg.rmat(a.scale, 16, 1, True)
@@ -30,8 +29,7 @@ w = sg.weights(g, 1)
 s = stream = torch.cuda.Stream()   # the library's work and the events on one stream
 torch.cuda.set_stream(stream)
 G = sage.load_csr(torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda(), torch.from_numpy(w).cuda(),
-                  symmetric=g.symmetric, borrow=True, stream=stream.cuda_stream, tile_cta=a.tile_cta, align=a.align,
-                  pr_blocked=a.pr_blocked)
+                  symmetric=g.symmetric, borrow=True, stream=stream.cuda_stream, tile_cta=a.tile_cta, align=a.align)
 src = sg.sources(g, a.reps, seed=2)
 lv = torch.empty(g.n, dtype=torch.int32, device="cuda")
 for i in range(a.reps):

@@ -16,7 +16,7 @@ g = sg.rmat(12, 16, seed=1, symmetric=True)
 w = sg.weights(g, 1)
 s = int(sg.sources(g, 1, seed=2)[0])
 ref = oracle.bfs(g.off, g.col, s)
-with sage.load_csr(g.off, g.col, w, symmetric=True, hub_filter=1, pr_blocked=1) as G:
+with sage.load_csr(g.off, g.col, w, symmetric=True, hub_filter=1) as G:
     for po in (True, False):
         lv, par, _ = G.bfs(s, push_only=po, parents=True)
         assert np.array_equal(lv, ref)

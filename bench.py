@@ -351,8 +351,10 @@ def main():
             "l2_hit_rate_pct": (tr or {}).get("lts_hit_rate_pct"),
             "compulsory_floor_bytes": floor,
             "floor_frac": floor / (kms * 1e-3) / 1e9 / peaks["hbm_gbs"],
-            "kernel": ("k_bfs<4> (persistent TP+RTS consumer)" if not multi else
-                       "host-sequenced NCCL levels (k_mpush + alltoall + k_mapply), time incl. exchange"),
+            "kernel": ("k_bfs_fused_hub<4,3> (persistent fused runtime-TP + RTS consumer)" if not multi else
+                       "host-sequenced levels (k_mpush + " + ("peer-memory inbox ORs + barrier" if G.peer_exchange
+                                                              else "NCCL all-to-all(v)")
+                       + " + k_mapply), time incl. exchange"),
             "peak_source": peak_src,
             "model": "SURVEY §8(d): 20 B/expanded vertex + 8 B/inspected arc + 8 B/discovered vertex",
             "kernel_ms": kms, "model_bytes_per_launch": kbytes}

@@ -78,6 +78,12 @@ typedef struct {
                                   caller (e.g. torch.distributed); required when world > 1       */
   int64_t v_begin, v_end;      /* global vertex block [v_begin, v_end) owned by this rank; ranks
                                   cover [0, n) contiguously in rank order                       */
+  int32_t exchange;            /* push-BFS frontier exchange: 0 = automatic - over
+                                  peer memory (the push kernel ORs each remote candidate into its
+                                  owner's inbox bitmap through NVLink, then one stream-ordered
+                                  barrier) when every rank can map every other rank's memory with
+                                  native atomics, else the collectives; 1 = collectives only (the
+                                  sparse / dense all-to-all(v)).  All ranks must pass the same value. */
 } sage_dist;
 
 /* Tile ladder used by every kernel and by the reorder's sample (Alg. 2; readings
@@ -221,7 +227,8 @@ sage_status sage_get_permutation(const sage_graph *g, int32_t *new_id_of_old);
  * col m, w m (w may be NULL).  Used to check the relabelled graph's isomorphism.             */
 sage_status sage_get_csr(const sage_graph *g, int64_t *off_out, int32_t *col_out, uint32_t *w_out);
 
-/* Graph sizes: any pointer may be NULL.                                                        */
+/* Graph sizes: any pointer may be NULL.  *flags = the load flags | 0x100 (rows sorted) | 0x200
+ * (reordered) | 0x400 (multi-GPU: the push exchange runs over peer memory, sage_dist.exchange). */
 sage_status sage_graph_info(const sage_graph *g, int64_t *n, int64_t *m, int64_t *n_local,
                             int64_t *v_begin, uint32_t *flags);
 

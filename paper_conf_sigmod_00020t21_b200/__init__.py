@@ -44,7 +44,7 @@ class Options(ctypes.Structure):
 
 class Dist(ctypes.Structure):
     _fields_ = [("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p),
-                ("v_begin", ctypes.c_int64), ("v_end", ctypes.c_int64)]
+                ("v_begin", ctypes.c_int64), ("v_end", ctypes.c_int64), ("exchange", ctypes.c_int32)]
 
 
 class Csr(ctypes.Structure):
@@ -174,6 +174,11 @@ class Graph:
     @property
     def handle(self):
         return self._h
+
+    @property
+    def peer_exchange(self) -> bool:
+        """Multi-GPU: the push frontier exchange runs over peer memory (sage_dist.exchange = 0)."""
+        return bool(self.flags & 0x400)
 
     def free(self):
         if self._h:
@@ -324,7 +329,8 @@ def load_csr(off, col, w=None, n: int | None = None, symmetric: bool = False, pu
              align: int = 4, alpha: float = 15.0, beta: float = 18.0, stream=None, ctas_per_sm: int = 0,
              hub_filter: int = 0,
              rank: int = 0, world: int = 1, nccl_unique_id: bytes | None = None,
-             v_begin: int = 0, v_end: int | None = None, host_columns: bool = False) -> Graph:
+             v_begin: int = 0, v_end: int | None = None, host_columns: bool = False,
+             exchange: int = 0) -> Graph:
     """sage_load_csr.  ``off``/``col``/``w`` are host arrays or tensors, or CUDA tensors."""
     po, ko, dev_o = _ptr(off, np.int64)
     pc, kc, dev_c = _ptr(col, np.int32)
@@ -359,7 +365,7 @@ def load_csr(off, col, w=None, n: int | None = None, symmetric: bool = False, pu
     if nccl_unique_id is not None:
         idbuf = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
         dist = Dist(rank, world, ctypes.cast(idbuf, ctypes.c_void_p).value, v_begin,
-                    v_end if v_end is not None else csr.n)
+                    v_end if v_end is not None else csr.n, exchange)
         csr.dist = ctypes.pointer(dist)
     h = ctypes.c_void_p()
     _check(lib().sage_load_csr(ctypes.byref(csr), ctypes.byref(h)))

@@ -75,6 +75,13 @@ struct Comm {
   unsigned long long *hmap = nullptr, *dmap = nullptr;   // mapped pinned stats (16 u64) + device alias
   unsigned long long pub_seq = 0;
   uint32_t *pcand = nullptr, *pown = nullptr;        // parents: p*P proposals, own P after min
+  // fused exchange over peer memory (sage_dist.exchange = 0 and every rank mappable): one
+  // cudaMalloc'd (IPC-able) region per rank = the BFS inbox bitmap (Wp words) followed by the
+  // SSSP candidate minima of the own rows (P words); peers[q] = rank q's region as seen from here
+  bool p2p = false;
+  uint32_t *inbox = nullptr;
+  void *peers[kMaxRanks] = {};
+  uint32_t **d_peers = nullptr;                       // device copy of peers (p entries)
   PartMap pm;
 };
 
@@ -101,6 +108,8 @@ struct MultiArgs {
   int vec_ok;
   int lvl;                         // current level L
   PartMap pm;
+  uint32_t *const *pin;            // peer form: pin[q] = rank q's region (inbox Wp words, then the
+                                   // SSSP minima P words), nullptr = collective form
   uint32_t *sp_send;               // sparse form: p blocks of (sp_cap + 2) words [count, 0, ids...]
   const uint32_t *sp_recv;
   long long sp_cap;                // 0 = dense form this level
@@ -149,6 +158,9 @@ struct BfsPushMulti {
         if (fb_next) atomicOr(fb_next + (p >> 5), bit);
         v[j] = lv;                   // enqueue the LOCAL row id
         in[j] = true;
+      } else if (a->pin) {          // candidate for its owner: OR into its inbox over NVLink
+        const int q = (int)(p / a->pm.P);
+        atomicOr(a->pin[q] + ((p >> 5) - (long long)q * (a->pm.P >> 5)), bit);
       } else if (a->sp_cap) {       // candidate for its owner: sparse form (global id)
         const int q = (int)(p / a->pm.P);
         uint32_t *blk = a->sp_send + (long long)q * (a->sp_cap + 2);
@@ -181,6 +193,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_mpush(const __grid_constant__ Mul
   f.flc = &a.ctl->set[(L + 1) % 3].flc.v;
   consume_log<VEC>(f, a.L, a.q[L & 1], &a.ctl->set[L % 3], a.off, a.col, nullptr, &wsm[warp],
                    fsrc[warp], a.vec_ok);
+  if (a.pin) __threadfence_system();   // the peer ORs are performed before the barrier that follows
 }
 
 // K2' of the deferred contraction for the vertices k_mpush claimed locally.
@@ -190,7 +203,8 @@ __global__ void __launch_bounds__(kBlock) k_mclassify(const __grid_constant__ Mu
                     &a.ctl->set[(L + 1) % 3]);
 }
 
-// Owners apply the candidates received from every other rank.
+// Owners apply the candidates received from every other rank (dense form: the p - 1 received
+// slices; peer form: the own inbox, cleared as it is read for the next level).
 __global__ void __launch_bounds__(kBlock) k_mapply(const __grid_constant__ MultiArgs a) {
   __shared__ WarpScratch wsm[kWarps];
   const int warp = threadIdx.x >> 5;
@@ -209,8 +223,14 @@ __global__ void __launch_bounds__(kBlock) k_mapply(const __grid_constant__ Multi
     uint32_t nw_bits = 0;
     if (w < words) {
       uint32_t cand = 0;
-      for (int r = 0; r < a.pm.p; ++r)
-        if (r != a.pm.rank) cand |= a.recv[(long long)r * Wp + w];
+      if (a.pin) {
+        uint32_t *box = a.pin[a.pm.rank] + w;
+        cand = *box;
+        if (cand) *box = 0u;
+      } else {
+        for (int r = 0; r < a.pm.p; ++r)
+          if (r != a.pm.rank) cand |= a.recv[(long long)r * Wp + w];
+      }
       if (w == words - 1 && (a.n_local & 31)) cand &= (1u << (a.n_local & 31)) - 1u;
       const long long gwd = (long long)a.pm.rank * Wp + w;
       const uint32_t own = a.visited[gwd];
@@ -390,8 +410,13 @@ struct SsspPushMulti {
           in[j] = !(atomicOr(a->inq_next + (lv >> 5), bit) & bit);
           v[j] = lv;                 // enqueue the LOCAL row id
         }
-      } else {
-        if (nd < ld_status(a->cand + p, keep)) atomicMin(a->cand + p, (uint32_t)nd);
+      } else if (nd < ld_status(a->cand + p, keep)) {
+        const uint32_t old = atomicMin(a->cand + p, (uint32_t)nd);
+        if (a->pin && (uint32_t)nd < old) {   // peer form: cand = the minimum sent so far; improve
+          const int q = (int)(p / a->pm.P);   // the owner's minimum over NVLink
+          const long long Wp = a->pm.P >> 5;
+          atomicMin(a->pin[q] + Wp + (p - (long long)q * a->pm.P), (uint32_t)nd);
+        }
       }
     }
   }
@@ -409,6 +434,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_msssp_push(const __grid_constant_
   f.next_cs = &a.ctl->set[(L + 1) % 3];
   consume_log<VEC>(f, a.L, a.q[L & 1], &a.ctl->set[L % 3], a.off, a.col, a.w, &wsm[warp], fsrc[warp],
                    a.vec_ok);
+  if (a.pin) __threadfence_system();
 }
 
 // Owners apply the minima received for their rows: one warp per 32-row word of the dedupe bitmap.
@@ -597,6 +623,17 @@ __global__ void k_fill_f64(double *p, long long n, double v) {
 }
 
 // ============================================================================ host side
+__global__ void k_peer_probe(uint32_t *const *peers, int world, int rank) {
+  const int q = threadIdx.x;
+  if (q < world && q != rank)
+    atomicOr(reinterpret_cast<unsigned long long *>(peers[q]), 1ull << rank);
+  __threadfence_system();
+}
+__global__ void k_peer_check(const unsigned long long *mine, int world, int rank, unsigned long long *bad) {
+  const unsigned long long all = world == 64 ? ~0ull : (1ull << world) - 1ull;
+  *bad = *mine != (all & ~(1ull << rank)) ? 1ull : 0ull;
+}
+
 sage_status init_comm(sage_graph *g, const sage_dist *ds) {
   Comm *c = new Comm();
   g->comm = c;
@@ -658,8 +695,41 @@ sage_status init_comm(sage_graph *g, const sage_dist *ds) {
     return SAGE_E_NOMEM;
   }
   memset(c->hmap, 0, 16 * sizeof(unsigned long long));
+  // the fused push exchange over peer memory (sage_dist.exchange == 0); every rank takes the same
+  // decision because peer_map's verdict is collective
+  if (c->world > 1 && ds->exchange == 0) {
+    cudaError_t e2 = cudaMalloc((void **)&c->inbox, 4 * (size_t)c->Wp * 33);
+    if (e2 != cudaSuccess) return cuda_fail(g, e2, "peer inbox");
+    cudaMemsetAsync(c->inbox, 0, 4 * (size_t)c->Wp * 33, g->stream);
+    s = c->x->peer_map(g, c->inbox, c->peers);
+    if (s == SAGE_OK) {
+      if ((s = dalloc(g, (void **)&c->d_peers, sizeof(void *) * (size_t)c->world)) != SAGE_OK) return s;
+      cudaMemcpyAsync(c->d_peers, c->peers, sizeof(void *) * (size_t)c->world, cudaMemcpyHostToDevice, g->stream);
+      // probe before trusting the mapping: every rank ORs its bit into every peer's first word
+      // pair, one barrier, every rank checks it holds exactly the others' bits; a collective
+      // verdict keeps all ranks on the same form
+      k_peer_probe<<<1, 64, 0, g->stream>>>(c->d_peers, c->world, c->rank);
+      XCHECK(c->x->barrier(g));
+      k_peer_check<<<1, 1, 0, g->stream>>>(reinterpret_cast<const unsigned long long *>(c->inbox), c->world,
+                                           c->rank, c->stats);
+      XCHECK(c->x->allreduce_sum_u64(g, c->stats, c->stats + 8, 1));
+      unsigned long long bad = 0;
+      cudaMemcpyAsync(&bad, c->stats + 8, sizeof(bad), cudaMemcpyDeviceToHost, g->stream);
+      cudaMemsetAsync(c->inbox, 0, 8, g->stream);
+      XCHECK(c->x->barrier(g));
+      if ((e2 = cudaStreamSynchronize(g->stream)) != cudaSuccess) return cuda_fail(g, e2, "peer map");
+      c->p2p = bad == 0;
+      if (!c->p2p) c->x->peer_unmap(c->peers);
+    } else if (s == SAGE_E_UNSUPPORTED) {
+      clear_error();
+    } else {
+      return s;
+    }
+  }
   return SAGE_OK;
 }
+
+bool comm_peer_exchange(const sage_graph *g) { return g->comm && g->comm->p2p; }
 
 void free_comm(sage_graph *g) {
   Comm *c = g->comm;
@@ -679,7 +749,10 @@ void free_comm(sage_graph *g) {
   dfree(g, c->glevel);
   dfree(g, c->pcand);
   dfree(g, c->pown);
+  dfree(g, c->d_peers);
   cudaStreamSynchronize(g->stream);
+  if (c->p2p) c->x->peer_unmap(c->peers);
+  if (c->inbox) cudaFree(c->inbox);
   if (c->hmap) cudaFreeHost(c->hmap);
   delete c->x;
   delete c;
@@ -755,6 +828,9 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
   a.do_enabled = do_enabled ? 1 : 0;
   a.vec_ok = g->vec_ok ? 1 : 0;
   a.pm = c->pm;
+  a.pin = c->p2p ? c->d_peers : nullptr;
+  if (c->p2p) cudaMemsetAsync(c->inbox, 0, 4 * (size_t)c->Wp, g->stream);   // ordered before any peer OR:
+                                                                            // the seed's stats allreduce follows
   if (source >= g->v_begin && source < g->v_end)
     k_mseed<<<1, 32, 0, g->stream>>>(a, (long long)source - g->v_begin);
   // global arcs of the source (level-0 frontier)
@@ -779,7 +855,7 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
     if (dir == 0) {
       // exchange form of this level (every rank knows the global arcs(F)): sparse lists of
       // capacity arcs(F) when that is smaller than a dense slice, else the dense slices
-      const long long cap = (c->world > 1 && (long long)aF_cur < c->Wp) ? (long long)aF_cur : 0;
+      const long long cap = (c->world > 1 && !c->p2p && (long long)aF_cur < c->Wp) ? (long long)aF_cur : 0;
       a.sp_cap = cap;
       if (cap) {
         const long long need = (cap + 2) * c->world;
@@ -800,7 +876,11 @@ sage_status run_bfs_multi(sage_graph *g, int32_t source, int32_t *level_out, int
       if (g->vec == 4) k_mpush<4><<<grid_push, kBlock, 0, g->stream>>>(a);
       else k_mpush<1><<<grid_push, kBlock, 0, g->stream>>>(a);
       k_mclassify<<<grid_push, kBlock, 0, g->stream>>>(a);
-      if (c->world > 1) {
+      if (c->p2p) {
+        // peer form: the candidates are already in the owners' inboxes; one barrier, then apply
+        XCHECK(c->x->barrier(g));
+        k_mapply<<<grid_push, kBlock, 0, g->stream>>>(a);
+      } else if (c->world > 1) {
         std::vector<size_t> off((size_t)c->world + 1);
         const size_t blk = cap ? 4 * (size_t)(cap + 2) : 4 * (size_t)c->Wp;
         for (int r = 0; r <= c->world; ++r) off[(size_t)r] = blk * (size_t)r;
@@ -932,6 +1012,7 @@ sage_status run_sssp_multi(sage_graph *g, int32_t source, uint32_t *dist_out, sa
   cudaMemsetAsync(ovf, 0, sizeof(int) * 4, g->stream);
   cudaMemsetAsync(t.dist, 0xff, sizeof(uint32_t) * (size_t)g->n_local, g->stream);
   cudaMemsetAsync(c->cand, 0xff, sizeof(uint32_t) * (size_t)P * c->world, g->stream);
+  if (c->p2p) cudaMemsetAsync(c->inbox + c->Wp, 0xff, sizeof(uint32_t) * (size_t)P, g->stream);
   for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * lwords, g->stream);
   cudaMemsetAsync(t.ctl, 0, offsetof(Ctl, rec), g->stream);
   MultiArgs a;
@@ -949,11 +1030,13 @@ sage_status run_sssp_multi(sage_graph *g, int32_t source, uint32_t *dist_out, sa
   a.pm = c->pm;
   a.dist = t.dist;
   a.cand = c->cand;
-  a.cown = c->cown;
+  a.cown = c->p2p ? c->inbox + c->Wp : c->cown;
+  a.pin = c->p2p ? c->d_peers : nullptr;
   a.overflow = ovf;
   if (source >= g->v_begin && source < g->v_end)
     k_msssp_seed<<<1, 32, 0, g->stream>>>(a, (long long)source - g->v_begin);
   const int grid = g->num_sms * 4;
+  if (c->p2p) XCHECK(c->x->barrier(g));   // every rank's minima reset before any peer update
   unsigned long long h6[6];
   long long exp_ = 0, arcs = 0, impr = 0;
   int iters = 0;
@@ -964,8 +1047,14 @@ sage_status run_sssp_multi(sage_graph *g, int32_t source, uint32_t *dist_out, sa
     a.inq_next = t.fb[(L + 1) % 3];
     if (g->vec == 4) k_msssp_push<4><<<grid, kBlock, 0, g->stream>>>(a);
     else k_msssp_push<1><<<grid, kBlock, 0, g->stream>>>(a);
-    XCHECK(c->x->reduce_scatter_min_u32(g, c->cand, c->cown, (size_t)P));
-    cudaMemsetAsync(c->cand, 0xff, sizeof(uint32_t) * (size_t)P * c->world, g->stream);
+    if (c->p2p) {
+      // peer form: the owners' minima were improved in place (monotone, never reset: an entry
+      // that does not beat dist is a no-op for k_msssp_apply); one barrier, then apply
+      XCHECK(c->x->barrier(g));
+    } else {
+      XCHECK(c->x->reduce_scatter_min_u32(g, c->cand, c->cown, (size_t)P));
+      cudaMemsetAsync(c->cand, 0xff, sizeof(uint32_t) * (size_t)P * c->world, g->stream);
+    }
     if (c->world > 1) k_msssp_apply<<<grid, kBlock, 0, g->stream>>>(a);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) {

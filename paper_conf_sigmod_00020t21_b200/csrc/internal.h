@@ -32,6 +32,7 @@ sage_status ensure_pagerank_log(sage_graph *g);
 // comm.cu (multi-GPU)
 sage_status init_comm(sage_graph *g, const sage_dist *ds);
 void free_comm(sage_graph *g);
+bool comm_peer_exchange(const sage_graph *g);   // the push exchange runs over peer memory
 
 // cooperative persistent launch helper
 sage_status launch_coop(sage_graph *g, const void *fn, int grid, void **args, const char *what,

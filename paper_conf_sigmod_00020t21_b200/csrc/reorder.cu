@@ -336,7 +336,10 @@ static sage_status sample_args(sage_graph *g, SampleArgs *a, int lgS) {
 // A sweep's counter updates are random over the n members; when the counters do not fit L2 the
 // sweep runs in passes over member ranges of at most kPassBytes of counters each (every pass reads
 // the sample again, ~1 ms of column stream at C3, but its atomics stay L2-resident).
-constexpr size_t kPassBytes = 48ull << 20;
+#ifndef SAGE_PASS_MB
+#define SAGE_PASS_MB 48
+#endif
+constexpr size_t kPassBytes = (size_t)SAGE_PASS_MB << 20;
 template <int MODE>
 static sage_status launch_sample(sage_graph *g, const SampleArgs &a0, size_t counter_bytes = 8) {
   const int bufn = g->ladder.B > 32 ? g->ladder.B : 32;

@@ -1062,6 +1062,11 @@ __device__ __forceinline__ void record_level_fused(Ctl *ctl, int L, const Counte
 
 // Push-only BFS level loop with the fused runtime tiling.
 constexpr unsigned long long kHubReloadMinChanges = 256;   // reload the CTA's hub table after such levels
+// Profiling builds only (tools/level_isolate.sh): the fused kernel stops after level L, so that the
+// counter difference of two builds (L and L-1) is level L alone.  Default -1 = off (dead code).
+#ifndef SAGE_BFS_STOP_AFTER
+#define SAGE_BFS_STOP_AFTER -1
+#endif
 template <int VEC, int HT>
 __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *wsm,
                                                typename BfsPushT<HT>::Src (*fsrc)[32], uint8_t *ht) {
@@ -1163,6 +1168,7 @@ __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *w
     const unsigned long long nF = ldcg(&nxt->nF.v);
     if (blockIdx.x == 0 && threadIdx.x == 0) record_level_fused(ctl, L, cur, nxt);
     if (nF == 0) break;
+    if (SAGE_BFS_STOP_AFTER >= 0 && L >= SAGE_BFS_STOP_AFTER) break;   // profiling build only (below)
     if (L + 1 >= a.max_levels) {
       if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = 1;
       break;
@@ -1178,6 +1184,7 @@ __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *w
       grid_barrier(&ctl->bar);
       if (ldcg(&ctl->tail_state) == 1) break;
       L = ldcg(&ctl->tail_resume) - 1;   // ++L resumes the grid at the returned level
+      if (SAGE_BFS_STOP_AFTER >= 0 && L >= SAGE_BFS_STOP_AFTER) break;
       continue;
     }
   }

@@ -30,6 +30,7 @@ struct NcclXport : Xport {
   ncclComm_t nc = nullptr;
   ~NcclXport() override {
     if (nc) ncclCommDestroy(nc);
+    if (scratch) cudaFree(scratch);
   }
   sage_status allgather(sage_graph *g, const void *send, void *recv, size_t bytes) override {
     XN(ncclAllGather(send, recv, bytes, ncclUint8, nc, g->stream), "ncclAllGather");
@@ -71,6 +72,75 @@ struct NcclXport : Xport {
     XN(ncclGroupEnd(), "ncclGroupEnd");
     return SAGE_OK;
   }
+  unsigned long long *scratch = nullptr;   // barrier word + IPC handle exchange (device)
+  sage_status ensure_scratch(sage_graph *g) {
+    if (scratch) return SAGE_OK;
+    const cudaError_t e = cudaMalloc((void **)&scratch, 64 + (size_t)world * sizeof(cudaIpcMemHandle_t));
+    if (e != cudaSuccess) return cuda_fail(g, e, "xport scratch");
+    cudaMemsetAsync(scratch, 0, 64, g->stream);
+    return SAGE_OK;
+  }
+  sage_status barrier(sage_graph *g) override {
+    sage_status s = ensure_scratch(g);
+    if (s != SAGE_OK) return s;
+    XN(ncclAllReduce(scratch, scratch + 1, 1, ncclUint64, ncclSum, nc, g->stream), "ncclAllReduce(barrier)");
+    return SAGE_OK;
+  }
+  sage_status peer_map(sage_graph *g, void *mine, void **peers) override {
+    sage_status s = ensure_scratch(g);
+    if (s != SAGE_OK) return s;
+    for (int q = 0; q < world; ++q) peers[q] = nullptr;
+    peers[rank] = mine;
+    // every rank's IPC handle, then every rank's verdict (all ranks must agree on the form)
+    cudaIpcMemHandle_t h;
+    memset(&h, 0, sizeof(h));
+    unsigned long long fail = cudaIpcGetMemHandle(&h, mine) != cudaSuccess;
+    cudaGetLastError();
+    char *hs = reinterpret_cast<char *>(scratch + 8);
+    std::vector<cudaIpcMemHandle_t> all((size_t)world);
+    cudaMemcpyAsync(hs + rank * sizeof(h), &h, sizeof(h), cudaMemcpyHostToDevice, g->stream);
+    XN(ncclAllGather(hs + rank * sizeof(h), hs, sizeof(h), ncclUint8, nc, g->stream), "ncclAllGather(ipc)");
+    cudaMemcpyAsync(all.data(), hs, sizeof(h) * (size_t)world, cudaMemcpyDeviceToHost, g->stream);
+    cudaError_t e = cudaStreamSynchronize(g->stream);
+    if (e != cudaSuccess) return cuda_fail(g, e, "peer handle exchange");
+    int dev = 0;
+    cudaGetDevice(&dev);
+    for (int q = 0; q < world && !fail; ++q) {
+      if (q == rank) continue;
+      if (cudaIpcOpenMemHandle(&peers[q], all[(size_t)q], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        cudaGetLastError();
+        peers[q] = nullptr;
+        fail = 1;
+        break;
+      }
+      cudaPointerAttributes at;
+      int atom = 0;
+      if (cudaPointerGetAttributes(&at, peers[q]) != cudaSuccess || at.device == dev ||
+          cudaDeviceGetP2PAttribute(&atom, cudaDevP2PAttrNativeAtomicSupported, dev, at.device) != cudaSuccess ||
+          !atom)
+        fail = 1;
+      cudaGetLastError();
+    }
+    cudaMemcpyAsync(scratch + 2, &fail, sizeof(fail), cudaMemcpyHostToDevice, g->stream);
+    XN(ncclAllReduce(scratch + 2, scratch + 3, 1, ncclUint64, ncclSum, nc, g->stream), "ncclAllReduce(peer)");
+    unsigned long long nfail = 0;
+    cudaMemcpyAsync(&nfail, scratch + 3, sizeof(nfail), cudaMemcpyDeviceToHost, g->stream);
+    e = cudaStreamSynchronize(g->stream);
+    if (e != cudaSuccess) return cuda_fail(g, e, "peer verdict");
+    if (nfail) {
+      peer_unmap(peers);
+      peers[rank] = mine;
+      return SAGE_E_UNSUPPORTED;
+    }
+    return SAGE_OK;
+  }
+  void peer_unmap(void **peers) override {
+    for (int q = 0; q < world; ++q)
+      if (q != rank && peers[q]) {
+        cudaIpcCloseMemHandle(peers[q]);
+        peers[q] = nullptr;
+      }
+  }
 };
 
 Xport *make_nccl_xport(sage_graph *g, const void *id128, int rank, int world, sage_status *st) {
@@ -99,6 +169,7 @@ struct LoopSlot {
   void *recv = nullptr;
   const size_t *soff = nullptr, *roff = nullptr;
   cudaEvent_t ready = nullptr, done = nullptr;
+  void *peer = nullptr;
 };
 struct LoopGroup {
   int world = 0;
@@ -212,6 +283,18 @@ struct LoopXport : Xport {
                                b, cudaMemcpyDeviceToDevice, g->stream);
       }
     });
+  }
+  // one device: every rank's buffer is directly addressable
+  sage_status peer_map(sage_graph *, void *mine, void **peers) override {
+    grp->slot[rank].peer = mine;
+    grp->barrier();
+    for (int q = 0; q < world; ++q) peers[q] = grp->slot[q].peer;
+    grp->barrier();
+    return SAGE_OK;
+  }
+  void peer_unmap(void **) override {}
+  sage_status barrier(sage_graph *g) override {
+    return run(g, nullptr, nullptr, nullptr, nullptr, [] {});
   }
 };
 

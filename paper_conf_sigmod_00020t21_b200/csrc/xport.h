@@ -3,7 +3,8 @@
 // The multi-GPU level loop needs six collectives on device buffers, all enqueued
 // on the graph's stream.  Two implementations:
 //   * NCCL (the product): ncclAllGather / ncclAllReduce / ncclReduceScatter and grouped
-//     ncclSend/ncclRecv for the all-to-all(v), one process per GPU over NVLink / NVSwitch;
+//     ncclSend/ncclRecv for the all-to-all(v), one process per GPU over NVLink / NVSwitch; peer
+//     memory through CUDA IPC handles exchanged over NCCL (the push BFS's fused exchange);
 //   * loopback (TEST ONLY): p logical ranks in one process on ONE GPU, one host thread per rank,
 //     collectives done with stream-ordered device copies / reduction kernels between the ranks'
 //     buffers.  It lets the single-GPU test pool run the r > 0 code paths (remote owners, padded
@@ -35,6 +36,15 @@ struct Xport {
   // soff / roff are host arrays of world + 1 byte offsets (the counts must agree pairwise)
   virtual sage_status alltoallv(sage_graph *g, const void *send, const size_t *soff, void *recv,
                                 const size_t *roff) = 0;
+  // Peer memory (collective call): every rank exposes `mine` (a cudaMalloc'd buffer); on return
+  // peers[q] is a pointer this rank's kernels may load / store / atomically update in rank q's
+  // buffer (peers[rank] = mine).  SAGE_E_UNSUPPORTED on EVERY rank when any rank cannot map any
+  // other's memory with native atomics (the caller then keeps the collective exchange).
+  virtual sage_status peer_map(sage_graph *g, void *mine, void **peers) = 0;
+  virtual void peer_unmap(void **peers) = 0;
+  // Stream-ordered barrier: work enqueued on any rank's stream before it completes (its peer
+  // writes included) before work enqueued on any rank's stream after it starts.
+  virtual sage_status barrier(sage_graph *g) = 0;
 };
 
 // NCCL transport from a 128-byte ncclUniqueId.

@@ -5,7 +5,9 @@ has a remote owner.  sage_debug_loopback_id (test-only, include/sage.h) swaps NC
 transport (xport.h): p graphs in one process, one host thread per rank, the collectives done as
 stream-ordered device copies / reductions between the ranks' buffers.  Everything else — k_mpush
 with remote owners, the padded indexing for r > 0, the sparse (C1a) and dense (C1b) exchanges,
-k_mapply / k_mapply_sparse, the pull allgather, the SSSP min reduce-scatter and k_msssp_apply, the
+k_mapply / k_mapply_sparse, the fused exchange over peer memory (exchange = 0: k_mpush ORs remote
+candidates straight into the owner's inbox, on one GPU every rank's buffer is addressable), the pull
+allgather, the SSSP min reduce-scatter and k_msssp_apply, the
 PageRank reduce-scatter, the parent post-pass — is the product code.  The gathered slices must
 equal the oracle's result (BFS / SSSP bit-exact, PageRank <= 1e-6 relative).
 """
@@ -79,13 +81,15 @@ def _parents_ok(g, lv, par, s):
         assert y in g.col[g.off[x]:g.off[x + 1]]
 
 
+@pytest.mark.parametrize("exchange", [0, 1])
 @pytest.mark.parametrize("p", [2, 3, 4])
 @pytest.mark.parametrize("sym", [True, False])
-def test_loopback_bfs(sage, p, sym):
+def test_loopback_bfs(sage, p, sym, exchange):
     g = sg.rmat(14, 16, seed=3, symmetric=sym)
     srcs = [int(s) for s in sg.sources(g, 3, seed=2)]
 
     def fn(G, r):
+        assert G.peer_exchange == (exchange == 0)
         res = []
         for s in srcs:
             for po in ((True, False) if sym else (True,)):
@@ -93,7 +97,7 @@ def test_loopback_bfs(sage, p, sym):
                 res.append((s, po, lv.copy(), par.copy(), st))
         return res
 
-    out = run_ranks(sage, g, None, p, fn, skew=(p == 3))
+    out = run_ranks(sage, g, None, p, fn, skew=(p == 3), exchange=exchange)
     for k in range(len(out[0])):
         s, po = out[0][k][0], out[0][k][1]
         lv = np.concatenate([o[k][2] for o in out])
@@ -106,24 +110,27 @@ def test_loopback_bfs(sage, p, sym):
         assert st["edges_traversed"] == int(np.diff(g.off)[ref >= 0].sum()) // (2 if sym else 1)
 
 
-def test_loopback_bfs_long_path_sparse_levels(sage):
-    """A UK-like graph (crawl order, tendrils): hundreds of tiny levels, sparse exchange, remote
-    discoveries on block boundaries."""
+@pytest.mark.parametrize("exchange", [0, 1])
+def test_loopback_bfs_long_path_sparse_levels(sage, exchange):
+    """A UK-like graph (crawl order, tendrils): hundreds of tiny levels, sparse exchange (or the
+    peer inboxes), remote discoveries on block boundaries."""
     uk = sg.uk_like(n=60000, seed=1, n_tendrils=20, tmin=30, tmax=120, hmax=1 << 10)
     srcs = [int(s) for s in sg.sources(uk, 2, seed=2)]
-    out = run_ranks(sage, uk, None, 4, lambda G, r: [G.bfs(s, push_only=True)[0].copy() for s in srcs])
+    out = run_ranks(sage, uk, None, 4, lambda G, r: [G.bfs(s, push_only=True)[0].copy() for s in srcs],
+                    exchange=exchange)
     for k, s in enumerate(srcs):
         lv = np.concatenate([o[k] for o in out])
         assert np.array_equal(lv, oracle.bfs(uk.off, uk.col, s))
 
 
+@pytest.mark.parametrize("exchange", [0, 1])
 @pytest.mark.parametrize("p", [2, 3])
 @pytest.mark.parametrize("sym", [True, False])
-def test_loopback_sssp(sage, p, sym):
+def test_loopback_sssp(sage, p, sym, exchange):
     g = sg.rmat(13, 16, seed=5, symmetric=sym)
     w = sg.weights(g, 1)
     srcs = [int(s) for s in sg.sources(g, 3, seed=2)]
-    out = run_ranks(sage, g, w, p, lambda G, r: [G.sssp(s)[0].copy() for s in srcs])
+    out = run_ranks(sage, g, w, p, lambda G, r: [G.sssp(s)[0].copy() for s in srcs], exchange=exchange)
     for k, s in enumerate(srcs):
         d = np.concatenate([o[k] for o in out])
         assert np.array_equal(d, oracle.sssp(g.off, g.col, w, s)[0]), (p, sym, s)
@@ -144,6 +151,28 @@ def test_loopback_sssp_overflow(sage):
         return 0
 
     assert run_ranks(sage, g, w, 3, fn) == [sage.E_OVERFLOW] * 3
+    assert run_ranks(sage, g, w, 3, fn, exchange=1) == [sage.E_OVERFLOW] * 3
+
+
+def test_loopback_mixed_queries_peer_form(sage):
+    """BFS and SSSP alternating on the same graphs in the peer form: each query resets only its
+    own part of the shared peer region, so neither may leak into the other."""
+    g = sg.rmat(12, 16, seed=9, symmetric=True)
+    w = sg.weights(g, 3)
+    srcs = [int(s) for s in sg.sources(g, 3, seed=4)]
+
+    def fn(G, r):
+        assert G.peer_exchange
+        res = []
+        for s in srcs:
+            res.append(G.bfs(s, push_only=True)[0].copy())
+            res.append(G.sssp(s)[0].copy())
+        return res
+
+    out = run_ranks(sage, g, w, 3, fn)
+    for k, s in enumerate(srcs):
+        assert np.array_equal(np.concatenate([o[2 * k] for o in out]), oracle.bfs(g.off, g.col, s))
+        assert np.array_equal(np.concatenate([o[2 * k + 1] for o in out]), oracle.sssp(g.off, g.col, w, s)[0])
 
 
 @pytest.mark.parametrize("p", [2, 3])

@@ -263,6 +263,13 @@ __device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned *p) {
 __device__ __forceinline__ void st_release_gpu(unsigned *p, unsigned v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
+// CTA-interleaved warp rank: rank r is warp r / gridDim.x of CTA r % gridDim.x, so a level with
+// fewer work units than warps (the first `grabs` ranks take one each) spreads them over every SM
+// instead of packing them into the first few CTAs (C2 level 1: 354 CTA tiles went to 11 SMs).
+__device__ __forceinline__ long long warp_rank() {
+  return (long long)(threadIdx.x >> 5) * gridDim.x + blockIdx.x;
+}
+
 __device__ __forceinline__ void grid_barrier(GridBar *b) {
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -616,7 +623,7 @@ __device__ __forceinline__ bool classify_deferred(const long long *__restrict__ 
   const unsigned long long fl = ldcg(flc);
   if (!fl) return false;
   const unsigned lane = threadIdx.x & 31;
-  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long gw = warp_rank();
   const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
   const long long first = gw * 32, step = nw * 32;
   // pass A: what this warp's groups need (next group's ids and rows loaded ahead)
@@ -779,12 +786,42 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
                                             typename F::Src *fsrc, bool vec_ok, bool steal = true) {
   const unsigned lane = lane_id();
   const unsigned long long pol = policy_evict_first();
-  const long long gwarp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long gwarp = warp_rank();
   const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
   // all queue sizes in one round of loads (lane c holds cnt[c])
   const unsigned long long my_cnt = (int)lane <= L.ncls ? ldcg(&cs->cnt[lane].v) : 0ull;
+  // Small logs (every class fits in one grab per warp of a 1/(ncls+1) share of the grid): the
+  // classes are consumed CONCURRENTLY by disjoint warp groups (group = rank mod (ncls+1)) instead
+  // of one after another by the same warps — a small level's latency is then the longest class's
+  // dependent chain (ticket -> log entry -> row -> columns -> status -> claim), not their sum.
+  const int G = L.ncls + 1;
+  long long rank = gwarp, nranks = nwarps;
+  int group = -1;
+  {
+    unsigned long long need = 0;
+    if ((int)lane < L.ncls) {
+      const int t = L.B >> lane;
+      const int tps = 32 / ((t / VEC) < 32 ? (t / VEC) : 32);
+      need = (my_cnt + tps - 1) / tps;
+    } else if ((int)lane == L.ncls) {
+      need = (my_cnt + 31) / 32;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const unsigned long long y = __shfl_xor_sync(FULL, need, o);
+      need = y > need ? y : need;
+    }
+    const long long per = nwarps / G;
+    if (steal && per >= 1 && need <= (unsigned long long)per) {
+      group = (int)(gwarp % G);
+      rank = gwarp / G;
+      nranks = per;
+      if (rank >= per) group = G;   // the remainder warps take nothing (but still close below)
+    }
+  }
   int bcnt = 0;   // warp-uniform fill of ws->buf
   for (int c = 0; c < L.ncls; ++c) {
+    if (group >= 0 && c != group) continue;
     const int t = L.B >> c;
     const unsigned long long count = shfl64(my_cnt, c);
     if (count == 0) continue;
@@ -793,12 +830,12 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
     const int spt = (t / VEC) > 32 ? (t / (32 * VEC)) : 1;  // steps per tile
     // adaptive ticket batch: ~2 grabs per warp, <= 16 KB of columns per grab; warps beyond the
     // number of grabs skip the class (no ticket traffic on small levels)
-    unsigned long long batch = (count + SAGE_TK_GRABS * nwarps - 1) / (SAGE_TK_GRABS * nwarps);
+    unsigned long long batch = (count + SAGE_TK_GRABS * nranks - 1) / (SAGE_TK_GRABS * nranks);
     const unsigned long long bmax = (SAGE_TK_ELEMS / t) > (unsigned)tps ? (SAGE_TK_ELEMS / t) : tps;
     if (batch > bmax) batch = bmax;
     batch = ((batch + tps - 1) / tps) * tps;
     const unsigned long long grabs = (count + batch - 1) / batch;
-    if ((unsigned long long)gwarp >= grabs) continue;
+    if ((unsigned long long)rank >= grabs) continue;
     const int sub = lane / lpt, sl = lane % lpt;
     const bool contiguous = lpt < 32 && vec_ok && (VEC % 4) == 0;
     const int lg_spt = __ffs(spt) - 1;
@@ -812,7 +849,7 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
         base = shfl64(tk_next, 0);
         if (base < count && lane == 0) tk_next = atomicAdd(&cs->tk[c].v, batch);
       } else {
-        base = ((unsigned long long)gwarp + rr * (unsigned long long)nwarps) * batch;
+        base = ((unsigned long long)rank + rr * (unsigned long long)nranks) * batch;
       }
       if (base >= count) break;
       const unsigned long long end = (base + batch < count) ? base + batch : count;
@@ -975,13 +1012,13 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
   const unsigned long long fgrabs = (fcount + 31) / 32;
   unsigned long long frr = 0;
   for (;;) {
-    if (fcount == 0 || (unsigned long long)gwarp >= fgrabs) break;
+    if (fcount == 0 || (group >= 0 && group != L.ncls) || (unsigned long long)rank >= fgrabs) break;
     unsigned long long base = 0;
     if (steal) {
       if (lane == 0) base = atomicAdd(&cs->tk[L.ncls].v, 32ull);
       base = shfl64(base, 0);
     } else {
-      base = ((unsigned long long)gwarp + frr++ * (unsigned long long)nwarps) * 32ull;
+      base = ((unsigned long long)rank + frr++ * (unsigned long long)nranks) * 32ull;
     }
     if (base >= fcount) break;
     const bool valid = base + lane < fcount;

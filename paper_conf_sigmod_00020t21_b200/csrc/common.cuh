@@ -138,9 +138,20 @@ __device__ __forceinline__ void ld_row_pair(const long long *off, int v, long lo
 
 // L2 cache policies: the column / weight stream is read once per level -> evict_first; the
 // status words (visited bitmap, dist) are re-read at random all level long -> evict_last.
+// SAGE_COL_POLICY (A/B builds only): 0 = evict_first (default), 1 = evict_normal, 2 = evict_first
+// on half of the lines (fractional 0.5, the rest evict_unchanged)
+#ifndef SAGE_COL_POLICY
+#define SAGE_COL_POLICY 0
+#endif
 __device__ __forceinline__ unsigned long long policy_evict_first() {
   unsigned long long p;
+#if SAGE_COL_POLICY == 1
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+#elif SAGE_COL_POLICY == 2
+  asm volatile("createpolicy.fractional.L2::evict_first.L2::evict_unchanged.b64 %0, 0.5;" : "=l"(p));
+#else
   asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+#endif
   return p;
 }
 __device__ __forceinline__ unsigned long long policy_evict_last() {
@@ -794,6 +805,8 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
   // classes are consumed CONCURRENTLY by disjoint warp groups (group = rank mod (ncls+1)) instead
   // of one after another by the same warps — a small level's latency is then the longest class's
   // dependent chain (ticket -> log entry -> row -> columns -> status -> claim), not their sum.
+  // (Splitting big logs in proportion to their classes' elements was measured 2x slower on C2
+  // SSSP / PageRank / BC: the groups finish far apart.)
   const int G = L.ncls + 1;
   long long rank = gwarp, nranks = nwarps;
   int group = -1;

@@ -1645,6 +1645,17 @@ static void fill_stats(sage_graph *g, const Ctl &h, bool bfs, bool symmetric, do
   }
 }
 
+// true when p is device memory of the graph's GPU (cudaMalloc / a CUDA tensor), not host memory
+static bool is_own_device_ptr(const sage_graph *g, const void *p) {
+  if (!p) return false;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeDevice && at.device == g->device;
+}
+
 static sage_status check_common(sage_graph *g, int32_t source, const void *out) {
   if (!g || !out) {
     set_error("null argument");
@@ -1690,18 +1701,25 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
 #else
   const bool fused = !do_enabled;   // push-only: Tiled Partitioning fused into the consumer
 #endif
+  // outputs written in place: when the caller's buffers are device memory of this GPU and no ID
+  // translation is needed, the kernel initialises and fills them directly (no output copy)
+  const bool direct_lv = !g->reordered && !g->online && is_own_device_ptr(g, level_out);
+  const bool direct_par = parent_out && !g->reordered && is_own_device_ptr(g, parent_out);
   cudaEvent_t e0 = t.ev[0], e1 = t.ev[1], e2 = t.ev[2];
   cudaEventRecord(e0, g->stream);
   const size_t words = (size_t)((g->n + 31) / 32 + 8);
   if (!fused) {   // (the fused kernel initialises its query state itself)
-    cudaMemsetAsync(t.level, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
-    if (parent_out) cudaMemsetAsync(t.parent, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
+    cudaMemsetAsync(direct_lv ? level_out : t.level, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
+    if (parent_out)
+      cudaMemsetAsync(direct_par ? parent_out : t.parent, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
     cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
     for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
     cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);
   }
   TravArgs a = make_args(g);
   a.parent = parent_out ? t.parent : nullptr;
+  if (direct_lv) a.level = level_out;
+  if (direct_par) a.parent = parent_out;
   a.do_enabled = do_enabled ? 1 : 0;
   a.steal = (call_flags & SAGE_F_NO_STEALING) ? 0 : 1;
   a.src = src;
@@ -1765,8 +1783,8 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   // counters and outputs in one stream round trip (one synchronisation per call)
   Ctl &h = *t.hctl;
   cudaMemcpyAsync(&h, t.ctl, offsetof(Ctl, rec), cudaMemcpyDeviceToHost, g->stream);
-  if ((s = translate_out_i32(g, t.level, level_out, false)) != SAGE_OK) return s;
-  if (parent_out && (s = translate_out_i32(g, t.parent, parent_out, true)) != SAGE_OK) return s;
+  if (!direct_lv && (s = translate_out_i32(g, t.level, level_out, false)) != SAGE_OK) return s;
+  if (parent_out && !direct_par && (s = translate_out_i32(g, t.parent, parent_out, true)) != SAGE_OK) return s;
   cudaError_t e = cudaStreamSynchronize(g->stream);
   if (e != cudaSuccess) return cuda_fail(g, e, "BFS");
   float ms = 0, kms = 0;
@@ -1811,11 +1829,15 @@ extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_o
   cudaEventRecord(e0, g->stream);
   const size_t words = (size_t)((g->n + 31) / 32 + 8);
   cudaMemsetAsync(ovf, 0, sizeof(int) * 2, g->stream);
-  cudaMemsetAsync(t.dist, 0xff, sizeof(uint32_t) * (size_t)g->n_local, g->stream);
+  // distances written in place when the caller's buffer is device memory of this GPU (no copy)
+  const bool direct = !g->reordered && is_own_device_ptr(g, dist_out);
+  uint32_t *dd = direct ? dist_out : t.dist;
+  cudaMemsetAsync(dd, 0xff, sizeof(uint32_t) * (size_t)g->n_local, g->stream);
   cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
   for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
   cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);
   TravArgs a = make_args(g);
+  a.dist = dd;
   k_seed<<<1, 32, 0, g->stream>>>(a, src, 1);
   cudaEventRecord(e1, g->stream);
   const void *fn = g->vec == 4 ? (const void *)k_sssp<4> : (const void *)k_sssp<1>;
@@ -1850,7 +1872,7 @@ extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_o
   if (hovf[0]) {
     cudaMemsetAsync(ovf + 1, 0, sizeof(int), g->stream);
     k_overflow_check<<<g->num_sms * 8, 256, 0, g->stream>>>((const long long *)g->off, g->col,
-                                                            t.dist, g->n_local, ovf + 1);
+                                                            dd, g->n_local, ovf + 1);
     cudaMemcpyAsync(hovf + 1, ovf + 1, sizeof(int), cudaMemcpyDeviceToHost, g->stream);
     cudaStreamSynchronize(g->stream);
   }
@@ -1864,14 +1886,14 @@ extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_o
     unsigned long long *dra = nullptr, hra = 0;
     if ((s = dalloc(g, (void **)&dra, sizeof(unsigned long long))) != SAGE_OK) return s;
     cudaMemsetAsync(dra, 0, sizeof(unsigned long long), g->stream);
-    k_reached_arcs<<<g->num_sms * 8, 256, 0, g->stream>>>((const long long *)g->off, t.dist,
+    k_reached_arcs<<<g->num_sms * 8, 256, 0, g->stream>>>((const long long *)g->off, dd,
                                                           g->n_local, dra);
     cudaMemcpyAsync(&hra, dra, sizeof(hra), cudaMemcpyDeviceToHost, g->stream);
     cudaStreamSynchronize(g->stream);
     dfree(g, dra);
     st->edges_traversed = (int64_t)((g->flags & SAGE_F_SYMMETRIC) ? hra / 2 : hra);
   }
-  if ((s = translate_out_u32(g, t.dist, dist_out)) != SAGE_OK) return s;
+  if (!direct && (s = translate_out_u32(g, t.dist, dist_out)) != SAGE_OK) return s;
   e = cudaStreamSynchronize(g->stream);
   if (e != cudaSuccess) return cuda_fail(g, e, "SSSP output");
   return SAGE_OK;

@@ -706,6 +706,9 @@ __device__ __forceinline__ void bfs_body(const TravArgs &a, WarpScratch *wsm, ty
 #ifndef SAGE_FUSED_PACK
 #define SAGE_FUSED_PACK 0
 #endif
+#ifndef SAGE_FUSED_LOGC
+#define SAGE_FUSED_LOGC 2   // classes logged for phase B (1 = CTA tiles only; 2 = + the B/2 tiles)
+#endif
 // Push-only BFS (the configuration of the headline): Tiled Partitioning runs INSIDE the consumer,
 // as Alg. 2's runtime tiling does (the expand kernel splits each frontier vertex's
 // adjacency list into tiles when it reaches it), instead of as a separate K2' grid phase with its
@@ -897,11 +900,20 @@ __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, Cou
 #endif
     {
     // (2) sub-CTA class tiles, consumed here: the class members' tile starts and sources are
-    //     staged in shared memory, then lane groups of t/VEC lanes take one tile each per step
+    //     staged in shared memory, then lane groups of t/VEC lanes take one tile each per step.
+    //     Classes below SAGE_FUSED_LOGC are logged for phase B's stealing instead (A/B knob: a
+    //     chunk's longest serial work shrinks from 32 x (B-1) to 32 x (B/2^LOGC - 1) elements).
     for (int c = 1; c < L.ncls; ++c) {
       const int t = L.B >> c;
       const unsigned cm = __ballot_sync(FULL, act && (s.r & t));
       if (!cm) continue;
+      if (c < SAGE_FUSED_LOGC) {
+        unsigned long long b0 = 0;
+        if (lane == 0) b0 = atomicAdd(&cur->cnt[c].v, (unsigned long long)__popc(cm));
+        b0 = shfl64(b0, 0);
+        if (cm & (1u << lane)) Q.cls[c][b0 + __popc(cm & lt)] = v;
+        continue;
+      }
       const int nt = __popc(cm);
       __syncwarp();
       if (cm & (1u << lane)) {
@@ -1152,8 +1164,8 @@ __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *w
     if (blockIdx.x == 0 && threadIdx.x == 0 && L < kMaxRec) ctl->rec[L].t_mid = globaltimer();
     // phase B: the logged tiles (CTA tiles; every class on a small level), Resident Tile Stealing
     bool logged = ldcg(&cur->cnt[0].v) > 0;
-    if (log_all)
-      for (int c = 1; c <= a.L.ncls; ++c) logged |= ldcg(&cur->cnt[c].v) > 0;
+    for (int c = 1; c <= a.L.ncls; ++c)
+      if (log_all || c < SAGE_FUSED_LOGC) logged |= ldcg(&cur->cnt[c].v) > 0;
     if constexpr (HT > 0) {   // the CTA's copy of the table with the hubs phase A inserted
       if (ldcg(&cur->hubc.v) >= kHubReloadMinChanges) {
         hub_load<HT>(a, ht);

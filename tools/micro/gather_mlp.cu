@@ -62,6 +62,15 @@ int main() {
   uint32_t *bm, *out;
   const uint32_t words = 1u << 19;  // 2 MB
   cudaMalloc(&bm, words * 4); cudaMemset(bm, 1, words * 4); cudaMalloc(&out, 64);
+  if (getenv("MLP_SWEEP")) {   // loads in flight per thread at the fused BFS's L1 (64 KB table + 35 KB static)
+    run<3, 1>(bm, words, out, sms, 1024, 1, 100);
+    run<3, 2>(bm, words, out, sms, 1024, 1, 100);
+    run<3, 4>(bm, words, out, sms, 1024, 1, 100);
+    run<3, 8>(bm, words, out, sms, 1024, 1, 100);
+    run<3, 16>(bm, words, out, sms, 1024, 1, 100);
+    run<3, 4>(bm, words, out, sms, 512, 2, 100);
+    return 0;
+  }
   for (int dyn : {0, 16, 48, 80, 112, 144, 176, 208}) {
     run<0, 8>(bm, words, out, sms, 1024, 1, dyn);
     run<3, 8>(bm, words, out, sms, 1024, 1, dyn);

@@ -62,8 +62,9 @@ enum {
                               expansion (Alg. 2/3).  Can also be set per call (sage_bfs_ex).     */
                            /* 32u: reserved (an experimental binned push level of round 1, removed;
                               DESIGN.md §5 keeps its measurements)                                */
-  SAGE_F_NO_STEALING = 64u /* per call (sage_bfs_ex), ablation (Fig. 10): tiles are dealt to
-                              warps statically instead of through Resident Tile Stealing        */
+  SAGE_F_NO_STEALING = 64u /* per call (sage_bfs_ex; sage_pagerank_ex push form, which then also
+                              skips the windowed form), ablation (Fig. 10): tiles are
+                              dealt to warps statically instead of through Resident Tile Stealing */
 };
 
 /* Multi-GPU description (1D vertex partition).  NULL in sage_csr = single GPU.
@@ -228,7 +229,9 @@ sage_status sage_get_permutation(const sage_graph *g, int32_t *new_id_of_old);
 sage_status sage_get_csr(const sage_graph *g, int64_t *off_out, int32_t *col_out, uint32_t *w_out);
 
 /* Graph sizes: any pointer may be NULL.  *flags = the load flags | 0x100 (rows sorted) | 0x200
- * (reordered) | 0x400 (multi-GPU: the push exchange runs over peer memory, sage_dist.exchange). */
+ * (reordered) | 0x400 (multi-GPU: the push exchange runs over peer memory, sage_dist.exchange)
+ * | 0x800 (push PageRank runs the windowed form: chosen at the first push PageRank call when most
+ * arcs stay near their source, e.g. web graphs in crawl order).               */
 sage_status sage_graph_info(const sage_graph *g, int64_t *n, int64_t *m, int64_t *n_local,
                             int64_t *v_begin, uint32_t *flags);
 

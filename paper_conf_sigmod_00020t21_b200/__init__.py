@@ -180,6 +180,13 @@ class Graph:
         """Multi-GPU: the push frontier exchange runs over peer memory (sage_dist.exchange = 0)."""
         return bool(self.flags & 0x400)
 
+    @property
+    def pagerank_windowed(self) -> bool:
+        """Push PageRank runs the windowed form (chosen at the first push PageRank call)."""
+        fl = ctypes.c_uint32()
+        _check(lib().sage_graph_info(self._h, None, None, None, None, ctypes.byref(fl)))
+        return bool(fl.value & 0x800)
+
     def free(self):
         if self._h:
             lib().sage_free(self._h)
@@ -220,12 +227,14 @@ class Graph:
         _check(lib().sage_sssp(self._h, int(source), o.ptr, ctypes.byref(st)))
         return o.obj, st.as_dict()
 
-    def pagerank(self, damping: float = 0.85, iterations: int = 20, out=None, push_only: bool = False):
-        """sage_pagerank_ex (pull form on symmetric graphs unless push_only)."""
+    def pagerank(self, damping: float = 0.85, iterations: int = 20, out=None, push_only: bool = False,
+                 stealing: bool = True):
+        """sage_pagerank_ex (pull form on symmetric graphs unless push_only; stealing=False runs the
+        log-based push without stealing, never the windowed form)."""
         o = _out(out, self.n_local, np.float64)
         st = Stats()
-        _check(lib().sage_pagerank_ex(self._h, float(damping), int(iterations), o.ptr,
-                                      F_PUSH_ONLY if push_only else 0, ctypes.byref(st)))
+        fl = (F_PUSH_ONLY if push_only else 0) | (0 if stealing else F_NO_STEALING)
+        _check(lib().sage_pagerank_ex(self._h, float(damping), int(iterations), o.ptr, fl, ctypes.byref(st)))
         return o.obj, st.as_dict()
 
     def bc(self, sources, out=None):

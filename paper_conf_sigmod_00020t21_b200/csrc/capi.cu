@@ -491,7 +491,7 @@ sage_status sage_graph_info(const sage_graph *g, int64_t *n, int64_t *m, int64_t
   if (n_local) *n_local = g->n_local;
   if (v_begin) *v_begin = g->v_begin;
   if (flags) *flags = g->flags | (g->rows_sorted ? 0x100u : 0u) | (g->reordered ? 0x200u : 0u) |
-                    (comm_peer_exchange(g) ? 0x400u : 0u);
+                    (comm_peer_exchange(g) ? 0x400u : 0u) | (g->pr.win == 1 ? 0x800u : 0u);
   return SAGE_OK;
 }
 

@@ -50,6 +50,8 @@ struct PageRankState {      // the all-V resident tile log (built once, reused; 
   void *c = nullptr;              // pull form: x_u / out(u) (fp32, or fp64 when damping > 0.9)
   size_t c_bytes = 0;
   CounterSet *cs = nullptr;       // device copy of the log's counters (+ rotating tickets)
+  int win = -1;                   // windowed push chosen for this graph (-1 = not measured yet)
+  double locality = 0.0;          // sampled fraction of arcs within the window's halo of their source
 };
 
 }  // namespace sage
@@ -95,5 +97,5 @@ struct sage_graph {
   long long online_thr = 0, online_pending = 0, online_rounds = 0, online_movers = 0, online_swaps = 0;
   uint32_t *samp_w = nullptr;
   unsigned long long *samp_acc = nullptr;
-  int grid_bfs = 0, grid_bfs_hub = 0, grid_bfs_fused = 0, grid_bfs_fused_hub = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0, grid_pr_pull64 = 0;   // persistent grid sizes
+  int grid_bfs = 0, grid_bfs_hub = 0, grid_bfs_fused = 0, grid_bfs_fused_hub = 0, grid_sssp = 0, grid_pr = 0, grid_pr_pull = 0, grid_pr_pull64 = 0, grid_pr_win = 0;   // persistent grid sizes
 };

@@ -522,6 +522,7 @@ static sage_status one_round(sage_graph *g, RoundBufs &b, int lgS, const uint8_t
   dfree(g, g->pr.dangling);
   g->pr.dangling = nullptr;
   g->pr.valid = false;
+  g->pr.win = -1;   // arc locality changes with the labels: measured again
   return SAGE_OK;
 }
 

@@ -404,3 +404,57 @@ def test_hub_filter_16bit_keys(sage):
             ref = oracle.bfs(g.off, g.col, s)
             lv, _, _ = G.bfs(s, push_only=True)
             assert np.array_equal(lv, ref)
+
+
+def _banded_graph(n=120000, seed=7):
+    """Directed graph whose arcs mostly stay near their source: offsets at and around the windowed
+    push's halo (4096) and chunk (8192) boundaries, empty rows, long rows (> 32 and > 128 arcs in
+    one 32-row group) and a few far arcs.  Duplicate arcs and self-loops are kept (R8)."""
+    rng = np.random.default_rng(seed)
+    offs = np.array([0, 1, -1, 2, 31, -32, 4095, -4095, 4096, -4096, 4097, 8191, 8192, -8193, 12287])
+    rows = []
+    for u in range(n):
+        k = int(rng.integers(0, 6))
+        if u % 997 == 0:
+            k = 300
+        if u % 13 == 0:
+            k = 0
+        t = u + rng.choice(offs, size=k)
+        far = rng.random(k) < 0.1
+        t[far] = rng.integers(0, n, size=int(far.sum()))
+        rows.append(np.clip(t, 0, n - 1))
+    deg = np.array([len(r) for r in rows], dtype=np.int64)
+    off = np.zeros(n + 1, dtype=np.int64)
+    off[1:] = np.cumsum(deg)
+    col = np.concatenate(rows).astype(np.int32)
+    return off, col
+
+
+@pytest.mark.gpu
+def test_pagerank_windowed_push(sage):
+    """Windowed push PageRank (shared-memory accumulation of near targets) vs the
+    oracle on graphs that select it: a banded multigraph with targets on the halo / chunk
+    boundaries, and a UK-like crawl-order graph; the log-based push (stealing off) agrees."""
+    off, col = _banded_graph()
+    uk = sg.uk_like(n=300000, seed=2, n_tendrils=20, tmin=20, tmax=80, hmax=1 << 14)
+    for o, c in ((off, col), (uk.off, uk.col)):
+        for d, it in ((0.85, 20), (0.99, 7)):
+            xr = oracle.pagerank(o, c, d, it)
+            with sage.load_csr(o, c) as G:
+                x, _ = G.pagerank(d, it)
+                assert G.pagerank_windowed
+                assert np.max(np.abs(x - xr) / xr) <= 1e-6
+                x2, _ = G.pagerank(d, it, stealing=False)
+                assert np.max(np.abs(x2 - xr) / xr) <= 1e-6
+    # more than one target block of the far-arc bins (blocks of 2^22 vertices)
+    big = sg.uk_like(n=5_000_000, seed=3, mu_ln=1.5, n_tendrils=10, tmin=20, tmax=40)
+    xr = oracle.pagerank(big.off, big.col, 0.85, 5)
+    with sage.load_csr(big.off, big.col) as G:
+        x, _ = G.pagerank(0.85, 5)
+        assert G.pagerank_windowed
+        assert np.max(np.abs(x - xr) / xr) <= 1e-6
+    # scrambled RMAT has no locality: the log-based push is kept
+    g = sg.rmat(18, 16, seed=3, symmetric=False)
+    with sage.load_csr(g.off, g.col) as G:
+        x, _ = G.pagerank(0.85, 5)
+        assert not G.pagerank_windowed

@@ -3,6 +3,7 @@
 // Build: nvcc -O3 -gencode arch=compute_100a,code=sm_100a -o atom64 atom64.cu
 #include <cstdio>
 #include <cstdint>
+#include <cstdlib>
 
 __device__ __forceinline__ uint32_t hsh(uint32_t x) {
   x ^= x >> 16; x *= 0x7feb352d; x ^= x >> 15; x *= 0x846ca68b; x ^= x >> 16; return x;
@@ -42,6 +43,12 @@ int main() {
   void *buf;
   const uint32_t big = 1u << 26;   // 512 MB of 8-byte words
   cudaMalloc(&buf, (size_t)big * 8); cudaMemset(buf, 0, (size_t)big * 8);
+  if (getenv("SIZE_SWEEP")) {   // footprint sweep: 2, 8, 16, 32, 64, 128 MB (fp64 atomicAdd = REDG when unused)
+    const char *names[] = {"2 MB", "8 MB", "16 MB", "32 MB", "64 MB", "128 MB", "512 MB"};
+    int i = 0;
+    for (uint32_t words : {1u << 18, 1u << 20, 1u << 21, 1u << 22, 1u << 23, 1u << 24, big}) run<0, 4>(buf, words, sms, 0, names[i++]);
+    return 0;
+  }
   for (uint32_t words : {1u << 18, big}) {
     const char *w = words == big ? "512 MB random" : "2 MB random";
     run<0, 4>(buf, words, sms, 0, w); run<1, 4>(buf, words, sms, 0, w); run<2, 4>(buf, words, sms, 0, w);

@@ -20,7 +20,15 @@ stream = torch.cuda.Stream()
 torch.cuda.set_stream(stream)
 G = sage.load_csr(torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda(), stream=stream.cuda_stream)
 x = torch.empty(g.n, dtype=torch.float64, device="cuda")
-G.pagerank(0.85, 2, out=x)
-_, st = G.pagerank(0.85, iters, out=x)
-print(json.dumps({"graph": g.name, "n": g.n, "arcs": g.m, "iters": iters, "ms_per_iteration": st["ms"] / iters,
-                  "gen_s": round(time.time() - t0, 1)}))
+res = {"graph": g.name, "n": g.n, "arcs": g.m, "iters": iters, "gen_s": round(time.time() - t0, 1)}
+for form, stealing in (("windowed", True),) + ((("log", False),) if not os.environ.get("PR_WIN_ONLY") else ()):
+    G.pagerank(0.85, 2, out=x, stealing=stealing)
+    _, st = G.pagerank(0.85, iters, out=x, stealing=stealing)
+    res[form] = {"ms_per_iteration": st["kernel_ms"] / iters,
+                 "model_GBps": st["model_bytes"] / (st["kernel_ms"] * 1e-3) / 1e9}
+    if stealing:
+        res[form]["selected"] = G.pagerank_windowed
+        xw = x.cpu()
+    else:
+        res["max_rel_diff_windowed_vs_log"] = float(((xw - x.cpu()).abs() / x.cpu()).max())
+print(json.dumps(res))

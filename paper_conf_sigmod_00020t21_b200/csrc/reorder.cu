@@ -44,7 +44,8 @@ struct SampleArgs {
   unsigned long long *loc1, *loc3;
   void *cd;                    // stage 2: L - R per vertex (int32 when it cannot overflow, else int64)
   int cd32;
-  const int2 *lohi;
+  const uint32_t *lohi;        // stage 2: (lo << 1) | e per vertex, interval length f + e (see k_s2_update)
+  long long f;                 // this step's floor length (nsec >> step)
   const int *target;
   unsigned long long *objective;
   const uint32_t *vw;          // online sampling: occurrences of each vertex's tiles (null = 1)
@@ -141,9 +142,10 @@ __global__ void __launch_bounds__(256) k_sample(const __grid_constant__ SampleAr
           const int cnt = lower_bound_s(seg, t, (sx + 1) << a.lgS) - lower_bound_s(seg, t, sx << a.lgS) - 1;
           if (cnt > 0) atomicAdd(a.loc1 + x, (unsigned long long)cnt * wt);
         } else if (MODE == 1) {
-          const int2 lh = a.lohi[x];
-          if (lh.y - lh.x > 1) {
-            const long long lo = lh.x, hi = lh.y, mid = lo + (hi - lo) / 2;
+          const uint32_t lh = a.lohi[x];
+          const long long len = a.f + (lh & 1u);
+          if (len > 1) {
+            const long long lo = lh >> 1, hi = lo + len, mid = lo + len / 2;
             const int ilo = lower_bound_s(seg, t, lo << a.lgS);
             const int imid = lower_bound_s(seg, t, mid << a.lgS);
             const int ihi = lower_bound_s(seg, t, hi << a.lgS);
@@ -174,22 +176,27 @@ __global__ void __launch_bounds__(256) k_sample(const __grid_constant__ SampleAr
   }
 }
 
-__global__ void k_s2_init(int2 *lohi, long long n, int nsec) {
+// Stage-2 intervals: every step halves every open interval, so after k steps of [0, nsec) a
+// length is floor(nsec / 2^k) or one more; one bit e per vertex holds which (4 B per vertex
+// instead of an explicit (lo, hi) pair: half the random-read footprint of a sweep).
+__global__ void k_s2_init(uint32_t *lohi, long long n) {
   const long long stride = (long long)gridDim.x * blockDim.x;
-  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
-    lohi[v] = make_int2(0, nsec);
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) lohi[v] = 0u;
 }
 // stage-2 decision: L >= R -> hi = mid, else lo = mid (R21), then reset the counts
-__global__ void k_s2_update(int2 *lohi, void *cd, int cd32, long long n) {
+__global__ void k_s2_update(uint32_t *lohi, void *cd, int cd32, long long n, long long f) {
   const long long stride = (long long)gridDim.x * blockDim.x;
+  const long long f2 = f >> 1;   // the next step's floor length
   for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
-    int2 lh = lohi[v];
+    const uint32_t lh = lohi[v];
     const long long d = cd32 ? (long long)static_cast<int *>(cd)[v] : static_cast<long long *>(cd)[v];
-    if (lh.y - lh.x > 1) {
-      const int mid = lh.x + (lh.y - lh.x) / 2;
-      if (d >= 0) lh.y = mid; else lh.x = mid;   // L >= R -> left half (R21)
-      lohi[v] = lh;
+    long long lo = lh >> 1, len = f + (lh & 1u);
+    if (len > 1) {
+      const long long half = len / 2;
+      if (d >= 0) len = half;                   // L >= R -> left half [lo, mid) (R21)
+      else { lo += half; len -= half; }         // right half [mid, hi)
     }
+    lohi[v] = ((uint32_t)lo << 1) | (uint32_t)(len - f2);
     if (cd32) static_cast<int *>(cd)[v] = 0;
     else static_cast<long long *>(cd)[v] = 0;
   }
@@ -210,10 +217,10 @@ __global__ void k_max_u32(const unsigned *x, long long n, unsigned *out) {
   }
   if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
 }
-__global__ void k_s2_final(const int2 *lohi, int *target, long long n) {
+__global__ void k_s2_final(const uint32_t *lohi, int *target, long long n) {
   const long long stride = (long long)gridDim.x * blockDim.x;
   for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
-    target[v] = lohi[v].x;
+    target[v] = (int)(lohi[v] >> 1);
 }
 // movers (R22): loc3 > loc1 (and a candidate); keys for the (gain desc) sort
 __global__ void k_movers(const unsigned long long *loc1, const unsigned long long *loc3,
@@ -333,11 +340,13 @@ static sage_status sample_args(sage_graph *g, SampleArgs *a, int lgS) {
   return SAGE_OK;
 }
 
-// A sweep's counter updates are random over the n members; when the counters do not fit L2 the
-// sweep runs in passes over member ranges of at most kPassBytes of counters each (every pass reads
-// the sample again, ~1 ms of column stream at C3, but its atomics stay L2-resident).
+// A sweep's counter updates are random over the n members; above kPassBytes of counters the sweep
+// runs in passes over member ranges (every pass reads the whole sample again).  Measured at C3
+// (166 MB of counters): 48 MB passes 2.13 s per round, one pass 1.28 s — the extra sample reads and
+// binary searches cost more than the DRAM-resident counter updates they avoid; so one pass up to
+// 1 GB of counters.
 #ifndef SAGE_PASS_MB
-#define SAGE_PASS_MB 48
+#define SAGE_PASS_MB 1024
 #endif
 constexpr size_t kPassBytes = (size_t)SAGE_PASS_MB << 20;
 template <int MODE>
@@ -378,7 +387,7 @@ static sage_status objective(sage_graph *g, int lgS, unsigned long long *out) {
 
 struct RoundBufs {
   unsigned long long *loc1 = nullptr, *loc3 = nullptr, *cl = nullptr;   // cl: stage-2 L - R
-  int2 *lohi = nullptr;
+  uint32_t *lohi = nullptr;
   int *target = nullptr, *ids = nullptr, *mids = nullptr, *mids2 = nullptr, *sr = nullptr;
   uint8_t *mover = nullptr, *cand = nullptr;
   unsigned long long *gkeys = nullptr, *gkeys2 = nullptr;
@@ -421,11 +430,12 @@ static sage_status one_round(sage_graph *g, RoundBufs &b, int lgS, const uint8_t
   // stage 1
   if ((s = launch_sample<0>(g, a)) != SAGE_OK) return s;
   // stage 2: ceil(log2(nsec)) halving sweeps
-  k_s2_init<<<grid, 256, 0, g->stream>>>(b.lohi, n, (int)nsec);
+  k_s2_init<<<grid, 256, 0, g->stream>>>(b.lohi, n);
   const int steps = ceil_log2(nsec);
   for (int it = 0; it < steps; ++it) {
+    a.f = nsec >> it;
     if ((s = launch_sample<1>(g, a, a.cd32 ? 4 : 8)) != SAGE_OK) return s;
-    k_s2_update<<<grid, 256, 0, g->stream>>>(b.lohi, a.cd, a.cd32, n);
+    k_s2_update<<<grid, 256, 0, g->stream>>>(b.lohi, a.cd, a.cd32, n, a.f);
   }
   k_s2_final<<<grid, 256, 0, g->stream>>>(b.lohi, b.target, n);
   // stage 3
@@ -545,7 +555,7 @@ static sage_status alloc_round(sage_graph *g, RoundBufs &b, bool with_cand) {
   void **ps[] = {(void **)&b.loc1, (void **)&b.loc3, (void **)&b.cl};
   for (auto p : ps)
     if ((s = dalloc(g, p, sizeof(unsigned long long) * (size_t)n)) != SAGE_OK) return s;
-  if ((s = dalloc(g, (void **)&b.lohi, sizeof(int2) * (size_t)n)) != SAGE_OK) return s;
+  if ((s = dalloc(g, (void **)&b.lohi, sizeof(uint32_t) * (size_t)n)) != SAGE_OK) return s;
   int **pi[] = {&b.target, &b.ids, &b.mids, &b.mids2, &b.sr};
   for (auto p : pi)
     if ((s = dalloc(g, (void **)p, sizeof(int) * (size_t)n)) != SAGE_OK) return s;

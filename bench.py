@@ -522,7 +522,11 @@ def _extras(a, G, g, srcs, level, flush, stream, sage):
         ex["c4_shape"] = {"graph": f"uk_like n={uk.n} arcs={uk.m} (C4 shape at 1/10.5 size)",
                           "bfs_ms": float(np.mean([t for t, _ in r])), "bfs_levels": r[-1][1]["levels"],
                           "bfs_gteps": len(r) / sum(t * 1e-3 * 1e9 / st["edges_traversed"] for t, st in r),
-                          "pagerank_ms_20_iter": rp[0][0]}
+                          "pagerank_ms_20_iter": rp[0][0],
+                          "pagerank_form": "windowed push" if U.pagerank_windowed else "log-based push"}
+        U.pagerank(0.85, 20, out=xu, stealing=False)
+        rl = _time_calls(lambda i: U.pagerank(0.85, 20, out=xu, stealing=False)[1], 1, flush, stream)
+        ex["c4_shape"]["pagerank_log_form_ms_20_iter"] = rl[0][0]
     # out-of-core (NEXT #4): C2 with col in pinned host memory read zero-copy over the host link
     # (copied into library-owned pinned memory at load); push and DO BFS, parity checked
     with sage.load_csr(g.off, g.col, symmetric=True, host_columns=True, align=32,

@@ -189,6 +189,11 @@ __device__ __forceinline__ uint32_t ld_colu(const uint32_t *p, unsigned long lon
 #ifndef SAGE_STATUS_L1
 #define SAGE_STATUS_L1 2
 #endif
+// small-log class split (`consume_log`): the classes run concurrently while every class needs at
+// most SAGE_SPLIT_K grabs per warp of its group (A/B knob)
+#ifndef SAGE_SPLIT_K
+#define SAGE_SPLIT_K 1
+#endif
 // stealing ticket batches (`consume_log`): grabs per warp per class, column elements per grab
 #ifndef SAGE_TK_GRABS
 #define SAGE_TK_GRABS 2
@@ -825,7 +830,7 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
       need = y > need ? y : need;
     }
     const long long per = nwarps / G;
-    if (steal && per >= 1 && need <= (unsigned long long)per) {
+    if (steal && per >= 1 && need <= (unsigned long long)per * SAGE_SPLIT_K) {
       group = (int)(gwarp % G);
       rank = gwarp / G;
       nranks = per;

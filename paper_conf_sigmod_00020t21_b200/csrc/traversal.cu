@@ -753,7 +753,10 @@ template <int HT> struct HtOf<BfsPushT<HT>> { static constexpr int value = HT; }
 // serially; instead phase A only classifies (Tiled Partitioning into the level's log, every class)
 // and phase B consumes the whole log with stealing — the latency of a small level is then one
 // classification round plus one parallel consume, as with the separate K2' phase.
-constexpr unsigned long long kFusedLogAll = 8192;
+#ifndef SAGE_LOGALL
+#define SAGE_LOGALL 8192
+#endif
+constexpr unsigned long long kFusedLogAll = SAGE_LOGALL;
 template <int VEC, class F>
 __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, CounterSet *cur, const int *fl_in,
                                               const Queues &Q, WarpScratch *ws, typename F::Src *fsrc,

@@ -52,7 +52,14 @@ def run(cfg):
             _, st = G.pagerank(0.85, 20, out=x)
             pr.append(st["ms"])
         res["pagerank_20_ms"] = pr
-        res["pagerank_form"] = "push (Alg. 1 l.26-29), fp64 atomics over the resident all-V log"
+        res["pagerank_form"] = ("push (Alg. 1 l.26-29), windowed: near targets in a shared-memory fp64 window, "
+                                "heavy far targets in a shared hot table, the rest fp64 reductions in global memory"
+                                if G.pagerank_windowed else
+                                "push (Alg. 1 l.26-29), fp64 reductions over the resident all-V log")
+        xl = torch.empty_like(x)
+        _, stl = G.pagerank(0.85, 20, out=xl, stealing=False)
+        res["pagerank_log_form_ms_per_iteration"] = stl["ms"] / 20
+        res["pagerank_log_form_max_rel_diff"] = float(((xl - x).abs() / x).max())
         res["pagerank_ms_per_iteration"] = min(pr) / 20
         res["pagerank_GBps_model"] = 20 * (40.0 * g.n + 12.0 * g.m) / (min(pr) * 1e-3) / 1e9
         t1 = time.time()

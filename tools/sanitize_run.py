@@ -1,6 +1,6 @@
 """Small workload for compute-sanitizer (memcheck / racecheck / synccheck / initcheck): every
 product kernel family on RMAT-12 (BFS push + DO with the fused tiling and the hub filter forced
-on, SSSP, PageRank pull / push / blocked push, a reorder round, BC), results checked against the
+on, SSSP, PageRank pull / push / windowed push, a reorder round, BC), results checked against the
 oracle so a sanitizer run that perturbs timing still has to produce the right answers."""
 import os
 import sys
@@ -31,4 +31,11 @@ with sage.load_csr(g.off, g.col, w, symmetric=True, hub_filter=1) as G:
     b, _ = G.bc([s])
     br = oracle.bc(g.off, g.col, [s])
     assert np.all(np.abs(b - br) <= 1e-9 * np.max(np.abs(br)) + 1e-6 * np.abs(br))
+# windowed push PageRank (chosen on a crawl-ordered UK-like graph)
+uk = sg.uk_like(n=200000, seed=1, n_tendrils=10, tmin=20, tmax=40, hmax=1 << 12)
+with sage.load_csr(uk.off, uk.col) as G:
+    x, _ = G.pagerank(0.85, 3)
+    assert G.pagerank_windowed
+    xr = oracle.pagerank(uk.off, uk.col, 0.85, 3)
+    assert np.max(np.abs(x - xr) / xr) <= 1e-6
 print("sanitize workload ok")

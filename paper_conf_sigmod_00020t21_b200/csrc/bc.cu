@@ -222,6 +222,7 @@ using namespace sage;
 
 extern "C" sage_status sage_bc(sage_graph *g, const int32_t *sources, int64_t n_sources, double *bc_out,
                                sage_stats *st) {
+  NvtxRange nvtx_("sage_bc");
   clear_error();
   if (!g || !bc_out || n_sources < 0 || (n_sources > 0 && !sources)) {
     set_error("null argument");

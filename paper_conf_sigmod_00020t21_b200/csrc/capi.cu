@@ -248,6 +248,7 @@ const char *sage_last_error(void) { return g_last_error.c_str(); }
 const char *sage_version(void) { return "sage-b200 0.1 (sm_100a)"; }
 
 sage_status sage_load_csr(const sage_csr *in, sage_graph **out) {
+  NvtxRange nvtx_("sage_load_csr");
   clear_error();
   if (!out) {
     set_error("out is NULL");

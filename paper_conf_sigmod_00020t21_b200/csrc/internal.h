@@ -1,10 +1,20 @@
 // internal.h — host functions shared between the .cu files of libsage.so (not exported).
 #pragma once
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "graph.h"
 
 namespace sage {
+
+// NVTX range over one C-ABI call (SURVEY §5 tracing): visible in Nsight Systems / ncu --nvtx;
+// header-only NVTX v3, a no-op without an attached tool.
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange &) = delete;
+  NvtxRange &operator=(const NvtxRange &) = delete;
+};
 
 sage_status cuda_fail(sage_graph *g, cudaError_t e, const char *what);
 bool is_device_ptr(const void *p);

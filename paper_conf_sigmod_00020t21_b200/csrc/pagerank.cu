@@ -242,14 +242,20 @@ __global__ void __launch_bounds__(kBlock, 4) k_pagerank_pull(const __grid_consta
 // contiguous segment of col, streamed 32 elements per round with the owner row of each element
 // found by a 5-step shuffle search over the group's row starts (empty rows share the next row's
 // start, and the search takes the last of equal starts, i.e. the non-empty row).
+#ifndef SAGE_WIN_HALO
+#define SAGE_WIN_HALO 4096
+#endif
+#ifndef SAGE_WIN_HOTLG
+#define SAGE_WIN_HOTLG 12
+#endif
 constexpr int kWinR = 8192;                 // rows per chunk
-constexpr int kWinH = 4096;                 // halo on each side
+constexpr int kWinH = SAGE_WIN_HALO;        // halo on each side
 constexpr int kWinS = kWinR + 2 * kWinH;    // window entries (fp64): 128 KB of shared memory
 constexpr int kWinBlock = 1024;
 constexpr int kWinUnroll = 4;               // rounds of 32 elements in flight per warp
 constexpr long long kWinMaxDegree = 1 << 16;  // one warp streams a 32-row group: no huge rows
 constexpr double kWinMinLocality = 0.25;     // sampled share of arcs inside the halo
-constexpr int kWinHotLg = 12;                // hot far-target table: 4096 slots (48 KB)
+constexpr int kWinHotLg = SAGE_WIN_HOTLG;    // hot far-target table: 4096 slots (48 KB)
 constexpr int kWinHot = 1 << kWinHotLg;
 constexpr size_t kWinDyn = sizeof(double) * (kWinS + kWinHot) + sizeof(int) * kWinHot;
 #ifndef SAGE_WIN_HOT
@@ -505,6 +511,7 @@ using namespace sage;
 
 extern "C" sage_status sage_pagerank_ex(sage_graph *g, double damping, int32_t iterations,
                                         double *rank_out, uint32_t call_flags, sage_stats *st) {
+  NvtxRange nvtx_("sage_pagerank");
   clear_error();
   if (!g || !rank_out) {
     set_error("null argument");

@@ -716,6 +716,7 @@ extern "C" sage_status sage_online_reorder_info(const sage_graph *g, int64_t *ro
 
 extern "C" sage_status sage_reorder(sage_graph *g, int32_t rounds, const sage_reorder_opts *opt,
                                     sage_stats *st) {
+  NvtxRange nvtx_("sage_reorder");
   clear_error();
   if (!g || rounds < 0) {
     set_error("null graph or negative rounds");

@@ -1697,6 +1697,7 @@ using namespace sage;
 
 extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level_out,
                                    int32_t *parent_out, uint32_t call_flags, sage_stats *st) {
+  NvtxRange nvtx_("sage_bfs");
   clear_error();
   sage_status s = check_common(g, source, level_out);
   if (s != SAGE_OK) return s;
@@ -1822,6 +1823,7 @@ extern "C" sage_status sage_bfs(sage_graph *g, int32_t source, int32_t *level_ou
 
 extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_out,
                                  sage_stats *st) {
+  NvtxRange nvtx_("sage_sssp");
   clear_error();
   sage_status s = check_common(g, source, dist_out);
   if (s != SAGE_OK) return s;

@@ -282,7 +282,11 @@ __device__ __forceinline__ void st_release_gpu(unsigned *p, unsigned v) {
 // CTA-interleaved warp rank: rank r is warp r / gridDim.x of CTA r % gridDim.x, so a level with
 // fewer work units than warps (the first `grabs` ranks take one each) spreads them over every SM
 // instead of packing them into the first few CTAs (C2 level 1: 354 CTA tiles went to 11 SMs).
+#ifndef SAGE_WARP_RANK_LINEAR
+#define SAGE_WARP_RANK_LINEAR 0   // A/B: 1 = rank r is warp r % (warps per CTA) of CTA r / (warps per CTA)
+#endif
 __device__ __forceinline__ long long warp_rank() {
+  if (SAGE_WARP_RANK_LINEAR) return ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   return (long long)(threadIdx.x >> 5) * gridDim.x + blockIdx.x;
 }
 

@@ -28,12 +28,13 @@ wr = float(d["dram__bytes_write.sum"]) * scale.get(un["dram__bytes_write.sum"], 
 stalls = {k.replace("smsp__pcsamp_warps_issue_stalled_", ""): float(x) for k, x in d.items()
           if k.startswith("smsp__pcsamp_warps_issue_stalled") and not k.endswith("not_issued") and x}
 tot = sum(stalls.values())
-json.dump({"kernel": "k_bfs<4> push-only (SAGE_F_PUSH_ONLY), RMAT-24 sym, 1 launch = 1 BFS",
+json.dump({"kernel": d.get("Kernel Name", "?").split("(")[0] + " push-only (SAGE_F_PUSH_ONLY), RMAT-24 sym, 1 launch = 1 BFS",
            "source": f"profiles/{tag}_bfs_push_ncu.md (ncu --set full --clock-control none)",
            "bfs_push_bytes_per_launch": rd + wr, "dram_read_bytes": rd, "dram_write_bytes": wr,
+           "lts_hit_rate_pct": float(d["lts__t_sector_hit_rate.pct"]),
            "ncu_duration_ms": float(d["gpu__time_duration.sum"])}, open("profiles/traffic.json", "w"), indent=1)
 with open(f"profiles/{tag}_bfs_push_ncu.md", "w") as f:
-    f.write(f"# {tag} — ncu --set full of the persistent push BFS kernel (k_bfs<4>)\n\n")
+    f.write(f"# {tag} — ncu --set full of the persistent push BFS kernel ({d.get('Kernel Name', '?').split('(')[0]})\n\n")
     f.write("`ncu --set full --clock-control none --import-source on -k regex:k_bfs -s 2 -c 1 python tools/prof_run.py "
             "--scale 24 --reps 3 --op bfs_push` on one B200 (RMAT-24 symmetric, push-only; one launch = one BFS).\n\n")
     f.write("| metric | value | unit |\n|---|---|---|\n")

@@ -194,6 +194,11 @@ __device__ __forceinline__ uint32_t ld_colu(const uint32_t *p, unsigned long lon
 #ifndef SAGE_SPLIT_K
 #define SAGE_SPLIT_K 1
 #endif
+// medium logs: proportional class split while the log holds <= SAGE_SPLIT_PROP elements per warp
+// (0 = off; big logs measured 2x slower with it)
+#ifndef SAGE_SPLIT_PROP
+#define SAGE_SPLIT_PROP 0
+#endif
 // stealing ticket batches (`consume_log`): grabs per warp per class, column elements per grab
 #ifndef SAGE_TK_GRABS
 #define SAGE_TK_GRABS 2
@@ -839,6 +844,29 @@ __device__ __forceinline__ void consume_log(const F &f, const Ladder &L, const Q
       rank = gwarp / G;
       nranks = per;
       if (rank >= per) group = G;   // the remainder warps take nothing (but still close below)
+    } else if (steal && SAGE_SPLIT_PROP && nwarps >= 2 * G) {
+      // medium logs (a few hundred elements per warp in all): the classes still run concurrently,
+      // each with a share of the warps proportional to its elements (fragments ~4 per entry)
+      unsigned long long wk = 0;
+      if ((int)lane < L.ncls) wk = my_cnt * (unsigned long long)(L.B >> lane);
+      else if ((int)lane == L.ncls) wk = my_cnt * 4ull;
+      const unsigned long long tot = warp_sum64(wk);
+      if (tot > 0 && tot <= (unsigned long long)nwarps * SAGE_SPLIT_PROP) {
+        const unsigned long long spare = (unsigned long long)(nwarps - G);
+        const unsigned long long share = wk ? 1ull + (unsigned long long)((double)spare * (double)wk / (double)tot) : 0ull;
+        unsigned long long incl = share;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const unsigned long long y = __shfl_up_sync(FULL, incl, o);
+          if ((int)lane >= o) incl += y;
+        }
+        const unsigned m = __ballot_sync(FULL, (int)lane <= L.ncls && incl <= (unsigned long long)gwarp);
+        group = __popc(m);   // the class whose share holds this rank (G = none: idle remainder)
+        if (group < G) {
+          rank = gwarp - (long long)(shfl64(incl, group) - shfl64(share, group));
+          nranks = (long long)shfl64(share, group);
+        }
+      }
     }
   }
   int bcnt = 0;   // warp-uniform fill of ws->buf

@@ -703,6 +703,9 @@ __device__ __forceinline__ void bfs_body(const TravArgs &a, WarpScratch *wsm, ty
 }
 
 // ============================================================================ fused runtime tiling
+#ifndef SAGE_FUSED_PACK_SMALL
+#define SAGE_FUSED_PACK_SMALL 0   // A/B: 1 = the small-graph fused kernel packs the classes (C1: 207 vs 204 us)
+#endif
 #ifndef SAGE_FUSED_PACK
 #define SAGE_FUSED_PACK 0
 #endif
@@ -821,13 +824,30 @@ __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, Cou
         }
       }
     }
-#if SAGE_FUSED_PACK
+    // classes below SAGE_FUSED_LOGC go to the log (phase B) in both forms below
+#pragma unroll
+    for (int c = 1; c < SAGE_FUSED_LOGC; ++c) {
+      if (c >= L.ncls) break;
+      const unsigned cm = __ballot_sync(FULL, act && (s.r & (L.B >> c)));
+      if (!cm) continue;
+      unsigned long long b0 = 0;
+      if (lane == 0) b0 = atomicAdd(&cur->cnt[c].v, (unsigned long long)__popc(cm));
+      b0 = shfl64(b0, 0);
+      if (cm & (1u << lane)) Q.cls[c][b0 + __popc(cm & lt)] = v;
+    }
+    // small graphs (the 256-thread kernel without the hub table): every class's tiles of the chunk
+    // are packed into common warp steps, so a level's dependent column-load chains overlap
+    // (latency-bound levels); the hub kernel keeps one class at a time (C2: 3.22 vs 2.52 ms)
+    constexpr bool kPack = SAGE_FUSED_PACK || (SAGE_FUSED_PACK_SMALL && HtOf<F>::value == 0);
+    bool packed = false;
+    if constexpr (kPack) {
     // (2) sub-CTA class tiles, consumed here, all classes of the chunk packed into warp steps: tile
     //     k of class c (t = B >> c elements, lpt = t / VEC lanes) takes lanes [base_c + k * lpt, ..)
     //     of the chunk's lane sequence; classes in descending size keep every group aligned.  A
     //     lane finds its class, tile and owner vertex (nth set bit of the class ballot) and reads
     //     the owner's row end / residual by shuffle; each lane loads VEC consecutive elements.
     if (VEC == 4 && contig_ok && (L.B >> 1) <= 32 * VEC) {
+      packed = true;
       int cbase[kMaxCls + 1];
       unsigned cms[kMaxCls];
       int tl = 0;
@@ -835,7 +855,7 @@ __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, Cou
       for (int c = 1; c < kMaxCls; ++c) {
         cms[c] = 0;
         cbase[c] = tl;
-        if (c < L.ncls) {
+        if (c < L.ncls && c >= SAGE_FUSED_LOGC) {
           const int t = L.B >> c;
           cms[c] = __ballot_sync(FULL, act && (s.r & t));
           tl += __popc(cms[c]) * (t / VEC);
@@ -899,9 +919,9 @@ __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, Cou
 #pragma unroll
         for (int j = 0; j < VEC; ++j) push_filtered(f, in[j], vv[j], ws, bcnt, a.off, L);
       }
-    } else
-#endif
-    {
+    }
+    }
+    if (!packed) {
     // (2) sub-CTA class tiles, consumed here: the class members' tile starts and sources are
     //     staged in shared memory, then lane groups of t/VEC lanes take one tile each per step.
     //     Classes below SAGE_FUSED_LOGC are logged for phase B's stealing instead (A/B knob: a
@@ -909,14 +929,7 @@ __device__ __forceinline__ void fused_phase_a(const TravArgs &a, const F &f, Cou
     for (int c = 1; c < L.ncls; ++c) {
       const int t = L.B >> c;
       const unsigned cm = __ballot_sync(FULL, act && (s.r & t));
-      if (!cm) continue;
-      if (c < SAGE_FUSED_LOGC) {
-        unsigned long long b0 = 0;
-        if (lane == 0) b0 = atomicAdd(&cur->cnt[c].v, (unsigned long long)__popc(cm));
-        b0 = shfl64(b0, 0);
-        if (cm & (1u << lane)) Q.cls[c][b0 + __popc(cm & lt)] = v;
-        continue;
-      }
+      if (!cm || c < SAGE_FUSED_LOGC) continue;   // (logged above)
       const int nt = __popc(cm);
       __syncwarp();
       if (cm & (1u << lane)) {

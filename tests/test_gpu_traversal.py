@@ -458,3 +458,46 @@ def test_pagerank_windowed_push(sage):
     with sage.load_csr(g.off, g.col) as G:
         x, _ = G.pagerank(0.85, 5)
         assert not G.pagerank_windowed
+
+
+def test_outputs_in_place_and_translated(sage):
+    """BFS levels / parents and SSSP distances written straight into caller device buffers (no
+    output copy) equal the host-buffer path and the oracle — on the fused push path, the DO path,
+    SSSP, and after a reorder (where the ids are translated and the in-place path is off); stale
+    contents of the caller's buffer never leak through (the kernel initialises every entry)."""
+    import torch
+    g = sg.rmat(16, 16, seed=9, symmetric=True)
+    w = sg.weights(g, 3)
+    srcs = [int(x) for x in sg.sources(g, 3, seed=4)]
+    with sage.load_csr(g.off, g.col, w, symmetric=True) as G:
+        for rnd in range(2):
+            for s in srcs:
+                ref = oracle.bfs(g.off, g.col, s)
+                for po in (True, False):
+                    lv = torch.full((g.n,), 12345, dtype=torch.int32, device="cuda")
+                    par = torch.full((g.n,), 777, dtype=torch.int32, device="cuda")
+                    G.bfs(s, out=lv, parent_out=par, push_only=po)
+                    lvh, parh, _ = G.bfs(s, parents=True, push_only=po)
+                    assert np.array_equal(lv.cpu().numpy(), ref) and np.array_equal(lvh, ref)
+                    _parents_ok(g.off, g.col, ref, par.cpu().numpy(), s)
+                    _parents_ok(g.off, g.col, ref, parh, s)
+                d = torch.full((g.n,), 5, dtype=torch.int32, device="cuda")
+                G.sssp(s, out=d)
+                dref, _ = oracle.sssp(g.off, g.col, w, s)
+                assert np.array_equal(d.cpu().numpy().view(np.uint32), dref)
+            if rnd == 0:
+                G.reorder(rounds=1)
+
+
+def test_pagerank_windowed_after_reorder(sage):
+    """A reorder changes the labels, so the windowed push's locality is measured again; the ranks
+    (original ids) stay equal to the oracle before and after."""
+    uk = sg.uk_like(n=200000, seed=4, n_tendrils=10, tmin=20, tmax=60, hmax=1 << 12)
+    xr = oracle.pagerank(uk.off, uk.col, 0.85, 10)
+    with sage.load_csr(uk.off, uk.col) as G:
+        x, _ = G.pagerank(0.85, 10)
+        assert G.pagerank_windowed
+        assert np.max(np.abs(x - xr) / xr) <= 1e-6
+        G.reorder(rounds=1)
+        x2, _ = G.pagerank(0.85, 10)
+        assert np.max(np.abs(x2 - xr) / xr) <= 1e-6

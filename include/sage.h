@@ -158,7 +158,12 @@ sage_status sage_free(sage_graph *g);
 /* BFS from `source` (global id): level_out[v] = hop distance, -1 = unreachable (Alg. 1 l.2,
  * P:112).  level_out has n entries (n_local multi-GPU, the rank's slice).  parent_out (nullable)
  * receives a valid BFS-tree parent (-1 for the source and for unreachable vertices).
- * Direction switching is used iff the graph is SAGE_F_SYMMETRIC and not SAGE_F_PUSH_ONLY.     */
+ * Direction switching is used iff the graph is SAGE_F_SYMMETRIC and not SAGE_F_PUSH_ONLY.
+ * Output buffers may be host or device memory (caller-owned; written before the call returns).
+ * Device buffers of the graph's GPU are written IN PLACE by the kernel when no ID translation
+ * applies (not reordered); those writes follow the caller's earlier work on the graph's stream
+ * (sage_csr.cuda_stream) or, without one, on the legacy default stream.  On an error the
+ * contents of the output buffers are unspecified.                                              */
 sage_status sage_bfs(sage_graph *g, int32_t source, int32_t *level_out, int32_t *parent_out,
                      sage_stats *st);
 
@@ -168,7 +173,8 @@ sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level_out, int32
 
 /* Integer-weight SSSP ("iteratively update neighbors' distances"; reading R4): frontier
  * Bellman-Ford with atomicMin.  dist_out[v] = shortest distance, UINT32_MAX = unreachable.
- * Requires weights.  A finite distance >= UINT32_MAX -> SAGE_E_OVERFLOW (dist_out unspecified). */
+ * Requires weights.  A finite distance >= UINT32_MAX -> SAGE_E_OVERFLOW (dist_out unspecified).
+ * dist_out: host or device memory, written in place like sage_bfs's outputs.                  */
 sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_out, sage_stats *st);
 
 /* PageRank, push form of Alg. 1 l.26-29 over the resident all-V tile log;

@@ -27,6 +27,7 @@ struct TraversalState {     // per-query scratch, allocated on first use and kep
   int32_t *level = nullptr;       // BFS levels (int32, -1 = unvisited), n_local
   int32_t *parent = nullptr;      // BFS parents (allocated on first parent request)
   uint32_t *dist = nullptr;       // SSSP distances, n_local
+  cudaEvent_t ev_caller = nullptr;   // orders in-place output writes after the caller's stream
   uint32_t *visited = nullptr;    // visited bitmap, ceil(n/32) words (+ padding)
   uint32_t *fb[3] = {nullptr, nullptr, nullptr};  // frontier bitmaps (rotated), pull + SSSP dedupe
   Queues q[2];                    // double-buffered per-level tile logs

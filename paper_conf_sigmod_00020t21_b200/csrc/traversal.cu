@@ -611,13 +611,75 @@ __device__ __forceinline__ void hub_load(const TravArgs &a, uint8_t *ht) {
 
 // The BFS level loop (one persistent cooperative launch per query).  HT > 0: hub filter on (the
 // CTA holds the table in `ht`, HubGeom<HT>::bytes of shared memory).
+// Query init (a2, Alg. 1 l.2) inside the persistent kernel for the level-log paths (direction-
+// optimising BFS: MODE 0, SSSP: MODE 1): the output (level = -1 / dist = UINT32_MAX), parents, the
+// visited bitmap and the three frontier bitmaps, the counters and statistics, then the source
+// seeded into level 0's log (Tiled Partitioning of its row) — two grid barriers instead of six
+// memsets and a seed launch per call.
+template <int MODE>
+__device__ __forceinline__ void query_init(const TravArgs &a, int *overflow) {
+  Ctl *ctl = a.ctl;
+  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long nth = (long long)gridDim.x * blockDim.x;
+  const long long n4 = a.n >> 2;
+  int4 *out4 = MODE == 0 ? reinterpret_cast<int4 *>(a.level) : reinterpret_cast<int4 *>(a.dist);
+  for (long long i = tid; i < n4; i += nth) {
+    out4[i] = make_int4(-1, -1, -1, -1);
+    if (MODE == 0 && a.parent) reinterpret_cast<int4 *>(a.parent)[i] = make_int4(-1, -1, -1, -1);
+  }
+  for (long long i = 4 * n4 + tid; i < a.n; i += nth) {
+    if (MODE == 0) a.level[i] = -1;
+    else a.dist[i] = 0xffffffffu;
+    if (MODE == 0 && a.parent) a.parent[i] = -1;
+  }
+  const long long words = ((a.n + 31) >> 5) + 8;
+  for (long long i = tid; i < words; i += nth) {
+    a.visited[i] = 0u;
+    a.fb[0][i] = 0u;
+    a.fb[1][i] = 0u;
+    a.fb[2][i] = 0u;
+  }
+  if (blockIdx.x == 0) {
+    constexpr int nctr = sizeof(CounterSet) / sizeof(PaddedCounter);
+    for (int i = threadIdx.x; i < 3 * nctr; i += blockDim.x) reinterpret_cast<PaddedCounter *>(ctl->set)[i].v = 0ull;
+    for (int i = threadIdx.x; i < 16; i += blockDim.x) ctl->prof[i] = 0ull;
+    if (threadIdx.x == 0) {
+      ctl->tot_push_expanded = ctl->tot_push_arcs = ctl->tot_push_disc = 0;
+      ctl->tot_pull_scanned = ctl->tot_pull_inspected = ctl->tot_pull_disc = 0;
+      ctl->tot_arcs_reached = ctl->tot_improved = ctl->tail_levels = 0;
+      ctl->levels = ctl->push_levels = ctl->pull_levels = ctl->status = 0;
+      ctl->tail_state = ctl->tail_resume = 0;
+      ctl->rec[0].t_work = ctl->rec[0].t_mid = 0;
+      if (overflow) overflow[0] = 0;
+    }
+  }
+  grid_barrier(&ctl->bar);
+  if (blockIdx.x == 0 && threadIdx.x < 32) {   // seed the source's row into level 0's log (one warp)
+    const int src = a.src;
+    const bool act = threadIdx.x == 0;
+    long long b = 0, e = 0;
+    if (act) {
+      b = a.off[src];
+      e = a.off[src + 1];
+      ctl->tot_arcs_reached = (unsigned long long)(e - b);   // the source's own arcs (R1)
+      a.visited[src >> 5] = 1u << (src & 31);
+      a.fb[0][src >> 5] = 1u << (src & 31);
+      if (MODE == 0) a.level[src] = 0;
+      else a.dist[src] = 0u;
+    }
+    enqueue_warp(act, src, b, e, a.L, a.q[0], &ctl->set[0]);
+  }
+  grid_barrier(&ctl->bar);
+}
+
 template <int VEC, int HT>
 __device__ __forceinline__ void bfs_body(const TravArgs &a, WarpScratch *wsm, typename BfsPushT<HT>::Src (*fsrc)[32],
                                          uint8_t *ht) {
   const int warp = threadIdx.x >> 5;
   Ctl *ctl = a.ctl;
-  double mU = (double)a.m - (double)ldcg(&ctl->set[0].arcsF.v);
   if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t0_ns = globaltimer();
+  query_init<0>(a, nullptr);
+  double mU = (double)a.m - (double)ldcg(&ctl->set[0].arcsF.v);
   int dir = 0;
   unsigned long long prev_nF = 1;
   const long long nwords = (a.n + 31) >> 5;
@@ -633,6 +695,7 @@ __device__ __forceinline__ void bfs_body(const TravArgs &a, WarpScratch *wsm, ty
     CounterSet *nxt = &ctl->set[(L + 1) % 3];
     __syncthreads();   // block 0: record_level(L-1) finished before set (L+2)%3 is zeroed
     zero_counterset(&ctl->set[(L + 2) % 3]);
+    if (blockIdx.x == 0 && threadIdx.x == 0 && L + 1 < kMaxRec) ctl->rec[L + 1].t_work = ctl->rec[L + 1].t_mid = 0;
     uint32_t *fbc = a.fb[L % 3], *fbn = a.fb[(L + 1) % 3];
     if (a.do_enabled) clear_words(a.fb[(L + 2) % 3], nwords);
     if (dir == 0) {
@@ -1262,11 +1325,13 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
     wsm[warp].ndisc = 0;
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t0_ns = globaltimer();
+  query_init<1>(a, overflow);
   for (int L = 0;; ++L) {
     CounterSet *cur = &ctl->set[L % 3];
     CounterSet *nxt = &ctl->set[(L + 1) % 3];
     __syncthreads();
     zero_counterset(&ctl->set[(L + 2) % 3]);
+    if (blockIdx.x == 0 && threadIdx.x == 0 && L + 1 < kMaxRec) ctl->rec[L + 1].t_work = ctl->rec[L + 1].t_mid = 0;
     clear_words(a.fb[(L + 2) % 3], nwords);
     SsspPush f;
     f.dist = a.dist;
@@ -1292,30 +1357,6 @@ __global__ void __launch_bounds__(kBlock, 4) k_sssp(const __grid_constant__ Trav
 }
 
 // Seed the level-0 log with the source (one warp).
-__global__ void k_seed(TravArgs a, int src, int mode /*0 bfs, 1 sssp, 2 bfs with fused tiling*/) {
-  const bool act = threadIdx.x == 0;
-  if (mode == 2) {   // level 0's frontier list = {src}
-    if (act) {
-      a.visited[src >> 5] |= 1u << (src & 31);
-      a.level[src] = 0;
-      a.fl[0][0] = src;
-      a.ctl->set[0].flc.v = 1ull;
-      a.ctl->set[0].nF.v = 1ull;
-    }
-    return;
-  }
-  long long b = 0, e = 0;
-  if (act) {
-    b = a.off[src];
-    e = a.off[src + 1];
-    a.ctl->tot_arcs_reached += (unsigned long long)(e - b);   // the source's own arcs (R1)
-    a.visited[src >> 5] |= 1u << (src & 31);
-    a.fb[0][src >> 5] |= 1u << (src & 31);
-    if (mode == 0) a.level[src] = 0;
-    else a.dist[src] = 0u;
-  }
-  enqueue_warp(act, src, b, e, a.L, a.q[0], &a.ctl->set[0]);
-}
 
 // SSSP overflow resolution: a finite distance >= UINT32_MAX exists iff some arc leaves a reached
 // vertex towards an unreached one.
@@ -1461,6 +1502,7 @@ void free_traversal_state(sage_graph *g) {
   dfree(g, t.level);
   dfree(g, t.parent);
   dfree(g, t.dist);
+  if (t.ev_caller) cudaEventDestroy(t.ev_caller);
   dfree(g, t.visited);
   for (int i = 0; i < 3; ++i) dfree(g, t.fb[i]);
   free_queues(g, &t.q[0]);
@@ -1684,6 +1726,22 @@ static bool is_own_device_ptr(const sage_graph *g, const void *p) {
   return at.type == cudaMemoryTypeDevice && at.device == g->device;
 }
 
+// Outputs written in place into caller device buffers: on the library's own (non-blocking) stream
+// the writes must follow the caller's earlier work on the legacy default stream (e.g. a torch
+// fill of the same buffer); with a caller stream they are ordered by that stream already.
+static void order_after_caller(sage_graph *g) {
+  if (!g->own_stream) return;
+  TraversalState &t = g->ts;
+  if (!t.ev_caller && cudaEventCreateWithFlags(&t.ev_caller, cudaEventDisableTiming) != cudaSuccess) {
+    cudaGetLastError();
+    t.ev_caller = nullptr;
+    cudaStreamSynchronize(cudaStreamLegacy);   // fallback: order by a host wait
+    return;
+  }
+  cudaEventRecord(t.ev_caller, cudaStreamLegacy);
+  cudaStreamWaitEvent(g->stream, t.ev_caller, 0);
+}
+
 static sage_status check_common(sage_graph *g, int32_t source, const void *out) {
   if (!g || !out) {
     set_error("null argument");
@@ -1734,17 +1792,9 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
   // translation is needed, the kernel initialises and fills them directly (no output copy)
   const bool direct_lv = !g->reordered && !g->online && is_own_device_ptr(g, level_out);
   const bool direct_par = parent_out && !g->reordered && is_own_device_ptr(g, parent_out);
+  if (direct_lv || direct_par) order_after_caller(g);
   cudaEvent_t e0 = t.ev[0], e1 = t.ev[1], e2 = t.ev[2];
   cudaEventRecord(e0, g->stream);
-  const size_t words = (size_t)((g->n + 31) / 32 + 8);
-  if (!fused) {   // (the fused kernel initialises its query state itself)
-    cudaMemsetAsync(direct_lv ? level_out : t.level, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
-    if (parent_out)
-      cudaMemsetAsync(direct_par ? parent_out : t.parent, 0xff, sizeof(int32_t) * (size_t)g->n_local, g->stream);
-    cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
-    for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
-    cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);
-  }
   TravArgs a = make_args(g);
   a.parent = parent_out ? t.parent : nullptr;
   if (direct_lv) a.level = level_out;
@@ -1770,7 +1820,6 @@ extern "C" sage_status sage_bfs_ex(sage_graph *g, int32_t source, int32_t *level
     a.fl[0] = t.flist;
     a.fl[1] = t.flist2;
   }
-  if (!fused) k_seed<<<1, 32, 0, g->stream>>>(a, src, 0);
   cudaEventRecord(e1, g->stream);
   if (fused) {
     const int ht = hub_mode(g);
@@ -1857,18 +1906,14 @@ extern "C" sage_status sage_sssp(sage_graph *g, int32_t source, uint32_t *dist_o
   cudaEventCreate(&e1);
   cudaEventCreate(&e2);
   cudaEventRecord(e0, g->stream);
-  const size_t words = (size_t)((g->n + 31) / 32 + 8);
-  cudaMemsetAsync(ovf, 0, sizeof(int) * 2, g->stream);
   // distances written in place when the caller's buffer is device memory of this GPU (no copy)
   const bool direct = !g->reordered && is_own_device_ptr(g, dist_out);
   uint32_t *dd = direct ? dist_out : t.dist;
-  cudaMemsetAsync(dd, 0xff, sizeof(uint32_t) * (size_t)g->n_local, g->stream);
-  cudaMemsetAsync(t.visited, 0, sizeof(uint32_t) * words, g->stream);
-  for (int i = 0; i < 3; ++i) cudaMemsetAsync(t.fb[i], 0, sizeof(uint32_t) * words, g->stream);
-  cudaMemsetAsync(t.ctl, 0, sizeof(Ctl), g->stream);
+  if (direct) order_after_caller(g);
+  // dist, bitmaps, counters and the seed: query_init<1> inside the kernel
   TravArgs a = make_args(g);
   a.dist = dd;
-  k_seed<<<1, 32, 0, g->stream>>>(a, src, 1);
+  a.src = src;
   cudaEventRecord(e1, g->stream);
   const void *fn = g->vec == 4 ? (const void *)k_sssp<4> : (const void *)k_sssp<1>;
   const int grid = coop_grid(g, fn, &g->grid_sssp, kBlock, 0);

@@ -97,6 +97,7 @@ struct Ctl {                             // control block of one query (device m
   GridBar bar;                           // grid barrier of the persistent kernel
   unsigned long long prof[16];           // SAGE_PROF builds: per-phase cycle sums
   int tail_state;                        // tail mode: 1 = traversal finished, 2 = resume grid mode
+  int tail_n;                            // fused tail entry: vertices of the compacted list
   int tail_resume;                       // tail mode: level at which the grid resumes
   unsigned long long tail_levels;        // levels run in tail mode (diagnostic)
   LevelRec rec[kMaxRec];

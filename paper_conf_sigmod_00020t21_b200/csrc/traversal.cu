@@ -404,10 +404,10 @@ __device__ void tail_run(const TravArgs &a, int Lstart, TailSmem &ts) {
   const int tid = threadIdx.x, lane = (int)lane_id(), warp = tid >> 5;
   int nf = 0;
   if constexpr (FUSED) {
-    // ---- the frontier of level Lstart is its list (each vertex once; -1 = empty slot)
-    const CounterSet *cs = &ctl->set[Lstart % 3];
-    const int *fl = a.fl[Lstart & 1];
-    const long long fc = (long long)ldcg(&cs->flc.v);
+    // ---- the frontier of level Lstart: its list, compacted by the whole grid before the entry
+    //      (bfs_body_fused) into the other list buffer, tail_n entries
+    const int *fl = a.fl[(Lstart + 1) & 1];
+    const long long fc = (long long)ldcg(&ctl->tail_n);
     if (tid == 0) ts.nnext = 0;
     __syncthreads();
     for (long long i = tid; i < fc; i += blockDim.x) {   // order is free: compact with a counter
@@ -1152,6 +1152,7 @@ __device__ __forceinline__ void record_level_fused(Ctl *ctl, int L, const Counte
 }
 
 // Push-only BFS level loop with the fused runtime tiling.
+constexpr long long kTailCompactGrid = 2048;   // list slots above which the grid compacts it
 constexpr unsigned long long kHubReloadMinChanges = 256;   // reload the CTA's hub table after such levels
 // Profiling builds only (tools/level_isolate.sh): the fused kernel stops after level L, so that the
 // counter difference of two builds (L and L-1) is level L alone.  Default -1 = off (dead code).
@@ -1219,7 +1220,10 @@ __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *w
     CounterSet *nxt = &ctl->set[(L + 1) % 3];
     __syncthreads();   // block 0: record of L-1 finished before set (L+2)%3 is zeroed
     if (L > 0) zero_counterset(&ctl->set[(L + 2) % 3]);
-    if (blockIdx.x == 0 && threadIdx.x == 0 && L + 1 < kMaxRec) ctl->rec[L + 1].t_work = ctl->rec[L + 1].t_mid = 0;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      if (L + 1 < kMaxRec) ctl->rec[L + 1].t_work = ctl->rec[L + 1].t_mid = 0;
+      ctl->tail_n = 0;   // (read after this level's barriers)
+    }
     BfsPushT<HT> f;
     f.keep = policy_evict_last();
     f.visited = a.visited;
@@ -1264,8 +1268,34 @@ __device__ __forceinline__ void bfs_body_fused(const TravArgs &a, WarpScratch *w
       if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = 1;
       break;
     }
-    // small frontier: block 0 runs the next levels alone (it hands back when arcs(F) is large)
+    // small frontier: block 0 runs the next levels alone (it hands back when arcs(F) is large).
+    // Level L+1's list is sparse (a 256-slot chunk per warp that discovered anything: up to ~10^5
+    // slots on C1 for a few hundred vertices), so the whole grid compacts it first — block 0
+    // alone scanning it cost up to 130 us.
     if (nF <= kTailV) {
+      {
+        const long long fc = (long long)ldcg(&nxt->flc.v);
+        // long lists: the whole grid compacts them (one more grid barrier); short ones: block 0
+        const bool grid_wide = fc > kTailCompactGrid;
+        const int *src = a.fl[(L + 1) & 1];
+        int *dst = a.fl[L & 1];
+        const long long tid = grid_wide ? (long long)blockIdx.x * blockDim.x + threadIdx.x : (long long)threadIdx.x;
+        const long long nth = grid_wide ? (long long)gridDim.x * blockDim.x : (long long)blockDim.x;
+        const unsigned lane = lane_id();
+        for (long long base = tid - lane; (grid_wide || blockIdx.x == 0) && base < fc; base += nth) {
+          const long long i = base + lane;
+          const int u = i < fc ? ldcg(src + i) : -1;
+          const unsigned m = __ballot_sync(FULL, u >= 0);
+          if (m) {
+            int pos = 0;
+            if (lane == 0) pos = atomicAdd(&ctl->tail_n, __popc(m));
+            pos = __shfl_sync(FULL, pos, 0);
+            if (u >= 0) dst[pos + __popc(m & lanemask_lt())] = u;
+          }
+        }
+        if (grid_wide) grid_barrier(&ctl->bar);
+        else __syncthreads();
+      }
       if (blockIdx.x == 0) {
         __syncthreads();
         if (threadIdx.x == 0) ctl->tail_state = 0;

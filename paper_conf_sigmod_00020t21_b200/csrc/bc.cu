@@ -8,8 +8,9 @@
 // Backward (Alg. 1 l.19-24): levels in decreasing order; the segment of level L is classified
 // into tiles again (Tiled Partitioning of the revisited rows) and consumed by the stealing
 // consumer with a gather filter: a tile of row u sums (1 + delta[v]) / sigma[v] over members v on
-// level L+1, and the lane group adds sigma[u] * sum to delta[u] with one fp64 atomic — the same
-// value as the paper's per-arc atomicAdd(delta[fr], sigma[fr]/sigma[nb] * (delta[nb] + 1)).
+// level L+1 (precomputed once per vertex into sigma[v] when its level is done), and the lane group
+// adds sigma[u] * sum to delta[u] with one fp64 atomic — the same value as the paper's per-arc
+// atomicAdd(delta[fr], sigma[fr]/sigma[nb] * (delta[nb] + 1)).
 // bc[v] += delta[v] for v != source.
 #include <cuda_runtime.h>
 #include <string.h>
@@ -106,7 +107,7 @@ struct BcBwd {
     for (int j = 0; j < N; ++j) {
       in[j] = false;
       if (valid && ldcg(level + v[j]) == child_level)
-        acc += (1.0 + ldcg(delta + v[j])) / ldcg(sigma + v[j]);   // Alg. 1 l.21-23
+        acc += ldcg(sigma + v[j]);   // = (1 + delta[v]) / sigma[v], Alg. 1 l.21-23 (k_bc_bwd)
     }
     for (int o = lpt >> 1; o > 0; o >>= 1) acc += __shfl_xor_sync(FULL, acc, o);
     if (valid && (lane_id() & (lpt - 1)) == 0 && acc != 0.0) red_add_f64(delta + s.u, ldcg(sigma + s.u) * acc);
@@ -183,6 +184,18 @@ __global__ void __launch_bounds__(kBlock, 4) k_bc_bwd(const __grid_constant__ Bc
       const long long i = base + lane;
       const bool act = i < e;
       enqueue_ids(act, act ? ldcg(a.order + i) : 0, a.off, a.L, qk, cs);
+    }
+    // the children's coefficients, once per vertex: sigma[w] <- (1 + delta[w]) / sigma[w] for w
+    // on level L+1 (their delta is final; their sigma is not read again), so the gather below
+    // reads one fp64 per child arc instead of two and divides once per vertex, not per arc
+    {
+      const long long cb = a.seg[L + 1], ce = a.seg[L + 2];
+      const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+      const long long nth = (long long)gridDim.x * blockDim.x;
+      for (long long i = cb + tid; i < ce; i += nth) {
+        const int w = ldcg(a.order + i);
+        a.sigma[w] = (1.0 + ldcg(a.delta + w)) / ldcg(a.sigma + w);
+      }
     }
     grid_barrier(&ctl->bar);
     BcBwd f;
